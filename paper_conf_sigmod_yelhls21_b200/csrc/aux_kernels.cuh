@@ -1,0 +1,91 @@
+// aux_kernels.cuh -- setup / frontier / histogram kernels (non-MFL steps).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "glp_internal.cuh"
+
+namespace glp {
+
+// CSR validation [P:97]: off[0]==0, off non-decreasing, off[nl]==nnz, col in [0,n).
+__global__ void k_validate_off(const int64_t* __restrict__ off, int64_t nl, int64_t nnz, int* bad) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= nl; v += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t x = off[v];
+    if (v == 0 && x != 0) atomicOr(bad, 1);
+    if (v == nl && x != nnz) atomicOr(bad, 2);
+    if (v < nl && off[v + 1] < x) atomicOr(bad, 4);
+  }
+}
+__global__ void k_validate_col(const int32_t* __restrict__ col, int64_t nnz, int64_t n, int* bad) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t u = col[e];
+    if (u < 0 || (int64_t)u >= n) atomicOr(bad, 8);
+  }
+}
+
+// PickLabel [P:99, P:109]: L[v] = v (CLASSIC, LLP) or UNLABELED (SEEDED, R12).
+__global__ void k_init_labels(int32_t* __restrict__ L0, int32_t* __restrict__ L1, int64_t n, int seeded) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t x = seeded ? -1 : (int32_t)v;
+    L0[v] = x;
+    L1[v] = x;
+  }
+}
+
+// Seeds carry their own id; owned seeds are marked and recorded as "changed at
+// t = 0" so that the first frontier is N(S) (exact: every other vertex has no
+// labelled neighbour and keeps -1, R5).
+__global__ void k_init_seeds(const int32_t* __restrict__ seeds, int64_t ns, int32_t* __restrict__ L0,
+                             int32_t* __restrict__ L1, uint8_t* __restrict__ is_seed, int2* __restrict__ so,
+                             int64_t vb, int64_t ve) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < ns; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t s = seeds[i];
+    L0[s] = s;
+    L1[s] = s;
+    if (s >= vb && s < ve) {
+      is_seed[s - vb] = 1;
+      so[s - vb] = make_int2(0, s);
+    }
+  }
+}
+
+// Frontier push: for every owned vertex changed at iteration t (so.x == t),
+// mark itself and its neighbours (global ids) active for t+1 (marking
+// the changed vertex itself keeps the unconditional-write invariant).  One
+// warp scans 32 stamps, then walks each changed vertex's row cooperatively.
+__global__ void k_push(const int64_t* __restrict__ off, const int32_t* __restrict__ col,
+                       const int2* __restrict__ so, int64_t nl, int64_t vb, int32_t t,
+                       uint8_t* __restrict__ flag) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t base = gw * 32; base < nl; base += nw * 32) {
+    const int64_t v = base + lane;
+    const bool ch = v < nl && so[v].x == t;
+    unsigned m = __ballot_sync(0xffffffffu, ch);
+    while (m) {
+      const int j = __ffs(m) - 1;
+      m &= m - 1;
+      const int64_t u = base + j;
+      if (lane == 0) flag[vb + u] = 1;
+      const int64_t e0 = off[u], e1 = off[u + 1];
+      for (int64_t e = e0 + lane; e < e1; e += 32) flag[col[e]] = 1;  // global ids
+    }
+  }
+}
+
+// LLP: V[l] = #{w : L[w] = l} [P:119].
+__global__ void k_hist(const int32_t* __restrict__ L, int64_t n, int32_t* __restrict__ V) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t l = L[v];
+    if (l >= 0) atomicAdd(V + l, 1);
+  }
+}
+
+// L2 flush helper for benchmarks (writes a buffer larger than L2).
+__global__ void k_fill(uint4* __restrict__ p, int64_t n16, unsigned x) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n16; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] = make_uint4(x, x, x, x);
+}
+
+}  // namespace glp

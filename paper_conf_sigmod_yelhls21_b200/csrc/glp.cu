@@ -1,0 +1,667 @@
+// glp.cu -- host runtime and C ABI of libglp.so (see include/glp.h).
+//
+// Per LP iteration t, all on the graph's stream:
+//   1. reset per-bin counters                                  (memset 256 B)
+//   2. mfl_huge, mfl_high, mfl_mid, mfl_low  R = L_{t-1} -> W = L_t
+//   3. [P > 1] ncclAllGather of the owned label slice, counters all-reduce
+//   4. read the counters (changed, d2, sum of changed degrees) -> stop rule R8
+//   5. frontier decision: dense when sum_{changed} deg > nnz / dense_divisor,
+//      else k_push marks N(v) + v for changed v (exact for CLASSIC/SEEDED, R9)
+//   6. LLP: rebuild the label histogram V from L_t               [P:119]
+//   7. swap R/W
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <string>
+#include <vector>
+
+#include "aux_kernels.cuh"
+#include "glp_internal.cuh"
+#include "mfl_kernels.cuh"
+#include "nccl_dyn.cuh"
+
+using namespace glp;
+
+namespace {
+
+thread_local std::string g_last_error = "";
+
+[[noreturn]] void fail(glp_status st, const std::string& m) { throw Err{st, m}; }
+
+#define CK(x)                                                                              \
+  do {                                                                                     \
+    cudaError_t e_ = (x);                                                                  \
+    if (e_ != cudaSuccess) {                                                               \
+      if (e_ == cudaErrorMemoryAllocation)                                                 \
+        fail(GLP_ERR_OUT_OF_MEMORY, std::string(#x) + ": " + cudaGetErrorString(e_));      \
+      fail(GLP_ERR_CUDA, std::string(#x) + ": " + cudaGetErrorName(e_) + " " + cudaGetErrorString(e_)); \
+    }                                                                                      \
+  } while (0)
+
+template <class T>
+T* dalloc(glp_graph* g, size_t count) {
+  void* p = nullptr;
+  size_t bytes = std::max<size_t>(count * sizeof(T), 16);
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    fail(GLP_ERR_OUT_OF_MEMORY, "cudaMalloc(" + std::to_string(bytes) + " B) failed: " + cudaGetErrorString(e));
+  }
+  g->allocs.push_back(p);
+  return (T*)p;
+}
+
+template <class T>
+T* upload(glp_graph* g, const std::vector<T>& h) {
+  T* d = dalloc<T>(g, h.size());
+  if (!h.empty()) CK(cudaMemcpyAsync(d, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice, g->stream));
+  return d;
+}
+
+int grid_for(int sms, const void* fn, int block, size_t smem) {
+  int per_sm = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, block, smem));
+  return std::max(1, per_sm) * sms;
+}
+
+glp_params default_params() {
+  glp_params p;
+  memset(&p, 0, sizeof(p));
+  p.struct_size = sizeof(glp_params);
+  p.gamma = 0.0;
+  p.frontier = -1;
+  p.stop_on_2cycle = 1;
+  p.validate = 1;
+  p.profile = 0;
+  p.dense_divisor = 4;
+  return p;
+}
+
+glp_params get_params(const glp_params* p) {
+  if (!p) return default_params();
+  if (p->struct_size != sizeof(glp_params))
+    fail(GLP_ERR_INVALID_ARGUMENT, "glp_params.struct_size mismatch (got " + std::to_string(p->struct_size) +
+                                       ", expected " + std::to_string(sizeof(glp_params)) + ")");
+  glp_params q = *p;
+  if (q.dense_divisor <= 0) q.dense_divisor = 4;
+  return q;
+}
+
+template <class F>
+glp_status guard(F f) {
+  try {
+    f();
+    return GLP_OK;
+  } catch (const Err& e) {
+    g_last_error = e.msg;
+    return e.st;
+  } catch (const std::bad_alloc&) {
+    g_last_error = "host allocation failed";
+    return GLP_ERR_OUT_OF_MEMORY;
+  } catch (...) {
+    g_last_error = "unknown internal error";
+    return GLP_ERR_CUDA;
+  }
+}
+
+void free_graph(glp_graph* g) {
+  if (!g) return;
+  if (g->device >= 0) cudaSetDevice(g->device);
+  if (g->stream) cudaStreamSynchronize(g->stream);
+  for (void* p : g->allocs) cudaFree(p);
+  g->allocs.clear();
+  if (g->h_cnt) cudaFreeHost(g->h_cnt);
+  if (g->ev_a) cudaEventDestroy(g->ev_a);
+  if (g->ev_b) cudaEventDestroy(g->ev_b);
+  for (auto& e : g->ev_pool) cudaEventDestroy(e);
+  nccl_destroy(g);
+  if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
+  delete g;
+}
+
+// ---------------------------------------------------------------- binning
+// Degree bins and low-degree warp chunks (host, once per graph).
+void build_bins(glp_graph* g, const int64_t* off_h) {
+  std::vector<int32_t> low, mid, high, huge, chunk;
+  for (int b = 0; b < NBINS; ++b) g->bin_verts[b] = g->bin_arcs[b] = 0;
+  int64_t maxd = 0;
+  for (int64_t v = 0; v < g->nl; ++v) {
+    const int64_t d = off_h[v + 1] - off_h[v];
+    maxd = std::max(maxd, d);
+    int b;
+    if (d == 0) b = BIN_ISO;
+    else if (d <= kLowMax) { b = BIN_LOW; low.push_back((int32_t)v); }
+    else if (d <= kMidMax) { b = BIN_MID; mid.push_back((int32_t)v); }
+    else if (d <= kHighMax) { b = BIN_HIGH; high.push_back((int32_t)v); }
+    else { b = BIN_HUGE; huge.push_back((int32_t)v); }
+    g->bin_verts[b] += 1;
+    g->bin_arcs[b] += d;
+  }
+  g->max_deg = maxd;
+  // greedy chunks: maximal runs of the low list with sum of degrees <= 32
+  chunk.push_back(0);
+  int sum = 0;
+  for (size_t k = 0; k < low.size(); ++k) {
+    const int d = (int)(off_h[low[k] + 1] - off_h[low[k]]);
+    if (sum + d > 32) {
+      chunk.push_back((int32_t)k);
+      sum = 0;
+    }
+    sum += d;
+  }
+  if (!low.empty()) chunk.push_back((int32_t)low.size());
+  // largest first: the block-per-vertex bins start the long rows early
+  auto by_deg = [&](int32_t a, int32_t b) {
+    const int64_t da = off_h[a + 1] - off_h[a], db = off_h[b + 1] - off_h[b];
+    return da != db ? da > db : a < b;
+  };
+  std::sort(huge.begin(), huge.end(), by_deg);
+  std::sort(high.begin(), high.end(), by_deg);
+  g->n_low = (int32_t)low.size();
+  g->n_chunks = low.empty() ? 0 : (int32_t)chunk.size() - 1;
+  g->n_mid = (int32_t)mid.size();
+  g->n_high = (int32_t)high.size();
+  g->n_huge = (int32_t)huge.size();
+  g->low_list = upload(g, low);
+  g->low_chunk = upload(g, chunk);
+  g->mid_list = upload(g, mid);
+  g->high_list = upload(g, high);
+  g->huge_list = upload(g, huge);
+}
+
+void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm, glp_graph** out) {
+  if (!out) fail(GLP_ERR_INVALID_ARGUMENT, "out is NULL");
+  *out = nullptr;
+  if (!csr) fail(GLP_ERR_INVALID_ARGUMENT, "csr is NULL");
+  glp_params p = get_params(prm);
+  const int64_t n = csr->n_global;
+  if (n < 0 || n >= (int64_t)INT32_MAX) fail(GLP_ERR_INVALID_ARGUMENT, "n_global out of range [0, 2^31-1)");
+  if (csr->v_begin < 0 || csr->v_end < csr->v_begin || csr->v_end > n)
+    fail(GLP_ERR_INVALID_ARGUMENT, "owned row range [v_begin, v_end) invalid");
+  if (csr->nnz_local < 0) fail(GLP_ERR_INVALID_ARGUMENT, "nnz_local < 0");
+  if (!csr->row_offsets) fail(GLP_ERR_INVALID_ARGUMENT, "row_offsets is NULL");
+  if (csr->nnz_local > 0 && !csr->col_idx) fail(GLP_ERR_INVALID_ARGUMENT, "col_idx is NULL");
+  int rank = 0, nranks = 1;
+  if (dist) {
+    rank = dist->rank;
+    nranks = dist->nranks;
+    if (nranks < 1 || rank < 0 || rank >= nranks) fail(GLP_ERR_INVALID_ARGUMENT, "bad rank/nranks");
+    if (nranks > 1 && !dist->nccl_unique_id) fail(GLP_ERR_INVALID_ARGUMENT, "nccl_unique_id required for nranks > 1");
+  }
+  if (nranks == 1 && (csr->v_begin != 0 || csr->v_end != n))
+    fail(GLP_ERR_INVALID_ARGUMENT, "single GPU: owned range must be [0, n_global)");
+
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    fail(GLP_ERR_UNSUPPORTED, "no CUDA device visible (libglp has no CPU fallback)");
+  }
+  int dev = 0;
+  if (dist) dev = dist->device;
+  else CK(cudaGetDevice(&dev));
+  if (dev < 0 || dev >= ndev) fail(GLP_ERR_INVALID_ARGUMENT, "device ordinal out of range");
+  CK(cudaSetDevice(dev));
+  cudaDeviceProp prop;
+  CK(cudaGetDeviceProperties(&prop, dev));
+  if (prop.major != 10)
+    fail(GLP_ERR_UNSUPPORTED, std::string("libglp is built for sm_100a (B200); device is ") + prop.name);
+
+  glp_graph* g = new glp_graph();
+  try {
+    g->device = dev;
+    g->rank = rank;
+    g->nranks = nranks;
+    if (dist && dist->cuda_stream) {
+      g->stream = (cudaStream_t)dist->cuda_stream;
+    } else {
+      CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
+      g->own_stream = true;
+    }
+    g->n = n;
+    g->vb = csr->v_begin;
+    g->ve = csr->v_end;
+    g->nl = g->ve - g->vb;
+    g->nnz = csr->nnz_local;
+    g->symmetric = csr->symmetric ? 1 : 0;
+    if (g->nnz >= ((int64_t)1 << 40)) fail(GLP_ERR_INVALID_ARGUMENT, "nnz_local too large");
+
+    std::vector<int64_t> off_h;
+    const int64_t* off_host = nullptr;
+    if (csr->on_device) {
+      g->off = csr->row_offsets;
+      g->col = csr->col_idx;
+      off_h.resize(g->nl + 1);
+      CK(cudaMemcpyAsync(off_h.data(), g->off, (g->nl + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, g->stream));
+      CK(cudaStreamSynchronize(g->stream));
+      off_host = off_h.data();
+    } else {
+      int64_t* doff = dalloc<int64_t>(g, g->nl + 1);
+      int32_t* dcol = dalloc<int32_t>(g, g->nnz);
+      CK(cudaMemcpyAsync(doff, csr->row_offsets, (g->nl + 1) * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
+      if (g->nnz)
+        CK(cudaMemcpyAsync(dcol, csr->col_idx, g->nnz * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
+      g->off = doff;
+      g->col = dcol;
+      g->own_csr = true;
+      off_host = csr->row_offsets;
+    }
+    // host-side structural checks on the offsets (cheap, always on)
+    if (off_host[0] != 0 || off_host[g->nl] != g->nnz)
+      fail(GLP_ERR_INVALID_GRAPH, "row_offsets[0] must be 0 and row_offsets[last] == nnz_local");
+    if (p.validate) {
+      for (int64_t v = 0; v < g->nl; ++v)
+        if (off_host[v + 1] < off_host[v]) fail(GLP_ERR_INVALID_GRAPH, "row_offsets not non-decreasing");
+      int* dbad = dalloc<int>(g, 1);
+      CK(cudaMemsetAsync(dbad, 0, sizeof(int), g->stream));
+      if (g->nnz) k_validate_col<<<prop.multiProcessorCount * 4, 256, 0, g->stream>>>(g->col, g->nnz, g->n, dbad);
+      CK(cudaGetLastError());
+      int bad = 0;
+      CK(cudaMemcpyAsync(&bad, dbad, sizeof(int), cudaMemcpyDeviceToHost, g->stream));
+      CK(cudaStreamSynchronize(g->stream));
+      if (bad) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
+    }
+    build_bins(g, off_host);
+
+    // labels: replicated full arrays, padded to a multiple of nranks for the
+    // in-place all-gather
+    const int64_t npad = ((n + nranks - 1) / nranks) * nranks;
+    g->npad = npad;
+    g->L[0] = dalloc<int32_t>(g, npad);
+    g->L[1] = dalloc<int32_t>(g, npad);
+    g->so = dalloc<int2>(g, g->nl);
+    g->V = dalloc<int32_t>(g, std::max<int64_t>(n, 1));
+    g->is_seed = dalloc<uint8_t>(g, g->nl);
+    g->flag[0] = dalloc<uint8_t>(g, npad);
+    g->flag[1] = dalloc<uint8_t>(g, npad);
+    CK(cudaMemsetAsync(g->flag[0], 0, std::max<int64_t>(npad, 1), g->stream));
+    CK(cudaMemsetAsync(g->flag[1], 0, std::max<int64_t>(npad, 1), g->stream));
+    g->d_cnt = dalloc<Counters>(g, 4);
+    CK(cudaMallocHost(&g->h_cnt, 4 * sizeof(Counters)));
+    CK(cudaEventCreate(&g->ev_a));
+    CK(cudaEventCreate(&g->ev_b));
+
+    const int sms = prop.multiProcessorCount;
+    g->sms = sms;
+    CK(cudaFuncSetAttribute(mfl_high<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHighSlots * 8));
+    CK(cudaFuncSetAttribute(mfl_high<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHighSlots * 8));
+    CK(cudaFuncSetAttribute(mfl_high<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHighSlots * 8));
+    CK(cudaFuncSetAttribute(mfl_huge<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHugeSlots * 8));
+    CK(cudaFuncSetAttribute(mfl_huge<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHugeSlots * 8));
+    CK(cudaFuncSetAttribute(mfl_huge<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHugeSlots * 8));
+    g->grid_low = grid_for(sms, (const void*)mfl_low<V_CLASSIC>, kLowBlock, 0);
+    g->grid_mid = grid_for(sms, (const void*)mfl_mid<V_CLASSIC>, kMidBlock, 0);
+    g->grid_high = grid_for(sms, (const void*)mfl_high<V_LLP>, kHighBlock, kHighSlots * 8);
+    g->grid_huge = grid_for(sms, (const void*)mfl_huge<V_LLP>, kHugeBlock, kHugeSlots * 8);
+    g->grid_aux = sms * 8;
+    if (g->n_huge > 0) {
+      g->grid_huge = std::min<int>(g->grid_huge, g->n_huge);
+      g->ght_slots = 2 * g->max_deg;
+      g->ght = dalloc<unsigned long long>(g, (size_t)g->ght_slots * g->grid_huge);
+    }
+    g->nnz_global = g->nnz;
+    if (nranks > 1) nccl_init(g, dist->nccl_unique_id);
+    CK(cudaStreamSynchronize(g->stream));
+  } catch (...) {
+    free_graph(g);
+    throw;
+  }
+  *out = g;
+}
+
+// ---------------------------------------------------------------- profiling
+struct Pending {
+  int kid;
+  cudaEvent_t a, b;
+};
+
+cudaEvent_t pool_event(glp_graph* g, size_t& used) {
+  if (used == g->ev_pool.size()) {
+    cudaEvent_t e;
+    CK(cudaEventCreate(&e));
+    g->ev_pool.push_back(e);
+  }
+  return g->ev_pool[used++];
+}
+
+const char* kKernelNames[] = {"mfl_low", "mfl_mid", "mfl_high", "mfl_huge", "push", "llp_hist", "exchange"};
+constexpr int kNumKernelNames = 7;
+
+template <class F>
+void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t& used, F f) {
+  if (!prof) {
+    f();
+    CK(cudaGetLastError());
+    return;
+  }
+  cudaEvent_t a = pool_event(g, used), b = pool_event(g, used);
+  CK(cudaEventRecord(a, g->stream));
+  f();
+  CK(cudaGetLastError());
+  CK(cudaEventRecord(b, g->stream));
+  pend.push_back({kid, a, b});
+}
+
+// ---------------------------------------------------------------- run
+template <int VAR>
+void launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, size_t& used) {
+  Counters* c = g->d_cnt;
+  if (g->n_huge) {
+    MflArgs b = a;
+    b.list = g->huge_list; b.list_len = g->n_huge; b.cnt = c + 3;
+    b.ght = g->ght; b.ght_slots = g->ght_slots;
+    timed(g, prof, 3, pend, used, [&] { mfl_huge<VAR><<<g->grid_huge, kHugeBlock, kHugeSlots * 8, g->stream>>>(b); });
+  }
+  if (g->n_high) {
+    MflArgs b = a;
+    b.list = g->high_list; b.list_len = g->n_high; b.cnt = c + 2;
+    const int grid = std::min<int>(g->grid_high, g->n_high);
+    timed(g, prof, 2, pend, used, [&] { mfl_high<VAR><<<grid, kHighBlock, kHighSlots * 8, g->stream>>>(b); });
+  }
+  if (g->n_mid) {
+    MflArgs b = a;
+    b.list = g->mid_list; b.list_len = g->n_mid; b.cnt = c + 1;
+    const int grid = std::min<int>(g->grid_mid, (g->n_mid + kMidBlock / 32 - 1) / (kMidBlock / 32));
+    timed(g, prof, 1, pend, used, [&] { mfl_mid<VAR><<<grid, kMidBlock, 0, g->stream>>>(b); });
+  }
+  if (g->n_chunks) {
+    MflArgs b = a;
+    b.list = g->low_list; b.list_len = g->n_low; b.chunk = g->low_chunk; b.n_chunks = g->n_chunks; b.cnt = c + 0;
+    const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock / 32 - 1) / (kLowBlock / 32));
+    timed(g, prof, 0, pend, used, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, g->stream>>>(b); });
+  }
+}
+
+void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_t* seeds, int64_t n_seeds,
+              const glp_params* prm, glp_run_info* info) {
+  if (!g) fail(GLP_ERR_INVALID_ARGUMENT, "graph is NULL");
+  glp_params p = get_params(prm);
+  if (variant < GLP_VARIANT_CLASSIC || variant > GLP_VARIANT_LLP) fail(GLP_ERR_INVALID_ARGUMENT, "unknown variant");
+  if (max_iters < 0) fail(GLP_ERR_INVALID_ARGUMENT, "max_iters < 0");
+  if (variant == GLP_VARIANT_LLP) {
+    if (!std::isfinite(p.gamma) || p.gamma < 0) fail(GLP_ERR_INVALID_ARGUMENT, "gamma must be finite and >= 0");
+    if (p.frontier == 1) fail(GLP_ERR_INVALID_ARGUMENT, "the frontier is not exact for LLP (frontier=1 rejected)");
+  }
+  if (variant != GLP_VARIANT_SEEDED && (seeds != nullptr || n_seeds != 0))
+    fail(GLP_ERR_INVALID_ARGUMENT, "seeds are only valid for GLP_VARIANT_SEEDED");
+  if (n_seeds < 0 || (n_seeds > 0 && !seeds)) fail(GLP_ERR_INVALID_ARGUMENT, "bad seeds/n_seeds");
+  for (int64_t i = 0; i < n_seeds; ++i)
+    if (seeds[i] < 0 || seeds[i] >= g->n) fail(GLP_ERR_INVALID_ARGUMENT, "seed id out of range");
+  if (p.frontier == 1 && !g->symmetric)
+    fail(GLP_ERR_INVALID_ARGUMENT, "frontier=1 needs a symmetric graph (glp_csr.symmetric)");
+  const bool use_frontier = variant != GLP_VARIANT_LLP && g->symmetric && p.frontier != 0;
+  const bool prof = p.profile != 0;
+
+  CK(cudaSetDevice(g->device));
+  cudaStream_t s = g->stream;
+  const int ga = g->grid_aux;
+  // PickLabel
+  k_init_labels<<<ga, 256, 0, s>>>(g->L[0], g->L[1], g->npad, variant == GLP_VARIANT_SEEDED);
+  CK(cudaGetLastError());
+  CK(cudaMemsetAsync(g->so, 0x80, std::max<int64_t>(g->nl, 1) * sizeof(int2), s));  // stamp = INT_MIN-ish
+  CK(cudaMemsetAsync(g->is_seed, 0, std::max<int64_t>(g->nl, 1), s));
+  for (int f = 0; f < 2; ++f)
+    if (!g->flag_clean[f]) {
+      CK(cudaMemsetAsync(g->flag[f], 0, std::max<int64_t>(g->npad, 1), s));
+      g->flag_clean[f] = true;
+    }
+  if (variant == GLP_VARIANT_SEEDED && n_seeds > 0) {
+    if (n_seeds > g->seeds_cap) {
+      g->d_seeds = dalloc<int32_t>(g, n_seeds);
+      g->seeds_cap = n_seeds;
+    }
+    CK(cudaMemcpyAsync(g->d_seeds, seeds, n_seeds * sizeof(int32_t), cudaMemcpyHostToDevice, s));
+    k_init_seeds<<<ga, 256, 0, s>>>(g->d_seeds, n_seeds, g->L[0], g->L[1], g->is_seed, g->so, g->vb, g->ve);
+    CK(cudaGetLastError());
+  }
+  if (variant == GLP_VARIANT_LLP) {
+    // V[l] = #{w : L_0[w] = l} = 1 for every l (L_0[v] = v)
+    CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
+    k_hist<<<ga, 256, 0, s>>>(g->L[0], g->n, g->V);
+    CK(cudaGetLastError());
+  }
+  int rb = 0;  // R = L[rb], W = L[1-rb]
+  int fb = 0;  // flags read this iteration
+  bool dense = true;
+  if (variant == GLP_VARIANT_SEEDED) {
+    // frontier of t = 1 is N(S) (+ S): push from the seeds (stamped t = 0)
+    if (use_frontier) {
+      k_push<<<ga, 256, 0, s>>>(g->off, g->col, g->so, g->nl, g->vb, 0, g->flag[fb]);
+      CK(cudaGetLastError());
+      g->flag_clean[fb] = false;
+      if (g->nranks > 1) nccl_merge_flags(g, g->flag[fb]);
+      dense = false;
+    }
+  }
+
+  g->iter_stats.clear();
+  g->kstats.assign(kNumKernelNames, KStat());
+  for (int k = 0; k < kNumKernelNames; ++k) g->kstats[k].name = kKernelNames[k];
+  std::vector<Pending> pend;
+  size_t used = 0;
+  cudaEvent_t ev_run0 = pool_event(g, used);
+  CK(cudaEventRecord(ev_run0, s));
+  // drain profiled launches (stream must be synchronised); counters attach
+  // algorithmic bytes to the MFL kernels (SURVEY §8(d) model)
+  auto drain = [&](bool with_counters) {
+    for (auto& pe : pend) {
+      float kms = 0;
+      CK(cudaEventElapsedTime(&kms, pe.a, pe.b));
+      KStat& ks = g->kstats[pe.kid];
+      ks.launches += 1;
+      ks.ms += kms;
+      if (with_counters && pe.kid < 4) {
+        const Counters& c = g->h_cnt[pe.kid];
+        ks.arcs += (double)c.arcs;
+        // 4 B/arc (col_idx) + 8 B/active vertex (row offsets) + 4 B/changed label
+        ks.bytes += 4.0 * (double)c.arcs + 8.0 * (double)c.verts + 4.0 * (double)c.changed;
+      }
+    }
+    pend.clear();
+  };
+
+  int32_t iters = 0;
+  int reason = GLP_STOP_MAX_ITERS;
+  int64_t changed_last = 0, arcs_total = 0;
+  for (int32_t t = 1; t <= max_iters; ++t) {
+    if (!pend.empty()) {  // profiled post-iteration kernels of t-1
+      CK(cudaStreamSynchronize(s));
+      drain(false);
+    }
+    used = 1;  // ev_run0 stays; everything else is recycled
+    cudaEvent_t e0 = pool_event(g, used), e1 = pool_event(g, used);
+    CK(cudaEventRecord(e0, s));
+    CK(cudaMemsetAsync(g->d_cnt, 0, 4 * sizeof(Counters), s));
+    MflArgs a;
+    memset(&a, 0, sizeof(a));
+    a.off = g->off; a.col = g->col; a.R = g->L[rb]; a.W = g->L[1 - rb]; a.so = g->so;
+    a.V = g->V; a.is_seed = g->is_seed; a.flag = g->flag[fb];
+    a.vb = g->vb; a.gamma = p.gamma; a.t = t; a.dense = dense ? 1 : 0;
+    switch (variant) {
+      case GLP_VARIANT_CLASSIC: launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
+      case GLP_VARIANT_SEEDED: launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
+      default: launch_mfl<V_LLP>(g, a, prof, pend, used); break;
+    }
+    if (g->nranks > 1) {
+      timed(g, prof, 6, pend, used, [&] { nccl_exchange(g, g->L[1 - rb]); });
+      nccl_sum_counters(g, g->d_cnt, 4 * sizeof(Counters) / sizeof(unsigned long long));
+    }
+    CK(cudaMemcpyAsync(g->h_cnt, g->d_cnt, 4 * sizeof(Counters), cudaMemcpyDeviceToHost, s));
+    CK(cudaEventRecord(e1, s));
+    CK(cudaStreamSynchronize(s));
+    Counters tot;
+    memset(&tot, 0, sizeof(tot));
+    for (int b = 0; b < 4; ++b) {
+      tot.changed += g->h_cnt[b].changed; tot.d2 += g->h_cnt[b].d2; tot.chdeg += g->h_cnt[b].chdeg;
+      tot.arcs += g->h_cnt[b].arcs; tot.verts += g->h_cnt[b].verts;
+    }
+    glp_iter_stat st;
+    memset(&st, 0, sizeof(st));
+    st.changed = (int64_t)tot.changed;
+    st.d2 = (int64_t)tot.d2;
+    st.active_vertices = (int64_t)tot.verts;
+    st.active_arcs = (int64_t)tot.arcs;
+    st.dense = dense ? 1 : 0;
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, e0, e1));
+    st.ms = ms;
+    drain(true);
+    iters = t;
+    changed_last = st.changed;
+    arcs_total += st.active_arcs;
+    // stop rule (R8): fixed point, or L_t == L_{t-2} (d2 == 0) with changes
+    bool stop = false;
+    if (st.changed == 0) { reason = GLP_STOP_FIXED_POINT; stop = true; }
+    else if (p.stop_on_2cycle && t >= 2 && st.d2 == 0) { reason = GLP_STOP_TWO_CYCLE; stop = true; }
+    // frontier of t+1: dense when the changed vertices touch > nnz/divisor arcs
+    const int nf = 1 - fb;
+    bool next_dense = true;
+    if (!stop && use_frontier)
+      next_dense = (double)tot.chdeg * (double)p.dense_divisor > (double)g->nnz_global;
+    if (!stop && !next_dense) {
+      timed(g, prof, 4, pend, used, [&] {
+        k_push<<<ga, 256, 0, s>>>(g->off, g->col, g->so, g->nl, g->vb, t, g->flag[nf]);
+        if (g->nranks > 1) nccl_merge_flags(g, g->flag[nf]);
+      });
+      g->flag_clean[nf] = false;
+    }
+    if (!dense && !g->flag_clean[fb]) {
+      CK(cudaMemsetAsync(g->flag[fb], 0, std::max<int64_t>(g->npad, 1), s));
+      g->flag_clean[fb] = true;
+    }
+    if (!stop && variant == GLP_VARIANT_LLP) {
+      timed(g, prof, 5, pend, used, [&] {
+        CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
+        k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb], g->n, g->V);
+      });
+    }
+    g->iter_stats.push_back(st);
+    rb = 1 - rb;
+    fb = nf;
+    dense = next_dense;
+    if (stop) break;
+  }
+  if (!pend.empty()) {
+    CK(cudaStreamSynchronize(s));
+    drain(false);
+  }
+  cudaEvent_t ev_run1 = pool_event(g, used);
+  CK(cudaEventRecord(ev_run1, s));
+  CK(cudaStreamSynchronize(s));
+  float run_ms = 0;
+  CK(cudaEventElapsedTime(&run_ms, ev_run0, ev_run1));
+  g->cur = rb;
+  g->has_run = true;
+  if (info) {
+    info->iterations = iters;
+    info->stop_reason = reason;
+    info->changed_last = changed_last;
+    info->arcs_processed = arcs_total;
+    info->elapsed_ms = run_ms;
+  }
+}
+
+}  // namespace
+
+// ================================================================ C ABI
+extern "C" {
+
+glp_status glp_graph_create(const glp_csr* csr, const glp_dist* dist, const glp_params* params, glp_graph** out) {
+  return guard([&] { create_impl(csr, dist, params, out); });
+}
+
+glp_status glp_run(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_t* seeds, int64_t n_seeds,
+                   const glp_params* params, glp_run_info* info) {
+  return guard([&] { run_impl(g, variant, max_iters, seeds, n_seeds, params, info); });
+}
+
+glp_status glp_labels_get(const glp_graph* g, int32_t* out, int64_t out_len, int32_t out_on_device) {
+  return guard([&] {
+    if (!g) fail(GLP_ERR_INVALID_ARGUMENT, "graph is NULL");
+    if (!g->has_run) fail(GLP_ERR_STATE, "glp_labels_get before glp_run");
+    if (out_len < g->n) fail(GLP_ERR_INVALID_ARGUMENT, "out_len < n_global");
+    if (g->n == 0) return;
+    if (!out) fail(GLP_ERR_INVALID_ARGUMENT, "out is NULL");
+    CK(cudaSetDevice(g->device));
+    CK(cudaMemcpyAsync(out, g->L[g->cur], g->n * sizeof(int32_t),
+                       out_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+  });
+}
+
+glp_status glp_iter_stats(const glp_graph* g, glp_iter_stat* out, int32_t max_entries, int32_t* n_out) {
+  return guard([&] {
+    if (!g || !n_out || max_entries < 0 || (max_entries > 0 && !out)) fail(GLP_ERR_INVALID_ARGUMENT, "bad arguments");
+    const int32_t k = std::min<int32_t>(max_entries, (int32_t)g->iter_stats.size());
+    for (int32_t i = 0; i < k; ++i) out[i] = g->iter_stats[i];
+    *n_out = (int32_t)g->iter_stats.size();
+  });
+}
+
+glp_status glp_kernel_stats(const glp_graph* g, glp_kernel_stat* out, int32_t max_entries, int32_t* n_out) {
+  return guard([&] {
+    if (!g || !n_out || max_entries < 0 || (max_entries > 0 && !out)) fail(GLP_ERR_INVALID_ARGUMENT, "bad arguments");
+    const int32_t k = std::min<int32_t>(max_entries, (int32_t)g->kstats.size());
+    for (int32_t i = 0; i < k; ++i) {
+      memset(&out[i], 0, sizeof(glp_kernel_stat));
+      strncpy(out[i].name, g->kstats[i].name.c_str(), sizeof(out[i].name) - 1);
+      out[i].launches = g->kstats[i].launches;
+      out[i].ms = g->kstats[i].ms;
+      out[i].bytes = g->kstats[i].bytes;
+      out[i].arcs = g->kstats[i].arcs;
+    }
+    *n_out = (int32_t)g->kstats.size();
+  });
+}
+
+glp_status glp_graph_info(const glp_graph* g, int64_t* out, int32_t max_entries) {
+  return guard([&] {
+    if (!g || (max_entries > 0 && !out)) fail(GLP_ERR_INVALID_ARGUMENT, "bad arguments");
+    std::vector<int64_t> v = {g->n, g->nnz};
+    for (int b = 0; b < NBINS; ++b) { v.push_back(g->bin_verts[b]); v.push_back(g->bin_arcs[b]); }
+    v.push_back(g->max_deg);
+    v.push_back(g->n_chunks);
+    for (int i = 0; i < max_entries && i < (int)v.size(); ++i) out[i] = v[i];
+  });
+}
+
+glp_status glp_partition(const int64_t* row_offsets_host, int64_t n, int32_t nranks, int32_t edge_balanced,
+                         int64_t* bounds_out) {
+  return guard([&] {
+    if (n < 0 || nranks < 1 || !bounds_out) fail(GLP_ERR_INVALID_ARGUMENT, "bad arguments");
+    if (edge_balanced && !row_offsets_host) fail(GLP_ERR_INVALID_ARGUMENT, "row_offsets_host required");
+    bounds_out[0] = 0;
+    if (!edge_balanced) {
+      const int64_t per = (n + nranks - 1) / nranks;
+      for (int r = 1; r <= nranks; ++r) bounds_out[r] = std::min<int64_t>(n, per * r);
+    } else {
+      const int64_t m = row_offsets_host[n];
+      for (int r = 1; r < nranks; ++r) {
+        const int64_t target = (int64_t)((double)m * r / nranks);
+        const int64_t* it = std::lower_bound(row_offsets_host, row_offsets_host + n + 1, target);
+        bounds_out[r] = std::max<int64_t>(bounds_out[r - 1], std::min<int64_t>(n, it - row_offsets_host));
+      }
+      bounds_out[nranks] = n;
+    }
+  });
+}
+
+glp_status glp_nccl_unique_id(uint8_t out[128]) {
+  return guard([&] {
+    if (!out) fail(GLP_ERR_INVALID_ARGUMENT, "out is NULL");
+    nccl_unique_id(out);
+  });
+}
+
+glp_status glp_graph_destroy(glp_graph* g) {
+  return guard([&] { free_graph(g); });
+}
+
+const char* glp_last_error(void) { return g_last_error.c_str(); }
+const char* glp_version(void) { return "glp-b200 0.1 (sm_100a)"; }
+
+}  // extern "C"

@@ -1,0 +1,21 @@
+"""Quick timing probe: generate a graph on the GPU, run LP, print per-iteration stats."""
+import sys, time, json, torch
+sys.path.insert(0, '.')
+import paper_conf_sigmod_yelhls21_b200 as glp
+from glp_inputs import graphs
+scale = int(sys.argv[1]) if len(sys.argv) > 1 else 20
+t0 = time.time()
+csr = graphs.rmat(scale, seed=1, device='cuda')
+torch.cuda.synchronize()
+print('gen', scale, csr.nnz, round(time.time() - t0, 2), 's', flush=True)
+g = glp.Graph(csr)
+print(json.dumps(g.info()), flush=True)
+for rep in range(3):
+    info = g.run('classic', 20, profile=(rep == 2))
+    print(info, flush=True)
+for s in g.iter_stats():
+    print({k: (round(v, 4) if isinstance(v, float) else v) for k, v in s.items()})
+for k in g.kernel_stats():
+    if k['launches']:
+        print(k['name'], k['launches'], round(k['ms'], 3), 'ms', round(k['bytes'] / max(k['ms'], 1e-9) / 1e6, 1), 'GB/s alg',
+              round(k['arcs'] / max(k['ms'], 1e-9) / 1e6, 2), 'Garcs/s')
