@@ -50,12 +50,12 @@ __global__ void k_init_seeds(const int32_t* __restrict__ seeds, int64_t ns, int3
 }
 
 // Frontier push: for every owned vertex changed at iteration t (so.x == t),
-// mark itself and its neighbours (global ids) active for t+1 (marking
-// the changed vertex itself keeps the unconditional-write invariant).  One
-// warp scans 32 stamps, then walks each changed vertex's row cooperatively.
-__global__ void k_push(const int64_t* __restrict__ off, const int32_t* __restrict__ col,
-                       const int2* __restrict__ so, int64_t nl, int64_t vb, int32_t t,
-                       uint8_t* __restrict__ flag) {
+// mark itself and its neighbours (global ids) active for t+1 (DESIGN.md
+// §Frontier: marking the changed vertex itself keeps the unconditional-write
+// invariant).  One warp scans 32 stamps, then walks each changed row.
+__global__ void k_push(const int64_t* __restrict__ ioff, const int32_t* __restrict__ ideg,
+                       const int32_t* __restrict__ col2, const int2* __restrict__ so, int64_t nl, int64_t vb,
+                       int32_t t, uint8_t* __restrict__ flag) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -68,9 +68,21 @@ __global__ void k_push(const int64_t* __restrict__ off, const int32_t* __restric
       m &= m - 1;
       const int64_t u = base + j;
       if (lane == 0) flag[vb + u] = 1;
-      const int64_t e0 = off[u], e1 = off[u + 1];
-      for (int64_t e = e0 + lane; e < e1; e += 32) flag[col[e]] = 1;  // global ids
+      const int64_t e0 = ioff[u], e1 = e0 + ideg[u];
+      for (int64_t e = e0 + lane; e < e1; e += 32) flag[col2[e]] = 1;  // global ids
     }
+  }
+}
+
+// Build the bin-major arc copy: row v of the caller's CSR -> col2[ioff[v]...].
+__global__ void k_relayout(const int64_t* __restrict__ off, const int32_t* __restrict__ col,
+                           const int64_t* __restrict__ ioff, int64_t nl, int32_t* __restrict__ col2) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t v = gw; v < nl; v += nw) {
+    const int64_t s = off[v], d = off[v + 1] - s, o = ioff[v];
+    for (int64_t j = lane; j < d; j += 32) col2[o + j] = col[s + j];
   }
 }
 

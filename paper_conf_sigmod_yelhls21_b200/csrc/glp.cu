@@ -2,7 +2,7 @@
 //
 // Per LP iteration t, all on the graph's stream:
 //   1. reset per-bin counters                                  (memset 256 B)
-//   2. mfl_huge, mfl_high, mfl_mid, mfl_low  R = L_{t-1} -> W = L_t
+//   2. MFL kernels huge, high, mid, low        R = L_{t-1} -> W = L_t
 //   3. [P > 1] ncclAllGather of the owned label slice, counters all-reduce
 //   4. read the counters (changed, d2, sum of changed degrees) -> stop rule R8
 //   5. frontier decision: dense when sum_{changed} deg > nnz / dense_divisor,
@@ -124,14 +124,20 @@ void free_graph(glp_graph* g) {
   delete g;
 }
 
-// ---------------------------------------------------------------- binning
-// Degree bins and low-degree warp chunks (host, once per graph).
-void build_bins(glp_graph* g, const int64_t* off_h) {
-  std::vector<int32_t> low, mid, high, huge, chunk;
+// ---------------------------------------------------------------- layout
+#define GLP_HIGH_KERNEL(VAR) mfl_block<VAR, kHighBlock, kHighSlots, false, kHighUnroll>
+#define GLP_HUGE_KERNEL(VAR) mfl_block<VAR, kHugeBlock, kHugeSlots, true, kHugeUnroll>
+
+// Degree bins, low-degree warp chunks and the bin-major arc copy col2
+// (DESIGN.md §Layout).  Host decides the order; a kernel moves the arcs.
+// off_h: host row offsets; off_d/col_d: the caller's CSR on the device.
+void build_layout(glp_graph* g, const int64_t* off_h, const int64_t* off_d, const int32_t* col_d) {
+  std::vector<int32_t> low, mid, high, huge;
   for (int b = 0; b < NBINS; ++b) g->bin_verts[b] = g->bin_arcs[b] = 0;
   int64_t maxd = 0;
   for (int64_t v = 0; v < g->nl; ++v) {
     const int64_t d = off_h[v + 1] - off_h[v];
+    if (d >= ((int64_t)1 << 30)) fail(GLP_ERR_INVALID_GRAPH, "row degree >= 2^30 is not supported");
     maxd = std::max(maxd, d);
     int b;
     if (d == 0) b = BIN_ISO;
@@ -143,35 +149,81 @@ void build_bins(glp_graph* g, const int64_t* off_h) {
     g->bin_arcs[b] += d;
   }
   g->max_deg = maxd;
-  // greedy chunks: maximal runs of the low list with sum of degrees <= 32
-  chunk.push_back(0);
-  int sum = 0;
-  for (size_t k = 0; k < low.size(); ++k) {
-    const int d = (int)(off_h[low[k] + 1] - off_h[low[k]]);
-    if (sum + d > 32) {
-      chunk.push_back((int32_t)k);
-      sum = 0;
-    }
-    sum += d;
-  }
-  if (!low.empty()) chunk.push_back((int32_t)low.size());
-  // largest first: the block-per-vertex bins start the long rows early
-  auto by_deg = [&](int32_t a, int32_t b) {
-    const int64_t da = off_h[a + 1] - off_h[a], db = off_h[b + 1] - off_h[b];
-    return da != db ? da > db : a < b;
-  };
+  auto deg = [&](int32_t v) { return off_h[v + 1] - off_h[v]; };
+  // largest rows first in the block-per-vertex bins (long rows start early)
+  auto by_deg = [&](int32_t a, int32_t b) { return deg(a) != deg(b) ? deg(a) > deg(b) : a < b; };
   std::sort(huge.begin(), huge.end(), by_deg);
   std::sort(high.begin(), high.end(), by_deg);
+  std::vector<int64_t> ioff(g->nl, 0);
+  std::vector<int32_t> ideg(g->nl, 0);
+  int64_t pos = 0;
+  // low bin: greedy chunks of consecutive low vertices with sum(deg) <= 32
+  std::vector<LowChunk> chunks;
+  {
+    size_t k = 0;
+    while (k < low.size()) {
+      LowChunk c;
+      c.vbase = (int32_t)k;
+      c.segmask = 0;
+      int total = 0;
+      const int64_t cstart = pos;
+      while (k < low.size() && total + deg(low[k]) <= 32) {
+        const int32_t v = low[k];
+        c.segmask |= 1u << total;
+        ioff[v] = pos;
+        ideg[v] = (int32_t)deg(v);
+        pos += deg(v);
+        total += (int)deg(v);
+        ++k;
+      }
+      c.st = (unsigned long long)cstart | ((unsigned long long)total << 56);
+      chunks.push_back(c);
+    }
+  }
+  auto place = [&](const std::vector<int32_t>& vs, std::vector<BinItem>& items) {
+    pos = (pos + 3) & ~(int64_t)3;
+    for (int32_t v : vs) {
+      BinItem it;
+      it.start = pos;
+      it.v = v;
+      it.d = (int32_t)deg(v);
+      ioff[v] = pos;
+      ideg[v] = it.d;
+      items.push_back(it);
+      pos += (deg(v) + 3) & ~(int64_t)3;
+    }
+  };
+  std::vector<BinItem> mid_i, high_i, huge_i;
+  place(mid, mid_i);
+  place(high, high_i);
+  place(huge, huge_i);
+  g->nnz2 = pos;
+  if (pos >= ((int64_t)1 << 56)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
   g->n_low = (int32_t)low.size();
-  g->n_chunks = low.empty() ? 0 : (int32_t)chunk.size() - 1;
-  g->n_mid = (int32_t)mid.size();
-  g->n_high = (int32_t)high.size();
-  g->n_huge = (int32_t)huge.size();
+  g->n_chunks = (int32_t)chunks.size();
+  g->n_mid = (int32_t)mid_i.size();
+  g->n_high = (int32_t)high_i.size();
+  g->n_huge = (int32_t)huge_i.size();
   g->low_list = upload(g, low);
-  g->low_chunk = upload(g, chunk);
-  g->mid_list = upload(g, mid);
-  g->high_list = upload(g, high);
-  g->huge_list = upload(g, huge);
+  g->chunks = upload(g, chunks);
+  g->mid_items = upload(g, mid_i);
+  g->high_items = upload(g, high_i);
+  g->huge_items = upload(g, huge_i);
+  g->ioff = upload(g, ioff);
+  g->ideg = upload(g, ideg);
+  g->col2 = dalloc<int32_t>(g, g->nnz2);
+  CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), g->stream));  // padding = -1
+  if (g->nl > 0 && g->nnz > 0) {
+    k_relayout<<<g->sms * 8, 256, 0, g->stream>>>(off_d, col_d, g->ioff, g->nl, g->col2);
+    CK(cudaGetLastError());
+  }
+  g->ovf_hint = dalloc<uint8_t>(g, std::max<int32_t>(g->n_huge, 1));
+  g->ovf_init.resize(g->n_huge);
+  for (int32_t i = 0; i < g->n_huge; ++i) {
+    // all-distinct estimate for t = 1: enough partitions for <= SLOTS/2 labels each
+    const int64_t p = (huge_i[i].d + kHugeSlots / 2 - 1) / (kHugeSlots / 2);
+    g->ovf_init[i] = (uint8_t)std::min<int64_t>(p, 255);
+  }
 }
 
 void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm, glp_graph** out) {
@@ -230,42 +282,63 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->symmetric = csr->symmetric ? 1 : 0;
     if (g->nnz >= ((int64_t)1 << 40)) fail(GLP_ERR_INVALID_ARGUMENT, "nnz_local too large");
 
+    g->sms = prop.multiProcessorCount;
     std::vector<int64_t> off_h;
     const int64_t* off_host = nullptr;
+    const int64_t* off_d = nullptr;
+    const int32_t* col_d = nullptr;
+    std::vector<void*> temps;  // caller-CSR staging freed after the relayout
     if (csr->on_device) {
-      g->off = csr->row_offsets;
-      g->col = csr->col_idx;
+      off_d = csr->row_offsets;
+      col_d = csr->col_idx;
       off_h.resize(g->nl + 1);
-      CK(cudaMemcpyAsync(off_h.data(), g->off, (g->nl + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, g->stream));
+      CK(cudaMemcpyAsync(off_h.data(), off_d, (g->nl + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, g->stream));
       CK(cudaStreamSynchronize(g->stream));
       off_host = off_h.data();
     } else {
-      int64_t* doff = dalloc<int64_t>(g, g->nl + 1);
-      int32_t* dcol = dalloc<int32_t>(g, g->nnz);
-      CK(cudaMemcpyAsync(doff, csr->row_offsets, (g->nl + 1) * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
-      if (g->nnz)
-        CK(cudaMemcpyAsync(dcol, csr->col_idx, g->nnz * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
-      g->off = doff;
-      g->col = dcol;
-      g->own_csr = true;
       off_host = csr->row_offsets;
+      void *po = nullptr, *pc = nullptr;
+      if (cudaMalloc(&po, (g->nl + 1) * sizeof(int64_t)) != cudaSuccess ||
+          cudaMalloc(&pc, std::max<int64_t>(g->nnz, 1) * sizeof(int32_t)) != cudaSuccess) {
+        cudaGetLastError();
+        if (po) cudaFree(po);
+        if (pc) cudaFree(pc);
+        fail(GLP_ERR_OUT_OF_MEMORY, "staging the CSR on the device failed");
+      }
+      temps.push_back(po);
+      temps.push_back(pc);
+      CK(cudaMemcpyAsync(po, csr->row_offsets, (g->nl + 1) * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
+      if (g->nnz)
+        CK(cudaMemcpyAsync(pc, csr->col_idx, g->nnz * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
+      off_d = (const int64_t*)po;
+      col_d = (const int32_t*)pc;
+      g->own_csr = true;
     }
+    struct TempGuard {
+      std::vector<void*>& v;
+      cudaStream_t s;
+      ~TempGuard() {
+        if (!v.empty()) cudaStreamSynchronize(s);
+        for (void* p : v) cudaFree(p);
+      }
+    } tg{temps, g->stream};
     // host-side structural checks on the offsets (cheap, always on)
     if (off_host[0] != 0 || off_host[g->nl] != g->nnz)
       fail(GLP_ERR_INVALID_GRAPH, "row_offsets[0] must be 0 and row_offsets[last] == nnz_local");
-    if (p.validate) {
-      for (int64_t v = 0; v < g->nl; ++v)
-        if (off_host[v + 1] < off_host[v]) fail(GLP_ERR_INVALID_GRAPH, "row_offsets not non-decreasing");
+    for (int64_t v = 0; v < g->nl; ++v)
+      if (off_host[v + 1] < off_host[v]) fail(GLP_ERR_INVALID_GRAPH, "row_offsets not non-decreasing");
+    if (p.validate && g->nnz) {
       int* dbad = dalloc<int>(g, 1);
       CK(cudaMemsetAsync(dbad, 0, sizeof(int), g->stream));
-      if (g->nnz) k_validate_col<<<prop.multiProcessorCount * 4, 256, 0, g->stream>>>(g->col, g->nnz, g->n, dbad);
+      k_validate_col<<<g->sms * 4, 256, 0, g->stream>>>(col_d, g->nnz, g->n, dbad);
       CK(cudaGetLastError());
       int bad = 0;
       CK(cudaMemcpyAsync(&bad, dbad, sizeof(int), cudaMemcpyDeviceToHost, g->stream));
       CK(cudaStreamSynchronize(g->stream));
       if (bad) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
     }
-    build_bins(g, off_host);
+    build_layout(g, off_host, off_d, col_d);
+    CK(cudaStreamSynchronize(g->stream));
 
     // labels: replicated full arrays, padded to a multiple of nranks for the
     // in-place all-gather
@@ -285,23 +358,23 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaEventCreate(&g->ev_a));
     CK(cudaEventCreate(&g->ev_b));
 
-    const int sms = prop.multiProcessorCount;
-    g->sms = sms;
-    CK(cudaFuncSetAttribute(mfl_high<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHighSlots * 8));
-    CK(cudaFuncSetAttribute(mfl_high<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHighSlots * 8));
-    CK(cudaFuncSetAttribute(mfl_high<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHighSlots * 8));
-    CK(cudaFuncSetAttribute(mfl_huge<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHugeSlots * 8));
-    CK(cudaFuncSetAttribute(mfl_huge<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHugeSlots * 8));
-    CK(cudaFuncSetAttribute(mfl_huge<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHugeSlots * 8));
-    g->grid_low = grid_for(sms, (const void*)mfl_low<V_CLASSIC>, kLowBlock, 0);
-    g->grid_mid = grid_for(sms, (const void*)mfl_mid<V_CLASSIC>, kMidBlock, 0);
-    g->grid_high = grid_for(sms, (const void*)mfl_high<V_LLP>, kHighBlock, kHighSlots * 8);
-    g->grid_huge = grid_for(sms, (const void*)mfl_huge<V_LLP>, kHugeBlock, kHugeSlots * 8);
+    const int sms = g->sms;
+    const int hs = kHighSlots * 8, us = kHugeSlots * 8;
+    CK(cudaFuncSetAttribute(GLP_HIGH_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, hs));
+    CK(cudaFuncSetAttribute(GLP_HIGH_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, hs));
+    CK(cudaFuncSetAttribute(GLP_HIGH_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, hs));
+    CK(cudaFuncSetAttribute(GLP_HUGE_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, us));
+    CK(cudaFuncSetAttribute(GLP_HUGE_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, us));
+    CK(cudaFuncSetAttribute(GLP_HUGE_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, us));
+    g->grid_low = grid_for(sms, (const void*)mfl_low<V_LLP>, kLowBlock, 0);
+    g->grid_mid = grid_for(sms, (const void*)mfl_mid<V_LLP>, kMidBlock, 0);
+    g->grid_high = grid_for(sms, (const void*)GLP_HIGH_KERNEL(V_LLP), kHighBlock, hs);
+    g->grid_huge = grid_for(sms, (const void*)GLP_HUGE_KERNEL(V_LLP), kHugeBlock, us);
     g->grid_aux = sms * 8;
     if (g->n_huge > 0) {
       g->grid_huge = std::min<int>(g->grid_huge, g->n_huge);
-      g->ght_slots = 2 * g->max_deg;
-      g->ght = dalloc<unsigned long long>(g, (size_t)g->ght_slots * g->grid_huge);
+      g->stage_stride = (g->max_deg + 3) & ~(int64_t)3;
+      g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 2 * g->grid_huge);
     }
     g->nnz_global = g->nnz;
     if (nranks > 1) nccl_init(g, dist->nccl_unique_id);
@@ -352,25 +425,29 @@ void launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, 
   Counters* c = g->d_cnt;
   if (g->n_huge) {
     MflArgs b = a;
-    b.list = g->huge_list; b.list_len = g->n_huge; b.cnt = c + 3;
-    b.ght = g->ght; b.ght_slots = g->ght_slots;
-    timed(g, prof, 3, pend, used, [&] { mfl_huge<VAR><<<g->grid_huge, kHugeBlock, kHugeSlots * 8, g->stream>>>(b); });
+    b.items = g->huge_items; b.n_items = g->n_huge; b.cnt = c + 3;
+    b.ovf_hint = g->ovf_hint; b.stage = g->stage; b.stage_stride = g->stage_stride;
+    timed(g, prof, 3, pend, used, [&] {
+      GLP_HUGE_KERNEL(VAR)<<<g->grid_huge, kHugeBlock, kHugeSlots * 8, g->stream>>>(b);
+    });
   }
   if (g->n_high) {
     MflArgs b = a;
-    b.list = g->high_list; b.list_len = g->n_high; b.cnt = c + 2;
+    b.items = g->high_items; b.n_items = g->n_high; b.cnt = c + 2;
     const int grid = std::min<int>(g->grid_high, g->n_high);
-    timed(g, prof, 2, pend, used, [&] { mfl_high<VAR><<<grid, kHighBlock, kHighSlots * 8, g->stream>>>(b); });
+    timed(g, prof, 2, pend, used, [&] {
+      GLP_HIGH_KERNEL(VAR)<<<grid, kHighBlock, kHighSlots * 8, g->stream>>>(b);
+    });
   }
   if (g->n_mid) {
     MflArgs b = a;
-    b.list = g->mid_list; b.list_len = g->n_mid; b.cnt = c + 1;
+    b.items = g->mid_items; b.n_items = g->n_mid; b.cnt = c + 1;
     const int grid = std::min<int>(g->grid_mid, (g->n_mid + kMidBlock / 32 - 1) / (kMidBlock / 32));
     timed(g, prof, 1, pend, used, [&] { mfl_mid<VAR><<<grid, kMidBlock, 0, g->stream>>>(b); });
   }
   if (g->n_chunks) {
     MflArgs b = a;
-    b.list = g->low_list; b.list_len = g->n_low; b.chunk = g->low_chunk; b.n_chunks = g->n_chunks; b.cnt = c + 0;
+    b.list = g->low_list; b.chunks = g->chunks; b.n_chunks = g->n_chunks; b.cnt = c + 0;
     const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock / 32 - 1) / (kLowBlock / 32));
     timed(g, prof, 0, pend, used, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, g->stream>>>(b); });
   }
@@ -424,13 +501,21 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     k_hist<<<ga, 256, 0, s>>>(g->L[0], g->n, g->V);
     CK(cudaGetLastError());
   }
+  if (g->n_huge) {
+    // t = 1 of CLASSIC/LLP has all-distinct labels: rows wider than the shared
+    // table start in the global table (performance hint only)
+    std::vector<uint8_t> h(g->ovf_init);
+    if (variant == GLP_VARIANT_SEEDED) std::fill(h.begin(), h.end(), 1);
+    CK(cudaMemcpyAsync(g->ovf_hint, h.data(), h.size(), cudaMemcpyHostToDevice, s));
+    CK(cudaStreamSynchronize(s));
+  }
   int rb = 0;  // R = L[rb], W = L[1-rb]
   int fb = 0;  // flags read this iteration
   bool dense = true;
   if (variant == GLP_VARIANT_SEEDED) {
     // frontier of t = 1 is N(S) (+ S): push from the seeds (stamped t = 0)
     if (use_frontier) {
-      k_push<<<ga, 256, 0, s>>>(g->off, g->col, g->so, g->nl, g->vb, 0, g->flag[fb]);
+      k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, 0, g->flag[fb]);
       CK(cudaGetLastError());
       g->flag_clean[fb] = false;
       if (g->nranks > 1) nccl_merge_flags(g, g->flag[fb]);
@@ -478,7 +563,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     CK(cudaMemsetAsync(g->d_cnt, 0, 4 * sizeof(Counters), s));
     MflArgs a;
     memset(&a, 0, sizeof(a));
-    a.off = g->off; a.col = g->col; a.R = g->L[rb]; a.W = g->L[1 - rb]; a.so = g->so;
+    a.col = g->col2; a.R = g->L[rb]; a.W = g->L[1 - rb]; a.so = g->so;
     a.V = g->V; a.is_seed = g->is_seed; a.flag = g->flag[fb];
     a.vb = g->vb; a.gamma = p.gamma; a.t = t; a.dense = dense ? 1 : 0;
     switch (variant) {
@@ -524,7 +609,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       next_dense = (double)tot.chdeg * (double)p.dense_divisor > (double)g->nnz_global;
     if (!stop && !next_dense) {
       timed(g, prof, 4, pend, used, [&] {
-        k_push<<<ga, 256, 0, s>>>(g->off, g->col, g->so, g->nl, g->vb, t, g->flag[nf]);
+        k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, g->flag[nf]);
         if (g->nranks > 1) nccl_merge_flags(g, g->flag[nf]);
       });
       g->flag_clean[nf] = false;

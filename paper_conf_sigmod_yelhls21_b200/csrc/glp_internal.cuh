@@ -1,8 +1,10 @@
 // glp_internal.cuh -- internal types of libglp.so (not part of the ABI).
 //
 // Data layout in HBM:
-//   off   int64[nl+1]   CSR row offsets of the owned rows           [P:97]
-//   col   int32[nnz]    global neighbour ids, streamed once/iter    [P:97]
+//   col2  int32[nnz2]   bin-major copy of the owned arcs (global ids):
+//                       low chunks contiguous, other rows 16-B aligned and
+//                       padded with -1; streamed once per iteration   [P:97]
+//   ioff/ideg [nl]      row start in col2 / degree (frontier push)
 //   L[2]  int32[n]      labels, double-buffered (R = L_{t-1}, W = L_t) [P:143]
 //   so    int2[nl]      (stamp, old): iteration of the last change and the
 //                       label before it -> exact 2-cycle test (R8)
@@ -25,17 +27,37 @@ namespace glp {
 // high/huge: block per vertex with a shared-memory hash table (PAPER §4.1).
 constexpr int kLowMax = 32;       // deg <= 32   -> mfl_low  (one warp, several vertices)
 constexpr int kMidMax = 256;      // deg <= 256  -> mfl_mid  (one warp, one vertex)
-constexpr int kHighMax = 4096;    // deg <= 4096 -> mfl_high (256-thread block per vertex)
-                                  // deg >  4096 -> mfl_huge (1024-thread block, smem
-                                  //                 table + global overflow table)
+constexpr int kHighMax = 2048;    // deg <= 2048 -> mfl_block<128 thr, 4096 slots>
+                                  // deg >  2048 -> mfl_block<1024 thr, 16384 slots,
+                                  //                 partitioned recount on overflow>
 constexpr int kLowBlock = 256;
 constexpr int kMidBlock = 256;
-constexpr int kMidSlots = 2 * kMidMax;      // per-warp table slots (u64)
-constexpr int kHighBlock = 256;
-constexpr int kHighSlots = 2 * kHighMax;    // 64 KB table
+constexpr int kMidSlots = 2 * kMidMax;      // per-warp table slots (key+count u32), load <= 1/2
+constexpr int kHighBlock = 128;
+constexpr int kHighSlots = 2 * kHighMax;    // 32 KB table, load <= 1/2
+constexpr int kHighUnroll = 2;
 constexpr int kHugeBlock = 1024;
-constexpr int kHugeSlots = 24576;           // 192 KB table
+constexpr int kHugeSlots = 16384;           // 128 KB table
+constexpr int kHugeUnroll = 2;
 constexpr int kHugeProbe = 32;              // probe limit before declaring overflow
+
+// A low-degree chunk: up to 32 consecutive arcs of consecutive low-list
+// vertices.  st = arc start in col2 | (arc count << 56); bit i of segmask set
+// iff a vertex's first arc is at lane i; vbase = index of its first vertex in
+// the low list.
+struct LowChunk {
+  unsigned long long st;
+  int32_t vbase;
+  uint32_t segmask;
+};
+
+// A mid/high/huge row: arcs col2[start, start + d) (start 16-byte aligned,
+// padded with -1 up to a multiple of 4).
+struct BinItem {
+  int64_t start;
+  int32_t v;  // local vertex id
+  int32_t d;
+};
 
 enum Bin { BIN_ISO = 0, BIN_LOW = 1, BIN_MID = 2, BIN_HIGH = 3, BIN_HUGE = 4, NBINS = 5 };
 
@@ -46,26 +68,27 @@ struct Counters {
   unsigned long long chdeg;     // sum of deg over changed vertices
   unsigned long long arcs;      // arcs scanned
   unsigned long long verts;     // vertices scanned
-  unsigned long long huge_next; // dynamic work counter of mfl_huge
+  unsigned long long work_next; // dynamic work counter (huge bin)
   unsigned long long pad[2];
 };
 
 // Arguments shared by the MFL kernels (passed by value).
 struct MflArgs {
-  const int64_t* __restrict__ off;      // [nl+1]
-  const int32_t* __restrict__ col;      // [nnz]
+  const int32_t* __restrict__ col;      // col2: bin-major arcs (global ids, -1 = padding)
   const int32_t* __restrict__ R;        // L_{t-1}, global ids [n]
   int32_t* __restrict__ W;              // L_t, global ids [n]
   int2* __restrict__ so;                // [nl] (stamp, old label)
   const int32_t* __restrict__ V;        // LLP histogram [n] or null
   const uint8_t* __restrict__ is_seed;  // [nl] or null
   const uint8_t* __restrict__ flag;     // [npad] frontier marks by global id (sparse)
-  const int32_t* __restrict__ list;     // bin vertex list (local ids)
-  int32_t list_len;
-  const int32_t* __restrict__ chunk;    // low bin: chunk starts into list [nchunks+1]
+  const int32_t* __restrict__ list;     // low bin: vertex list (local ids)
+  const LowChunk* __restrict__ chunks;  // low bin
   int32_t n_chunks;
-  unsigned long long* __restrict__ ght; // huge: per-block global overflow tables
-  int64_t ght_slots;                    // slots per block
+  const BinItem* __restrict__ items;    // mid/high/huge bins
+  int32_t n_items;
+  uint8_t* __restrict__ ovf_hint;       // huge bin: hash partitions to start with
+  int32_t* __restrict__ stage;          // huge bin: per-block staged row labels
+  int64_t stage_stride;
   Counters* cnt;
   int64_t vb;                           // global id of local row 0
   double gamma;
@@ -105,12 +128,17 @@ struct glp_graph {
   int symmetric = 1;
   int64_t max_deg = 0;
 
-  // degree bins (device lists of local ids)
+  // bin-major arc layout
+  int32_t* col2 = nullptr;  int64_t nnz2 = 0;
+  int64_t* ioff = nullptr;  // [nl] start of row v in col2
+  int32_t* ideg = nullptr;  // [nl] degree of row v
   int32_t* low_list = nullptr;  int32_t n_low = 0;
-  int32_t* low_chunk = nullptr; int32_t n_chunks = 0;
-  int32_t* mid_list = nullptr;  int32_t n_mid = 0;
-  int32_t* high_list = nullptr; int32_t n_high = 0;
-  int32_t* huge_list = nullptr; int32_t n_huge = 0;
+  glp::LowChunk* chunks = nullptr;   int32_t n_chunks = 0;
+  glp::BinItem* mid_items = nullptr; int32_t n_mid = 0;
+  glp::BinItem* high_items = nullptr; int32_t n_high = 0;
+  glp::BinItem* huge_items = nullptr; int32_t n_huge = 0;
+  uint8_t* ovf_hint = nullptr;
+  std::vector<uint8_t> ovf_init;  // per-run initial hints (host)
   int64_t bin_verts[glp::NBINS] = {0}, bin_arcs[glp::NBINS] = {0};
 
   // per-rank row bounds (all ranks), for the exchange
@@ -123,8 +151,8 @@ struct glp_graph {
   uint8_t* is_seed = nullptr;
   uint8_t* flag[2] = {nullptr, nullptr};
   bool flag_clean[2] = {true, true};
-  unsigned long long* ght = nullptr;
-  int64_t ght_slots = 0;
+  int32_t* stage = nullptr;  // huge bin staging buffers (grid_huge x stage_stride)
+  int64_t stage_stride = 0;
   glp::Counters* d_cnt = nullptr;
   glp::Counters* h_cnt = nullptr;  // pinned
   int32_t* d_seeds = nullptr;

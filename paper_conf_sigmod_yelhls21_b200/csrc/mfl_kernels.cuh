@@ -6,16 +6,21 @@
 // the best label (score desc, label asc: R4) to W = L_t (UpdateVertex [P:112],
 // Lnext [P:143]).
 //
+// Arcs are read from the library's bin-major copy `col2`:
+// the arcs of each low-degree chunk are contiguous, and every mid/high/huge row
+// starts 16-byte aligned and is padded with -1 to a multiple of 4, so rows are
+// streamed with one 128-bit load per lane.
+//
 // Kernels by degree bin:
-//   mfl_low   deg <= 32: one warp serves several vertices whose arcs are
-//             contiguous ("one-warp-multi-vertices" [P:227-234 §4.2]):
-//             activemask/vmask/lmask + popc, then a segmented redux arg-max.
+//   mfl_low   deg <= 32: one warp serves several vertices whose arcs fill its
+//             32 lanes ("one-warp-multi-vertices" [P:227-234 §4.2]): lane
+//             masks from the chunk's segment-start bitmap, label frequency per
+//             segment, shuffle-tree arg-max per segment.
 //   mfl_mid   deg <= 256: one warp per vertex, per-warp shared-memory table.
-//   mfl_high  deg <= 4096: one block per vertex, shared-memory table
-//             ("SharedMemBigNodes" HT [P:132-182 §4.1]).
-//   mfl_huge  deg > 4096: as high with a 192 KB table; when a label finds no
-//             slot within kHugeProbe probes the vertex is recounted exactly in a
-//             per-block global-memory table (GlobalInsert/GHT [P:166, P:182]).
+//   mfl_block deg > 256: one block per vertex with a shared-memory hash table
+//             ("SharedMemBigNodes" HT [P:132-182 §4.1]); the largest bin
+//             recounts rows whose distinct labels overflow the table in hash
+//             partitions (replacing GlobalInsert/GHT [P:166, P:182]).
 //
 // Exactness of the running arg-max (the paper's ht_score taken from the
 // atomicAdd return value [P:150-156]): a label's count only grows, and its
@@ -32,7 +37,6 @@
 namespace glp {
 
 constexpr unsigned kFull = 0xffffffffu;
-constexpr unsigned long long kEmpty = ~0ull;  // table slot: (label << 32) | count
 constexpr unsigned kNoLabel = 0xffffffffu;
 
 enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
@@ -42,7 +46,14 @@ __device__ __forceinline__ int ld_stream(const int32_t* p) {
   asm volatile("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(r) : "l"(p));
   return r;
 }
+__device__ __forceinline__ int4 ld_stream4(const int32_t* p) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
 __device__ __forceinline__ int ld_label(const int32_t* p) { return __ldg(p); }
+__device__ __forceinline__ int gather(const MflArgs& a, int u) { return u >= 0 ? ld_label(a.R + u) : -1; }
 
 // LLP score val = k - gamma * (v - k) [P:119], double, no contraction (R11).
 __device__ __forceinline__ double llp_score(unsigned k, int v, double gamma) {
@@ -52,63 +63,112 @@ __device__ __forceinline__ double llp_score(unsigned k, int v, double gamma) {
   return __dsub_rn(kd, prod);
 }
 
-// Order-preserving map double -> u64 (finite and infinite values).
+// Order-preserving map double -> u64 (finite and infinite values); 0 = none.
 __device__ __forceinline__ unsigned long long dkey(double x) {
   unsigned long long b = (unsigned long long)__double_as_longlong(x);
   return (b >> 63) ? ~b : (b | 0x8000000000000000ull);
 }
 
-// Score key of label `lab` with count `k`: larger is better.
+// Running best (score desc, label asc).  CLASSIC/SEEDED pack (count, ~label)
+// into one u64 so "better" is a single 64-bit max; LLP keeps (score key, label).
 template <int VAR>
-__device__ __forceinline__ unsigned long long score_key(unsigned k, unsigned lab, const MflArgs& a) {
-  if (VAR == V_LLP) return dkey(llp_score(k, ld_label(a.V + lab), a.gamma));
-  return (unsigned long long)k;
-}
-
 struct Best {
-  unsigned long long key;  // 0 = none
-  unsigned lab;
-};
-__device__ __forceinline__ bool better(unsigned long long k1, unsigned l1, unsigned long long k2, unsigned l2) {
-  return k1 > k2 || (k1 == k2 && l1 < l2);
-}
-__device__ __forceinline__ void best_update(Best& b, unsigned long long k, unsigned l) {
-  if (better(k, l, b.key, b.lab)) { b.key = k; b.lab = l; }
-}
-__device__ __forceinline__ Best warp_best(Best b) {
-#pragma unroll
-  for (int s = 16; s > 0; s >>= 1) {
-    unsigned long long k = __shfl_xor_sync(kFull, b.key, s);
-    unsigned l = __shfl_xor_sync(kFull, b.lab, s);
-    best_update(b, k, l);
+  unsigned long long key = 0ull;
+  unsigned lab = kNoLabel;
+  __device__ __forceinline__ void observe(unsigned cnt, unsigned l, const MflArgs& a) {
+    if (VAR == V_LLP) {
+      const unsigned long long k = dkey(llp_score(cnt, ld_label(a.V + l), a.gamma));
+      if (k > key || (k == key && l < lab)) { key = k; lab = l; }
+    } else {
+      const unsigned long long k = ((unsigned long long)cnt << 32) | (unsigned long long)(~l);
+      key = k > key ? k : key;
+    }
   }
-  return b;
-}
+  __device__ __forceinline__ void merge(unsigned long long k, unsigned l) {
+    if (VAR == V_LLP) {
+      if (k > key || (k == key && l < lab)) { key = k; lab = l; }
+    } else {
+      key = k > key ? k : key;
+    }
+  }
+  __device__ __forceinline__ bool have() const { return key != 0ull; }
+  __device__ __forceinline__ unsigned label() const { return VAR == V_LLP ? lab : ~(unsigned)key; }
+  __device__ __forceinline__ void warp_reduce() {
+#pragma unroll
+    for (int s = 16; s > 0; s >>= 1) {
+      const unsigned long long k = __shfl_xor_sync(kFull, key, s);
+      const unsigned l = VAR == V_LLP ? __shfl_xor_sync(kFull, lab, s) : 0u;
+      merge(k, l);
+    }
+  }
+};
 
 __device__ __forceinline__ unsigned slot_hash(unsigned lab, unsigned tsz) {
   return __umulhi(lab * 0x9E3779B1u, tsz);
 }
 
-// Insert `c` occurrences of `lab` into an open-addressing table of `tsz` slots
-// (shared or global memory).  Returns the post-increment count, or 0 when no
-// slot was found within `max_probe` probes (overflow).
-__device__ __forceinline__ unsigned ht_add(unsigned long long* tab, unsigned tsz, unsigned lab,
-                                           unsigned c, unsigned max_probe) {
-  unsigned h = slot_hash(lab, tsz);
-  for (unsigned p = 0; p < max_probe; ++p) {
-    unsigned long long e = *((volatile unsigned long long*)(tab + h));
+// Open-addressing count table in shared memory: tsz (a power of two) u64
+// slots holding (label << 32) | count, kEmpty when free; linear probing.
+constexpr unsigned long long kEmpty = ~0ull;
+struct Table {
+  unsigned long long* slots;
+  unsigned tsz;
+  // cooperative clear by `nthr` threads starting at thread `tid` (16-B stores)
+  __device__ __forceinline__ void clear(unsigned tid, unsigned nthr) const {
+    uint4* s4 = (uint4*)slots;
+    for (unsigned j = tid; j < tsz / 2; j += nthr) s4[j] = make_uint4(kFree32, kFree32, kFree32, kFree32);
+  }
+  static constexpr unsigned kFree32 = 0xffffffffu;
+};
+
+// Insert `c` occurrences of `lab`.  Returns the post-increment count, or 0
+// when no slot was found within `max_probe` probes (overflow).  *fresh is set
+// when this call claimed a new slot (distinct-label accounting).  A new label
+// costs one CAS that claims the slot and sets its count.
+__device__ __forceinline__ unsigned ht_add(const Table& t, unsigned lab, unsigned c, unsigned max_probe,
+                                           bool* fresh) {
+  unsigned h = slot_hash(lab, t.tsz);
+  for (unsigned p = 0;; ++p) {
+    unsigned long long e = *((volatile unsigned long long*)(t.slots + h));
     if (e == kEmpty) {
-      unsigned long long prev = atomicCAS(tab + h, kEmpty, ((unsigned long long)lab << 32) | c);
-      if (prev == kEmpty) return c;
+      const unsigned long long prev = atomicCAS(t.slots + h, kEmpty, ((unsigned long long)lab << 32) | c);
+      if (prev == kEmpty) {
+        *fresh = true;
+        return c;
+      }
       e = prev;
     }
-    if ((unsigned)(e >> 32) == lab) {
-      unsigned long long old = atomicAdd(tab + h, (unsigned long long)c);
-      return (unsigned)old + c;
-    }
-    if (++h == tsz) h = 0;
+    // increments go to the count half with a native 32-bit shared atomic (a
+    // 64-bit add would be a CAS loop under hot-key contention); a CAS.64 can no
+    // longer succeed on a claimed slot, so the two never race.
+    if ((unsigned)(e >> 32) == lab) return atomicAdd((unsigned*)(t.slots + h), c) + c;
+    if (p + 1 >= max_probe) return 0u;
+    h = (h + 1) & (t.tsz - 1);
   }
-  return 0;
+}
+
+// Insert one label per voting lane.  The warp's "hot" label -- lane 0's best
+// label so far (its own label on a fresh row) -- is merged with one ballot
+// first, so a collapsed neighbourhood (most neighbours share a community label
+// [P:130]) costs one shared atomic instead of 32 same-address atomics; the
+// other voting lanes insert individually (distinct-label regime, e.g. t = 1).
+// Returns the number of newly claimed slots in the warp when COUNT_NEW.
+template <int VAR, bool COUNT_NEW>
+__device__ __forceinline__ unsigned warp_insert(const MflArgs& a, const Table& t, unsigned max_probe, int lab,
+                                                bool vote, Best<VAR>& b, volatile int* overflow) {
+  const int lane = threadIdx.x & 31;
+  const int cand = b.have() ? (int)b.label() : lab;
+  const int hot = __shfl_sync(kFull, cand, 0);
+  const unsigned m = __ballot_sync(kFull, vote && lab == hot);
+  unsigned c = 0;
+  if (vote) c = (lab != hot) ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u);
+  bool fresh = false;
+  if (c) {
+    const unsigned cnt = ht_add(t, (unsigned)lab, c, max_probe, &fresh);
+    if (cnt == 0u) *overflow = 1;
+    else b.observe(cnt, (unsigned)lab, a);
+  }
+  return COUNT_NEW ? (unsigned)__popc(__ballot_sync(kFull, fresh)) : 0u;
 }
 
 // Per-thread iteration statistics, block-reduced once at kernel exit.
@@ -158,6 +218,7 @@ __device__ __forceinline__ void update_vertex(const MflArgs& a, int v, int deg, 
   const int l2 = (so.x == a.t - 1) ? so.y : r;  // L_{t-2}[v]
   a.W[gv] = nw;
   ty.verts += 1;
+  ty.arcs += (unsigned long long)deg;
   ty.d2 += (nw != l2);
   if (nw != r) {
     ty.changed += 1;
@@ -167,257 +228,327 @@ __device__ __forceinline__ void update_vertex(const MflArgs& a, int v, int deg, 
 }
 
 // ---------------------------------------------------------------------------
-// mfl_low: one warp, up to 32 arcs of several consecutive low-degree vertices
-// (a static "chunk" of the low list with sum of degrees <= 32).
-// Fig. 3 / [P:229-232]: activemask = ballot(valid label); vmask = lanes of the
-// same vertex (from the chunk's segment starts); lmask = match_any(label) &
-// vmask; frequency = popc(lmask).  Arg-max: redux max(count), then redux
-// min(label) over the lanes of the vertex (R4).
+// mfl_low: one warp per chunk = up to 32 consecutive arcs of several low-degree
+// vertices.  Fig. 3 / [P:229-232]: activemask = lanes holding a valid label;
+// vmask = lanes of the same vertex (from the chunk's segment-start bitmap);
+// frequency = number of lanes of vmask with the same label (a shuffle loop as
+// long as the chunk's longest segment: match.any.sync costs ~60 SM cycles per
+// warp on distinct keys on sm_100, tools/ubench); arg-max = shuffle tree over
+// the segment.
 template <int VAR>
 __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
   const int lane = threadIdx.x & 31;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
+  const unsigned le = kFull >> (31 - lane);  // lanes 0..lane
   Tally ty;
   for (int c = gw; c < a.n_chunks; c += nwarps) {
-    const int k0 = a.chunk[c];
-    const int nv = a.chunk[c + 1] - k0;
-    int v = 0, d = 0;
-    int64_t o = 0;
-    if (lane < nv) {
-      v = a.list[k0 + lane];
-      o = a.off[v];
-      d = (int)(a.off[v + 1] - o);
-    }
+    const LowChunk ch = a.chunks[c];
+    const int64_t start = (int64_t)(ch.st & ((1ull << 56) - 1));
+    const int total = (int)(ch.st >> 56);
+    const unsigned segs = ch.segmask;
     if (!a.dense) {
-      const bool act = lane < nv && a.flag[a.vb + v];
+      const int nv = __popc(segs);
+      const bool act = lane < nv && a.flag[a.vb + a.list[ch.vbase + lane]];
       if (__ballot_sync(kFull, act) == 0) continue;  // whole chunk inactive
     }
-    // exclusive prefix of degrees -> segment starts
-    int incl = d;
+    const bool valid = lane < total;
+    const unsigned below = segs & le;
+    const int seg = __popc(below) - 1;                   // vertex index in chunk
+    const int vstart = 31 - __clz(below | 1u);           // first lane of my vertex
+    const unsigned above = segs & ~le;
+    const int vend = above ? __ffs(above) - 1 : total;   // one past my last lane
+    const int vd = vend - vstart;
+    int lab = -1;
+    if (valid) lab = gather(a, ld_stream(a.col + start + lane));
+    const bool vote = valid && lab >= 0;
+    if (!vote) lab = -1;
+    // label frequency inside the vertex's lanes [P:231-232]
+    const unsigned maxlen = __reduce_max_sync(kFull, valid ? (unsigned)vd : 0u);
+    unsigned k = 0;
+    for (unsigned j = 0; j < maxlen; ++j) {
+      const int other = __shfl_sync(kFull, lab, (vstart + (int)j) & 31);
+      k += (j < (unsigned)vd && other == lab) ? 1u : 0u;
+    }
+    // segmented arg-max toward the segment's first lane
+    Best<VAR> b;
+    if (vote) b.observe(k, (unsigned)lab, a);
 #pragma unroll
     for (int s = 1; s < 32; s <<= 1) {
-      int x = __shfl_up_sync(kFull, incl, s);
-      if (lane >= s) incl += x;
+      const unsigned long long ok = __shfl_down_sync(kFull, b.key, s);
+      const unsigned ol = VAR == V_LLP ? __shfl_down_sync(kFull, b.lab, s) : 0u;
+      if (lane + s < vend) b.merge(ok, ol);
     }
-    const int start = incl - d;
-    const int total = __shfl_sync(kFull, incl, 31);
-    const unsigned segstarts = __reduce_or_sync(kFull, lane < nv ? (1u << start) : 0u);
-    const bool valid = lane < total;
-    const int seg = max(__popc(segstarts & (kFull >> (31 - lane))) - 1, 0);
-    const int64_t vo = __shfl_sync(kFull, o, seg);
-    const int vstart = __shfl_sync(kFull, start, seg);
-    const int vd = __shfl_sync(kFull, d, seg);
-    int lab = -1;
-    if (valid) {
-      const int u = ld_stream(a.col + vo + (lane - vstart));
-      lab = ld_label(a.R + u);
-    }
-    const bool vote = valid && (VAR != V_SEEDED || lab >= 0);
-    // vmask: lanes of this lane's vertex [P:230]; idle lanes form singleton groups
-    const unsigned vmask = valid ? ((vd == 32 ? kFull : ((1u << vd) - 1u)) << vstart) : (1u << lane);
-    const unsigned activemask = __ballot_sync(kFull, vote);  // [P:229]
-    const unsigned key = vote ? (unsigned)lab : kNoLabel;
-    const unsigned lmask = __match_any_sync(kFull, key) & vmask & activemask;  // [P:231]
-    const unsigned k = __popc(lmask);                                           // [P:232]
-    unsigned bestlab;
-    if (VAR == V_LLP) {
-      const unsigned long long sk = vote ? score_key<VAR>(k, (unsigned)lab, a) : 0ull;
-      const unsigned hi = (unsigned)(sk >> 32), lo = (unsigned)sk;
-      const unsigned mhi = __reduce_max_sync(vmask, hi);
-      const unsigned mlo = __reduce_max_sync(vmask, (vote && hi == mhi) ? lo : 0u);
-      bestlab = __reduce_min_sync(vmask, (vote && hi == mhi && lo == mlo) ? (unsigned)lab : kNoLabel);
-    } else {
-      const unsigned cnt = vote ? k : 0u;
-      const unsigned maxc = __reduce_max_sync(vmask, cnt);
-      bestlab = __reduce_min_sync(vmask, (vote && cnt == maxc) ? (unsigned)lab : kNoLabel);
-    }
-    if (lane == 0) ty.arcs += (unsigned long long)total;
-    // the first lane of each segment updates its vertex
-    const int vv = __shfl_sync(kFull, v, seg);
     if (valid && lane == vstart) {
-      const bool have = (activemask & vmask) != 0u;
-      update_vertex<VAR>(a, vv, vd, have, bestlab, ty);
+      const int v = a.list[ch.vbase + seg];
+      update_vertex<VAR>(a, v, vd, b.have(), b.label(), ty);
     }
   }
   tally_flush(ty, a.cnt);
 }
 
 // ---------------------------------------------------------------------------
-// mfl_mid: one warp per vertex (33..256 arcs), per-warp shared table of
-// 2*deg slots.  Labels of a 32-arc round are warp-aggregated with
-// match_any before the table insert (hot keys after communities form [P:130]).
-constexpr int kMidUnroll = 8;  // 8 x 32 = 256 arcs in flight per warp
-
+// mfl_mid: one warp per vertex (33..256 arcs, padded to a multiple of 4), one
+// or two 128-bit loads per lane cover the row; per-warp shared table of
+// pow2 >= 2*deg slots.
 template <int VAR>
 __global__ void __launch_bounds__(kMidBlock) mfl_mid(MflArgs a) {
-  __shared__ unsigned long long tabs[kMidBlock / 32][kMidSlots];
+  __shared__ __align__(16) unsigned long long tabs[kMidBlock / 32][kMidSlots];
+  __shared__ int s_never;  // mid tables never overflow
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  unsigned long long* tab = tabs[wid];
+  if (threadIdx.x == 0) s_never = 0;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
   Tally ty;
-  for (int i = gw; i < a.list_len; i += nwarps) {
-    const int v = a.list[i];
-    if (!a.dense && !a.flag[a.vb + v]) continue;
-    const int64_t o = a.off[v];
-    const int d = (int)(a.off[v + 1] - o);
-    const unsigned tsz = 2u * (unsigned)d;
-    for (unsigned j = lane; j < tsz; j += 32) tab[j] = kEmpty;
+  for (int i = gw; i < a.n_items; i += nwarps) {
+    const BinItem it = a.items[i];
+    if (!a.dense && !a.flag[a.vb + it.v]) continue;
+    const unsigned tsz = max(64u, 1u << (32 - __clz(2u * (unsigned)it.d - 1u)));
+    const Table tab{tabs[wid], tsz};
+    tab.clear(lane, 32);
+    int4 u0 = make_int4(-1, -1, -1, -1), u1 = u0;
+    if (4 * lane < it.d) u0 = ld_stream4(a.col + it.start + 4 * lane);
+    if (128 + 4 * lane < it.d) u1 = ld_stream4(a.col + it.start + 128 + 4 * lane);
+    int l[8];
+    l[0] = gather(a, u0.x); l[1] = gather(a, u0.y); l[2] = gather(a, u0.z); l[3] = gather(a, u0.w);
+    l[4] = gather(a, u1.x); l[5] = gather(a, u1.y); l[6] = gather(a, u1.z); l[7] = gather(a, u1.w);
     __syncwarp();
-    Best b{0ull, kNoLabel};
-    for (int base = 0; base < d; base += 32 * kMidUnroll) {
-      int u[kMidUnroll], lab[kMidUnroll];
+    Best<VAR> b;
+    const int nj = it.d > 128 ? 8 : 4;  // warp-uniform
 #pragma unroll
-      for (int j = 0; j < kMidUnroll; ++j) {
-        const int idx = base + j * 32 + lane;
-        u[j] = idx < d ? ld_stream(a.col + o + idx) : -1;
-      }
-#pragma unroll
-      for (int j = 0; j < kMidUnroll; ++j) lab[j] = u[j] >= 0 ? ld_label(a.R + u[j]) : -1;
-#pragma unroll
-      for (int j = 0; j < kMidUnroll; ++j) {
-        if (base + j * 32 >= d) break;  // warp-uniform
-        const bool vote = u[j] >= 0 && lab[j] >= 0;
-        const unsigned key = vote ? (unsigned)lab[j] : kNoLabel;
-        const unsigned m = __match_any_sync(kFull, key);
-        if (vote && lane == __ffs(m) - 1) {
-          const unsigned cnt = ht_add(tab, tsz, (unsigned)lab[j], __popc(m), tsz);
-          best_update(b, score_key<VAR>(cnt, (unsigned)lab[j], a), (unsigned)lab[j]);
-        }
-      }
-    }
-    b = warp_best(b);
-    if (lane == 0) {
-      ty.arcs += (unsigned long long)d;
-      update_vertex<VAR>(a, v, d, b.key != 0ull, b.lab, ty);
-    }
+    for (int j = 0; j < 8; ++j)
+      if (j < nj) warp_insert<VAR, false>(a, tab, tsz, l[j], l[j] >= 0, b, &s_never);
+    b.warp_reduce();
+    if (lane == 0) update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
     __syncwarp();
   }
   tally_flush(ty, a.cnt);
 }
 
 // ---------------------------------------------------------------------------
-// Block-per-vertex counting shared by mfl_high and mfl_huge.
-template <int VAR, int BLOCK, int UNROLL>
-__device__ __forceinline__ bool block_count(const MflArgs& a, int64_t o, int d, unsigned long long* tab,
-                                            unsigned tsz, unsigned max_probe, volatile int* overflow,
-                                            Best& b) {
-  const int lane = threadIdx.x & 31;
-  for (int base = 0; base < d; base += BLOCK * UNROLL) {
-    int u[UNROLL], lab[UNROLL];
-#pragma unroll
-    for (int j = 0; j < UNROLL; ++j) {
-      const int idx = base + j * BLOCK + (int)threadIdx.x;
-      u[j] = idx < d ? ld_stream(a.col + o + idx) : -1;
-    }
-#pragma unroll
-    for (int j = 0; j < UNROLL; ++j) lab[j] = u[j] >= 0 ? ld_label(a.R + u[j]) : -1;
-#pragma unroll
-    for (int j = 0; j < UNROLL; ++j) {
-      const bool vote = u[j] >= 0 && lab[j] >= 0;
-      const unsigned key = vote ? (unsigned)lab[j] : kNoLabel;
-      const unsigned m = __match_any_sync(kFull, key);
-      if (vote && lane == __ffs(m) - 1) {
-        const unsigned cnt = ht_add(tab, tsz, (unsigned)lab[j], __popc(m), max_probe);
-        if (cnt == 0) {
-          *overflow = 1;
-        } else {
-          best_update(b, score_key<VAR>(cnt, (unsigned)lab[j], a), (unsigned)lab[j]);
-        }
-      }
-    }
-    if (overflow != nullptr && __any_sync(kFull, *overflow != 0)) return false;  // warp-uniform exit
-  }
-  return true;
+// Block-per-vertex counting of one row into `tab` (UNROLL 128-bit loads per
+// thread in flight).  Only labels of hash partition `part` of `nparts` vote
+// (multi-pass counting of rows with more distinct labels than the table
+// holds).  Stops early (warp-uniformly) once a label overflowed.
+__device__ __forceinline__ unsigned label_part(unsigned lab, unsigned nparts) {
+  return __umulhi(lab * 0x85EBCA77u + 0x165667B1u, nparts);
 }
 
-template <int BLOCK>
-__device__ __forceinline__ Best block_best(Best b) {
+template <int VAR, int BLOCK, int UNROLL, bool COUNT_NEW>
+__device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int d, const Table& tab,
+                                            unsigned max_probe, unsigned part, unsigned nparts,
+                                            const int32_t* stage_in, int32_t* stage_out,
+                                            volatile int* overflow, int* distinct, Best<VAR>& b) {
+  unsigned fresh = 0;
+  for (int base = 0; base < d; base += BLOCK * 4 * UNROLL) {
+    int lab[4 * UNROLL];
+    if (stage_in != nullptr) {
+      // labels of this row already gathered by an earlier pass (coalesced)
+#pragma unroll
+      for (int j = 0; j < UNROLL; ++j) {
+        const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
+        const int4 x = idx < d ? __ldcg((const int4*)(stage_in + idx)) : make_int4(-1, -1, -1, -1);
+        lab[4 * j + 0] = x.x; lab[4 * j + 1] = x.y; lab[4 * j + 2] = x.z; lab[4 * j + 3] = x.w;
+      }
+    } else {
+      int4 u[UNROLL];
+#pragma unroll
+      for (int j = 0; j < UNROLL; ++j) {
+        const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
+        u[j] = idx < d ? ld_stream4(a.col + start + idx) : make_int4(-1, -1, -1, -1);
+      }
+#pragma unroll
+      for (int j = 0; j < UNROLL; ++j) {
+        lab[4 * j + 0] = gather(a, u[j].x);
+        lab[4 * j + 1] = gather(a, u[j].y);
+        lab[4 * j + 2] = gather(a, u[j].z);
+        lab[4 * j + 3] = gather(a, u[j].w);
+        const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
+        if (stage_out != nullptr && idx < d)
+          __stcg((int4*)(stage_out + idx), make_int4(lab[4 * j], lab[4 * j + 1], lab[4 * j + 2], lab[4 * j + 3]));
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < 4 * UNROLL; ++j) {
+      const bool vote = lab[j] >= 0 && (nparts == 1u || label_part((unsigned)lab[j], nparts) == part);
+      fresh += warp_insert<VAR, COUNT_NEW>(a, tab, max_probe, lab[j], vote, b, overflow);
+    }
+    if (__any_sync(kFull, *overflow != 0)) break;  // warp-uniform exit
+  }
+  if (COUNT_NEW && (threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
+}
+
+template <int VAR, int BLOCK>
+__device__ __forceinline__ Best<VAR> block_best(Best<VAR> b) {
   __shared__ unsigned long long rk[BLOCK / 32];
   __shared__ unsigned rl[BLOCK / 32];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  b = warp_best(b);
+  b.warp_reduce();
   if (lane == 0) { rk[wid] = b.key; rl[wid] = b.lab; }
   __syncthreads();
   if (wid == 0) {
-    Best x{0ull, kNoLabel};
+    Best<VAR> x;
     if (lane < BLOCK / 32) { x.key = rk[lane]; x.lab = rl[lane]; }
-    x = warp_best(x);
+    x.warp_reduce();
     b = x;
   }
   return b;  // valid in thread 0
 }
 
-constexpr int kHighUnroll = 4;
-
-template <int VAR>
-__global__ void __launch_bounds__(kHighBlock) mfl_high(MflArgs a) {
-  extern __shared__ unsigned long long tab[];  // kHighSlots
-  Tally ty;
-  for (int i = blockIdx.x; i < a.list_len; i += gridDim.x) {
-    const int v = a.list[i];
-    if (!a.dense && !a.flag[a.vb + v]) continue;  // block-uniform
-    const int64_t o = a.off[v];
-    const int d = (int)(a.off[v + 1] - o);
-    const unsigned tsz = 2u * (unsigned)d;
-    for (unsigned j = threadIdx.x; j < tsz; j += kHighBlock) tab[j] = kEmpty;
-    __syncthreads();
-    Best b{0ull, kNoLabel};
-    block_count<VAR, kHighBlock, kHighUnroll>(a, o, d, tab, tsz, tsz, nullptr, b);
-    __syncthreads();
-    b = block_best<kHighBlock>(b);
-    if (threadIdx.x == 0) {
-      ty.arcs += (unsigned long long)d;
-      update_vertex<VAR>(a, v, d, b.key != 0ull, b.lab, ty);
-    }
-    __syncthreads();
+// Count the labels lab[off .. off + cnt) of stage (one hash partition of a
+// huge row) into `tab`; every non-negative label votes.
+template <int VAR, int BLOCK>
+__device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* stage, int cnt, const Table& tab,
+                                             unsigned max_probe, volatile int* overflow, int* distinct,
+                                             Best<VAR>& b) {
+  unsigned fresh = 0;
+  for (int j0 = 0; j0 < cnt; j0 += BLOCK) {
+    const int j = j0 + (int)threadIdx.x;
+    const int lab = j < cnt ? __ldcg(stage + j) : -1;
+    fresh += warp_insert<VAR, true>(a, tab, max_probe, lab, lab >= 0, b, overflow);
+    if (__any_sync(kFull, *overflow != 0)) break;
   }
-  tally_flush(ty, a.cnt);
+  if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
 }
 
-constexpr int kHugeUnroll = 4;
-
-template <int VAR>
-__global__ void __launch_bounds__(kHugeBlock) mfl_huge(MflArgs a) {
-  extern __shared__ unsigned long long tab[];  // kHugeSlots
-  __shared__ int s_i, s_over;
-  unsigned long long* gtab = a.ght + (int64_t)blockIdx.x * a.ght_slots;
+// mfl_block: one block per vertex.  SLOTS = shared table capacity (pow2).
+// OVF = the bin may hold rows with more distinct labels than the table holds
+// (largest bin).  Such rows are radix-partitioned by a hash of the label into
+// P parts (gather pass -> per-block staging buffer + shared histogram,
+// scatter pass -> partition-contiguous copy), then each part is counted
+// exactly in the shared table; the best over the parts is the row's MFL.  A
+// part whose labels still overflow (probe limit) restarts the row with 2P.
+// P comes from the row's distinct-label count of the previous iteration
+// (performance hint only; t = 1 of CLASSIC/LLP starts from the all-distinct
+// estimate).  This replaces the paper's global-memory fallback table [P:166]:
+// on B200 re-streaming a staged row costs less than clearing and probing a
+// per-row global table.
+template <int VAR, int BLOCK, int SLOTS, bool OVF, int UNROLL>
+__global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
+  extern __shared__ __align__(16) unsigned long long smem_tab[];  // SLOTS
+  __shared__ int s_i, s_over, s_distinct;
+  __shared__ int s_hist[OVF ? 256 : 1], s_cur[OVF ? 256 : 1];
   Tally ty;
-  for (;;) {
-    if (threadIdx.x == 0) {
-      s_i = (int)atomicAdd(&a.cnt->huge_next, 1ull);
-      s_over = 0;
-    }
-    __syncthreads();
-    const int i = s_i;
-    if (i >= a.list_len) break;
-    const int v = a.list[i];
-    if (!a.dense && !a.flag[a.vb + v]) { __syncthreads(); continue; }
-    const int64_t o = a.off[v];
-    const int d = (int)(a.off[v + 1] - o);
-    const unsigned tsz = min(2u * (unsigned)d, (unsigned)kHugeSlots);
-    for (unsigned j = threadIdx.x; j < tsz; j += kHugeBlock) tab[j] = kEmpty;
-    __syncthreads();
-    Best b{0ull, kNoLabel};
-    block_count<VAR, kHugeBlock, kHugeUnroll>(a, o, d, tab, tsz, kHugeProbe, &s_over, b);
-    __syncthreads();
-    if (s_over) {
-      // GlobalInsert [P:166]: exact recount of the whole neighbourhood in a
-      // per-block global table of 2*deg slots (labels never split between the
-      // two tables, so the shared-memory observations are discarded).
-      const unsigned gsz = 2u * (unsigned)d;
-      for (unsigned j = threadIdx.x; j < gsz; j += kHugeBlock) gtab[j] = kEmpty;
-      __syncthreads();
-      b = Best{0ull, kNoLabel};
-      block_count<VAR, kHugeBlock, kHugeUnroll>(a, o, d, gtab, gsz, gsz, nullptr, b);
+  int32_t* stageA = OVF ? a.stage + (int64_t)blockIdx.x * 2 * a.stage_stride : nullptr;
+  int32_t* stageB = OVF ? stageA + a.stage_stride : nullptr;
+  for (int i0 = blockIdx.x;; i0 += gridDim.x) {
+    if (OVF) {
+      if (threadIdx.x == 0) s_i = (int)atomicAdd(&a.cnt->work_next, 1ull);
       __syncthreads();
     }
-    b = block_best<kHugeBlock>(b);
-    if (threadIdx.x == 0) {
-      ty.arcs += (unsigned long long)d;
-      update_vertex<VAR>(a, v, d, b.key != 0ull, b.lab, ty);
+    const int i = OVF ? s_i : i0;
+    if (i >= a.n_items) break;
+    const BinItem it = a.items[i];
+    if (!a.dense && !a.flag[a.vb + it.v]) {
+      if (OVF) __syncthreads();
+      continue;
     }
+    const int d = it.d;
+    Best<VAR> b;
+    unsigned nparts = OVF ? max(1u, (unsigned)a.ovf_hint[i]) : 1u;
+    bool staged = false;  // stageA holds the row's gathered labels
+    if (OVF && threadIdx.x == 0) s_distinct = 0;
+    if (nparts == 1u) {
+      // single pass: gather + count (stage the labels if an overflow is possible)
+      const unsigned tsz = min(1u << (32 - __clz(2u * (unsigned)d - 1u)), (unsigned)SLOTS);
+      const Table tab{smem_tab, tsz};
+      if (threadIdx.x == 0) s_over = 0;
+      tab.clear(threadIdx.x, BLOCK);
+      __syncthreads();
+      const bool may_over = OVF && 2u * (unsigned)d > (unsigned)SLOTS;
+      block_count<VAR, BLOCK, UNROLL, OVF>(a, it.start, d, tab, may_over ? kHugeProbe : tsz, 0u, 1u, nullptr,
+                                           may_over ? stageA : nullptr, &s_over, &s_distinct, b);
+      __syncthreads();
+      const bool over = s_over != 0;
+      __syncthreads();
+      if (over) {
+        nparts = max(2u, ((unsigned)d + SLOTS / 2 - 1) / (SLOTS / 2));
+        nparts = min(nparts, 255u);
+        b = Best<VAR>();
+      }
+    }
+    if (OVF) {
+      while (nparts > 1u) {
+        // (a) histogram of partitions (gathering + staging the row if needed)
+        if (threadIdx.x < 256) s_hist[threadIdx.x] = 0;
+        if (threadIdx.x == 0) { s_over = 0; s_distinct = 0; }
+        __syncthreads();
+        for (int base = 0; base < d; base += BLOCK * 4) {
+          const int idx = base + (int)threadIdx.x * 4;
+          if (idx < d) {
+            int4 x;
+            if (staged) {
+              x = __ldcg((const int4*)(stageA + idx));
+            } else {
+              const int4 u = ld_stream4(a.col + it.start + idx);
+              x = make_int4(gather(a, u.x), gather(a, u.y), gather(a, u.z), gather(a, u.w));
+              __stcg((int4*)(stageA + idx), x);
+            }
+            if (x.x >= 0) atomicAdd(&s_hist[label_part((unsigned)x.x, nparts)], 1);
+            if (x.y >= 0) atomicAdd(&s_hist[label_part((unsigned)x.y, nparts)], 1);
+            if (x.z >= 0) atomicAdd(&s_hist[label_part((unsigned)x.z, nparts)], 1);
+            if (x.w >= 0) atomicAdd(&s_hist[label_part((unsigned)x.w, nparts)], 1);
+          }
+        }
+        staged = true;
+        __syncthreads();
+        // (b) exclusive scan -> cursors (one warp, nparts <= 255)
+        if (threadIdx.x < 32) {
+          int carry = 0;
+          for (int p0 = 0; p0 < (int)nparts; p0 += 32) {
+            const int p = p0 + (int)threadIdx.x;
+            const int h = p < (int)nparts ? s_hist[p] : 0;
+            int x = h;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+              const int y = __shfl_up_sync(kFull, x, o);
+              if ((int)threadIdx.x >= o) x += y;
+            }
+            if (p < (int)nparts) s_cur[p] = carry + x - h;
+            carry += __shfl_sync(kFull, x, 31);
+          }
+        }
+        __syncthreads();
+        // (c) scatter into partition-contiguous order
+        for (int base = 0; base < d; base += BLOCK * 4) {
+          const int idx = base + (int)threadIdx.x * 4;
+          if (idx < d) {
+            const int4 x = __ldcg((const int4*)(stageA + idx));
+            if (x.x >= 0) __stcg(stageB + atomicAdd(&s_cur[label_part((unsigned)x.x, nparts)], 1), x.x);
+            if (x.y >= 0) __stcg(stageB + atomicAdd(&s_cur[label_part((unsigned)x.y, nparts)], 1), x.y);
+            if (x.z >= 0) __stcg(stageB + atomicAdd(&s_cur[label_part((unsigned)x.z, nparts)], 1), x.z);
+            if (x.w >= 0) __stcg(stageB + atomicAdd(&s_cur[label_part((unsigned)x.w, nparts)], 1), x.w);
+          }
+        }
+        __syncthreads();
+        // (d) count each partition exactly (s_cur[p] now = end of part p)
+        b = Best<VAR>();
+        bool over = false;
+        for (unsigned p = 0; p < nparts && !over; ++p) {
+          const int end = s_cur[p];
+          const int cnt = s_hist[p];
+          const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * (unsigned)max(cnt, 1) - 1u))), (unsigned)SLOTS);
+          const Table tab{smem_tab, tsz};
+          tab.clear(threadIdx.x, BLOCK);
+          __syncthreads();
+          const unsigned probe = 2u * (unsigned)cnt <= (unsigned)SLOTS ? tsz : kHugeProbe;
+          count_staged<VAR, BLOCK>(a, stageB + (end - cnt), cnt, tab, probe, &s_over, &s_distinct, b);
+          __syncthreads();
+          over = s_over != 0;
+          __syncthreads();
+        }
+        if (!over) break;
+        nparts = min(nparts * 2u, 255u);  // a part overflowed: finer partitions (exact recount)
+      }
+      if (threadIdx.x == 0) {
+        // next iteration starts from the partitions this row's distinct labels
+        // need at load <= 1/2 (labels collapse over iterations [P:130])
+        const unsigned need = ((unsigned)s_distinct + SLOTS / 2 - 1) / (SLOTS / 2);
+        a.ovf_hint[i] = (uint8_t)min(max(need, 1u), 255u);
+      }
+    }
+    b = block_best<VAR, BLOCK>(b);
+    if (threadIdx.x == 0) update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty);
     __syncthreads();
   }
   tally_flush(ty, a.cnt);

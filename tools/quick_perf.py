@@ -19,3 +19,10 @@ for k in g.kernel_stats():
     if k['launches']:
         print(k['name'], k['launches'], round(k['ms'], 3), 'ms', round(k['bytes'] / max(k['ms'], 1e-9) / 1e6, 1), 'GB/s alg',
               round(k['arcs'] / max(k['ms'], 1e-9) / 1e6, 2), 'Garcs/s')
+# per-iteration kernel breakdown (profiled runs of 1..4 iterations, differences)
+prev = {}
+for t in range(1, 5):
+    g.run('classic', t, profile=True)
+    cur = {k['name']: k['ms'] for k in g.kernel_stats()}
+    print('iter', t, {k: round(cur[k] - prev.get(k, 0), 3) for k in cur if cur[k] - prev.get(k, 0) > 0})
+    prev = cur
