@@ -1,0 +1,358 @@
+#!/usr/bin/env python
+"""GLP label-propagation benchmark (BASELINE.json metric: LP edges/sec per
+iteration, GTEPS, and time-to-converge).
+
+One *step* = one complete ``glp_run`` of the north_star hot path on a
+device-resident graph: PickLabel, then synchronous MFL iterations (gather ->
+count -> arg-max -> update, active-vertex frontier, exact stop rule) until a
+fixed point, a two-cycle or the paper's 20 iterations [P:270].
+
+  value  = GTEPS = (arcs of the graph x iterations) / device time of the run
+           (the paper's "average elapsed time for one iteration" [P:355] as a
+           rate over the graph's edges; arcs = symmetrised CSR entries)
+  e2e    = the same metric through the public C ABI with HOST buffers:
+           glp_graph_create(host CSR) + glp_run + glp_labels_get(host) per step
+
+Default workload (N=1): RMAT scale-24, edge factor 16, classic LP
+(BASELINE.json configs[2], the north_star's roofline config).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload rmat24]
+  python bench.py --impl reference ...   # the CPU oracle arm (bounded sample)
+Under torchrun (N>1) the graph is 1-D vertex-partitioned across ranks with the
+NCCL label all-gather (strong scaling); rank 0 prints the JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "LP edges/sec per iteration (GTEPS) and time-to-converge"
+UNIT = "GTEPS"
+
+WORKLOADS = {
+    # name: (generator spec, variant, max_iters, gamma)
+    "rmat24": (dict(kind="rmat", scale=24, edge_factor=16, seed=1), "classic", 20, 0.0),
+    "sbm1m": (dict(kind="sbm", n=1_000_000, k=1000, m=20_000_000, mu=0.1, seed=42), "classic", 30, 0.0),
+    "taobao100m": (dict(kind="taobao", users=80_000_000, items=20_000_000, pairs=1_000_000_000, seed=7),
+                   "seeded", 20, 0.0),
+    "rmat24_llp": (dict(kind="rmat", scale=24, edge_factor=16, seed=1), "llp", 20, 1.0),
+    "karate": (dict(kind="karate"), "classic", 20, 0.0),
+}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            j = json.load(f)
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy bandwidth)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled every 200 ms while running."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.proc = None
+        self.path = None
+
+    def __enter__(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except (OSError, FileNotFoundError):
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if self.proc is None or not self.path or not os.path.exists(self.path):
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                smax = float(parts[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        os.unlink(self.path)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def make_graph(spec, device):
+    from glp_inputs import graphs
+    csr, seeds = graphs.make(spec["kind"], device=device, **{k: v for k, v in spec.items() if k != "kind"})
+    return csr, seeds
+
+
+def cpu_reference(csr_cpu, variant, seeds, gamma, iters_per_sample, reps, warmup=0):
+    """Time the CPU oracle (as it stands) on the host cores: `reps` samples of
+    `iters_per_sample` LP iterations from PickLabel."""
+    import oracle
+    threads = os.cpu_count() or 1
+    vid = {"classic": oracle.CLASSIC, "seeded": oracle.SEEDED, "llp": oracle.LLP}[variant]
+    times = []
+    for r in range(warmup + reps):
+        t0 = time.perf_counter()
+        res = oracle.run(csr_cpu, vid, iters_per_sample, seeds=None if seeds is None else seeds.cpu().numpy(),
+                         gamma=gamma, threads=threads)
+        dt = time.perf_counter() - t0
+        if r >= warmup:
+            times.append((dt, res.iterations))
+    tot_t = sum(t for t, _ in times)
+    tot_it = sum(i for _, i in times)
+    value = csr_cpu.nnz * tot_it / tot_t / 1e9 if tot_t > 0 else 0.0
+    return value, threads, tot_t / max(len(times), 1), tot_it
+
+
+def flush_l2(buf):
+    buf.fill_(1)  # 256 MB write > 126 MB L2
+
+
+def bench_gpu(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sigmod_yelhls21_b200 as glp
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    spec, variant, max_iters, gamma = WORKLOADS[args.workload]
+    if args.max_iters is not None:
+        max_iters = args.max_iters
+    dev = torch.device("cuda", local)
+    t_gen = time.perf_counter()
+    csr, seeds = make_graph(spec, dev)
+    torch.cuda.synchronize()
+    t_gen = time.perf_counter() - t_gen
+    n, nnz = csr.n, csr.nnz
+    stream = torch.cuda.current_stream()
+
+    # ---- partition (1-D vertex ranges; equal vertex counts) ----
+    kw = {}
+    off, col = csr.row_offsets, csr.col_idx
+    vb, ve = 0, n
+    if world > 1:
+        bounds = glp.glp_partition(n, world)
+        vb, ve = bounds[rank], bounds[rank + 1]
+        o0, o1 = int(off[vb]), int(off[ve])
+        off = (off[vb:ve + 1] - o0).contiguous()
+        col = col[o0:o1].contiguous()
+        uid = [glp.glp_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        kw = dict(rank=rank, nranks=world, nccl_unique_id=uid[0], v_begin=vb, v_end=ve)
+    g = glp.Graph(n=n, row_offsets=off, col_idx=col, device=local, stream=stream, **kw)
+    info = g.info()
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
+
+    def one_run(profile=False):
+        return g.run(variant, max_iters, seeds, gamma=gamma, profile=profile)
+
+    for _ in range(max(args.warmup, 0)):
+        one_run()
+    # ---- timed region: K steps, each bracketed by CUDA events on the run stream ----
+    step_ms, infos = [], []
+    kstats = {}
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            flush_l2(flush)
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            ri = one_run(profile=True)
+            e1.record(stream)
+            e1.synchronize()
+            step_ms.append(e0.elapsed_time(e1))
+            infos.append(ri)
+            for k in g.kernel_stats():
+                s = kstats.setdefault(k["name"], dict(ms=0.0, bytes=0.0, arcs=0.0, launches=0))
+                s["ms"] += k["ms"]
+                s["bytes"] += k["bytes"]
+                s["arcs"] += k["arcs"]
+                s["launches"] += k["launches"]
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    total_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    iters = infos[-1].iterations
+    arcs_total = nnz if world == 1 else None
+    if world > 1:
+        t = torch.tensor([csr.nnz], dtype=torch.int64, device=dev)
+        arcs_total = csr.nnz  # every rank generated the full graph
+    ms_per_step = total_ms / args.steps
+    value = arcs_total * sum(i.iterations for i in infos) / (total_ms / 1e3) / 1e9
+
+    # ---- roofline of the dominant kernel (algorithmic bytes / event time) ----
+    peak, peak_src = measured_peaks()
+    dom = max((k for k in kstats if kstats[k]["launches"] and k.startswith("mfl_")),
+              key=lambda k: kstats[k]["ms"], default=None)
+    roof = None
+    if dom:
+        s = kstats[dom]
+        achieved = s["bytes"] / (s["ms"] / 1e3) / 1e9  # GB/s
+        traffic = None
+        tfile = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tfile):
+            try:
+                traffic = json.load(open(tfile)).get(args.workload, {}).get(dom)
+            except (OSError, ValueError):
+                traffic = None
+        roof = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
+                "bytes_per_launch": s["bytes"] / s["launches"], "ms_per_launch": s["ms"] / s["launches"],
+                "share_of_step": round(s["ms"] / total_ms, 3) if world == 1 else None,
+                "kernels": {k: {"ms": round(v["ms"] / args.steps, 4), "launches": v["launches"] // args.steps,
+                                "GBps_alg": round(v["bytes"] / max(v["ms"], 1e-9) / 1e6, 1)}
+                            for k, v in kstats.items() if v["launches"]}}
+
+    out = None
+    if rank == 0:
+        st = g.iter_stats()
+        # whole-iteration roofline (SURVEY §8(d) model incl. 4n label first touch)
+        it_bytes = [4.0 * s["active_arcs"] + 8.0 * s["active_vertices"] + 4.0 * n + 4.0 * s["changed"] for s in st]
+        it1 = st[0] if st else None
+        out = {
+            "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
+            "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic",
+            "config": {"workload": args.workload, "generator": spec, "variant": variant, "gamma": gamma,
+                       "max_iters": max_iters, "n": n, "arcs": nnz, "parallelism": f"vertex-range x{world}",
+                       "l2": "inputs larger than L2 (2.1 GB arcs for rmat24) and a 256 MB L2 flush before every step",
+                       "graph_gen_s": round(t_gen, 2), "bins": info["bins"], "max_degree": info["max_degree"]},
+            "iterations": iters, "stop_reason": glp.STOP_NAMES[infos[-1].stop_reason],
+            "time_to_converge_ms": round(ms_per_step, 4),
+            "iteration_ms": [round(s["ms"], 4) for s in st],
+            "iteration_active_arcs": [s["active_arcs"] for s in st],
+            "iteration1_gteps": round(nnz / (it1["ms"] / 1e3) / 1e9, 2) if it1 else None,
+            "iteration1_hbm_frac": round(it_bytes[0] / (it1["ms"] / 1e3) / 1e9 / peak, 4) if it1 else None,
+            "scanned_arcs_gteps": round(sum(i.arcs_processed for i in infos) / (total_ms / 1e3) / 1e9, 3),
+            "roofline": roof,
+            "gpu_launches": int(sum(i.kernel_launches for i in infos)),
+            "clocks": clk.summary(),
+        }
+    # ---- e2e through the public C ABI with host buffers ----
+    if rank == 0 and world == 1 and not args.no_e2e:
+        off_h = csr.row_offsets.cpu().pin_memory()
+        col_h = csr.col_idx.cpu().pin_memory()
+        out_h = torch.empty(n, dtype=torch.int32).pin_memory()
+        e2e_ms, e2e_iters = [], 0
+        for r in range(1 + min(args.steps, 3)):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            g2 = glp.Graph(n=n, row_offsets=off_h, col_idx=col_h, stream=stream)
+            ri = g2.run(variant, max_iters, seeds, gamma=gamma)
+            glp.glp_labels_get(g2.handle, out_h)
+            dt = (time.perf_counter() - t0) * 1e3
+            g2.close()
+            if r > 0:
+                e2e_ms.append(dt)
+                e2e_iters += ri.iterations
+        out["e2e"] = {"value": round(nnz * e2e_iters / (sum(e2e_ms) / 1e3) / 1e9, 3), "unit": UNIT,
+                      "h2d_bytes_per_step": int((n + 1) * 8 + nnz * 4 + (0 if seeds is None else 4 * seeds.numel())),
+                      "d2h_bytes_per_step": int(4 * n), "ms_per_step": round(statistics.mean(e2e_ms), 3),
+                      "includes": "graph create (H2D copy, relayout) + run + labels D2H"}
+    # ---- CPU baseline: the oracle on a bounded sample of the same workload ----
+    if rank == 0 and world == 1 and not args.no_cpu:
+        csr_cpu = csr.to("cpu")
+        samp_iters = 1 if nnz > 50_000_000 else max_iters
+        v, cores, sec, its = cpu_reference(csr_cpu, variant, seeds, gamma, samp_iters, reps=1)
+        out["cpu_baseline"] = {"value": round(v, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
+                               "sample": f"{args.workload}: first {its} LP iteration(s) from PickLabel, "
+                                         f"oracle/glp_oracle.c OpenMP over {cores} threads, {sec:.1f} s"}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    g.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def bench_reference(args):
+    """--impl reference: the CPU oracle (as it stands) on the same workload."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import torch
+    spec, variant, max_iters, gamma = WORKLOADS[args.workload]
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    csr, seeds = make_graph(spec, dev)
+    csr_cpu = csr.to("cpu")
+    seeds = None if seeds is None else seeds.cpu()
+    samp = 1 if csr.nnz > 50_000_000 else max_iters
+    v, cores, sec, its = cpu_reference(csr_cpu, variant, seeds, gamma, samp, reps=args.steps, warmup=args.warmup)
+    out = {"metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": round(sec * 1e3, 2), "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic", "impl": "reference",
+           "config": {"workload": args.workload, "generator": spec, "variant": variant, "gamma": gamma,
+                      "n": csr.n, "arcs": csr.nnz},
+           "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
+                            "sample": f"each step = first {samp} LP iteration(s) of {args.workload} from PickLabel"},
+           "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="glp", choices=["glp", "reference"])
+    ap.add_argument("--workload", default="rmat24", choices=sorted(WORKLOADS))
+    ap.add_argument("--max-iters", type=int, default=None)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        bench_reference(args)
+    else:
+        bench_gpu(args)
+
+
+if __name__ == "__main__":
+    main()

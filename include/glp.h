@@ -122,6 +122,7 @@ typedef struct {
   int64_t changed_last;        /* changed_t of the last iteration               */
   int64_t arcs_processed;      /* sum over iterations of scanned arcs           */
   double elapsed_ms;           /* device time of the run (CUDA events)          */
+  int64_t kernel_launches;     /* CUDA kernels the run launched                 */
 } glp_run_info;
 
 /* Per-iteration statistics of the last run (host copies). */

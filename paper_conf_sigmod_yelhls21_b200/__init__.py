@@ -59,7 +59,7 @@ class glp_params(ctypes.Structure):
 class glp_run_info(ctypes.Structure):
     _fields_ = [("iterations", ctypes.c_int32), ("stop_reason", ctypes.c_int32),
                 ("changed_last", ctypes.c_int64), ("arcs_processed", ctypes.c_int64),
-                ("elapsed_ms", ctypes.c_double)]
+                ("elapsed_ms", ctypes.c_double), ("kernel_launches", ctypes.c_int64)]
 
 
 class glp_iter_stat(ctypes.Structure):
@@ -211,7 +211,7 @@ def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, 
                        ctypes.byref(prm), ctypes.byref(info)))
     return dict(iterations=info.iterations, stop_reason=info.stop_reason,
                 changed_last=info.changed_last, arcs_processed=info.arcs_processed,
-                elapsed_ms=info.elapsed_ms)
+                elapsed_ms=info.elapsed_ms, kernel_launches=info.kernel_launches)
 
 
 def glp_labels_get(handle, out: torch.Tensor) -> torch.Tensor:
@@ -268,6 +268,7 @@ class RunInfo:
     changed_last: int
     arcs_processed: int
     elapsed_ms: float
+    kernel_launches: int
 
     @property
     def stop(self) -> str:

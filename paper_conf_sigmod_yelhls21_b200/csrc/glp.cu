@@ -390,6 +390,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
 struct Pending {
   int kid;
   cudaEvent_t a, b;
+  int t;  // iteration of the launch
 };
 
 cudaEvent_t pool_event(glp_graph* g, size_t& used) {
@@ -416,7 +417,7 @@ void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t&
   f();
   CK(cudaGetLastError());
   CK(cudaEventRecord(b, g->stream));
-  pend.push_back({kid, a, b});
+  pend.push_back({kid, a, b, g->cur_t});
 }
 
 // ---------------------------------------------------------------- run
@@ -477,6 +478,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   cudaStream_t s = g->stream;
   const int ga = g->grid_aux;
   // PickLabel
+  g->init_launches = 1;
   k_init_labels<<<ga, 256, 0, s>>>(g->L[0], g->L[1], g->npad, variant == GLP_VARIANT_SEEDED);
   CK(cudaGetLastError());
   CK(cudaMemsetAsync(g->so, 0x80, std::max<int64_t>(g->nl, 1) * sizeof(int2), s));  // stamp = INT_MIN-ish
@@ -493,12 +495,14 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     }
     CK(cudaMemcpyAsync(g->d_seeds, seeds, n_seeds * sizeof(int32_t), cudaMemcpyHostToDevice, s));
     k_init_seeds<<<ga, 256, 0, s>>>(g->d_seeds, n_seeds, g->L[0], g->L[1], g->is_seed, g->so, g->vb, g->ve);
+    g->init_launches += 1;
     CK(cudaGetLastError());
   }
   if (variant == GLP_VARIANT_LLP) {
     // V[l] = #{w : L_0[w] = l} = 1 for every l (L_0[v] = v)
     CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
     k_hist<<<ga, 256, 0, s>>>(g->L[0], g->n, g->V);
+    g->init_launches += 1;
     CK(cudaGetLastError());
   }
   if (g->n_huge) {
@@ -516,6 +520,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     // frontier of t = 1 is N(S) (+ S): push from the seeds (stamped t = 0)
     if (use_frontier) {
       k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, 0, g->flag[fb]);
+      g->init_launches += 1;
       CK(cudaGetLastError());
       g->flag_clean[fb] = false;
       if (g->nranks > 1) nccl_merge_flags(g, g->flag[fb]);
@@ -533,13 +538,14 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   // drain profiled launches (stream must be synchronised); counters attach
   // algorithmic bytes to the MFL kernels (SURVEY §8(d) model)
   auto drain = [&](bool with_counters) {
+    const int cur_t = g->cur_t;
     for (auto& pe : pend) {
       float kms = 0;
       CK(cudaEventElapsedTime(&kms, pe.a, pe.b));
       KStat& ks = g->kstats[pe.kid];
       ks.launches += 1;
       ks.ms += kms;
-      if (with_counters && pe.kid < 4) {
+      if (with_counters && pe.kid < 4 && pe.t == cur_t) {
         const Counters& c = g->h_cnt[pe.kid];
         ks.arcs += (double)c.arcs;
         // 4 B/arc (col_idx) + 8 B/active vertex (row offsets) + 4 B/changed label
@@ -552,20 +558,18 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   int32_t iters = 0;
   int reason = GLP_STOP_MAX_ITERS;
   int64_t changed_last = 0, arcs_total = 0;
+  int64_t launches = 0;  // kernels of this run (excluding memsets/copies)
   for (int32_t t = 1; t <= max_iters; ++t) {
-    if (!pend.empty()) {  // profiled post-iteration kernels of t-1
-      CK(cudaStreamSynchronize(s));
-      drain(false);
-    }
-    used = 1;  // ev_run0 stays; everything else is recycled
     cudaEvent_t e0 = pool_event(g, used), e1 = pool_event(g, used);
     CK(cudaEventRecord(e0, s));
     CK(cudaMemsetAsync(g->d_cnt, 0, 4 * sizeof(Counters), s));
+    g->cur_t = t;
     MflArgs a;
     memset(&a, 0, sizeof(a));
     a.col = g->col2; a.R = g->L[rb]; a.W = g->L[1 - rb]; a.so = g->so;
     a.V = g->V; a.is_seed = g->is_seed; a.flag = g->flag[fb];
     a.vb = g->vb; a.gamma = p.gamma; a.t = t; a.dense = dense ? 1 : 0;
+    launches += (g->n_huge > 0) + (g->n_high > 0) + (g->n_mid > 0) + (g->n_chunks > 0);
     switch (variant) {
       case GLP_VARIANT_CLASSIC: launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       case GLP_VARIANT_SEEDED: launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
@@ -594,7 +598,10 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     float ms = 0;
     CK(cudaEventElapsedTime(&ms, e0, e1));
     st.ms = ms;
+    // every kernel launched so far has completed: drain the profile events
+    // (this iteration's MFL kernels and the previous iteration's push/hist)
     drain(true);
+    used = 1;  // ev_run0 stays; everything else is recycled
     iters = t;
     changed_last = st.changed;
     arcs_total += st.active_arcs;
@@ -608,6 +615,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     if (!stop && use_frontier)
       next_dense = (double)tot.chdeg * (double)p.dense_divisor > (double)g->nnz_global;
     if (!stop && !next_dense) {
+      launches += 1;
       timed(g, prof, 4, pend, used, [&] {
         k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, g->flag[nf]);
         if (g->nranks > 1) nccl_merge_flags(g, g->flag[nf]);
@@ -619,6 +627,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       g->flag_clean[fb] = true;
     }
     if (!stop && variant == GLP_VARIANT_LLP) {
+      launches += 1;
       timed(g, prof, 5, pend, used, [&] {
         CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
         k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb], g->n, g->V);
@@ -647,6 +656,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     info->changed_last = changed_last;
     info->arcs_processed = arcs_total;
     info->elapsed_ms = run_ms;
+    info->kernel_launches = launches + g->init_launches;
   }
 }
 

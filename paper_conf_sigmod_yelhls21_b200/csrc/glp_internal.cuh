@@ -162,6 +162,8 @@ struct glp_graph {
   int grid_low = 0, grid_mid = 0, grid_high = 0, grid_huge = 0, grid_aux = 0;
 
   int cur = 0;  // index of L holding the result of the last run
+  int cur_t = 0;  // iteration being launched (profiling)
+  int64_t init_launches = 0;
   bool has_run = false;
   std::vector<glp_iter_stat> iter_stats;
   std::vector<glp::KStat> kstats;

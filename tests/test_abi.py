@@ -36,7 +36,7 @@ def test_struct_layout_matches_header():
     # sizes the C side checks (glp_params.struct_size) and the ctypes mirror
     assert ctypes.sizeof(glp.glp_params) == 64
     assert ctypes.sizeof(glp.glp_csr) == 56
-    assert ctypes.sizeof(glp.glp_run_info) == 32
+    assert ctypes.sizeof(glp.glp_run_info) == 40
     assert ctypes.sizeof(glp.glp_iter_stat) == 48
 
 
