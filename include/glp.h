@@ -113,7 +113,10 @@ typedef struct {
                                   (glp_kernel_stats); default 0                */
   int32_t dense_divisor;       /* go dense when sum_{changed} deg > nnz/this;
                                   0 = default (4)                              */
-  int32_t reserved[7];
+  int32_t debug_pred_cap;      /* testing only: clamp each row's predicted
+                                  distinct-label count (forces the overflow /
+                                  re-queue paths; results are unchanged); 0 off */
+  int32_t reserved[6];
 } glp_params;
 
 typedef struct {

@@ -53,7 +53,8 @@ class glp_params(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_uint32), ("gamma", ctypes.c_double),
                 ("frontier", ctypes.c_int32), ("stop_on_2cycle", ctypes.c_int32),
                 ("validate", ctypes.c_int32), ("profile", ctypes.c_int32),
-                ("dense_divisor", ctypes.c_int32), ("reserved", ctypes.c_int32 * 7)]
+                ("dense_divisor", ctypes.c_int32), ("debug_pred_cap", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 6)]
 
 
 class glp_run_info(ctypes.Structure):
@@ -120,7 +121,8 @@ def _check(st: int):
 
 
 def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = True,
-                validate: bool = True, profile: bool = False, dense_divisor: int = 0) -> glp_params:
+                validate: bool = True, profile: bool = False, dense_divisor: int = 0,
+                debug_pred_cap: int = 0) -> glp_params:
     p = glp_params()
     p.struct_size = ctypes.sizeof(glp_params)
     p.gamma = float(gamma)
@@ -129,6 +131,7 @@ def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = T
     p.validate = int(bool(validate))
     p.profile = int(bool(profile))
     p.dense_divisor = int(dense_divisor)
+    p.debug_pred_cap = int(debug_pred_cap)
     return p
 
 
@@ -196,7 +199,7 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
 
 def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, gamma: float = 0.0,
             frontier: int = -1, stop_on_2cycle: bool = True, profile: bool = False,
-            dense_divisor: int = 0) -> dict:
+            dense_divisor: int = 0, debug_pred_cap: int = 0) -> dict:
     import numpy as np
     lib = load_library()
     sd = None
@@ -206,7 +209,7 @@ def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, 
         ns = int(sd.size)
     info = glp_run_info()
     prm = make_params(gamma=gamma, frontier=frontier, stop_on_2cycle=stop_on_2cycle, profile=profile,
-                      dense_divisor=dense_divisor)
+                      dense_divisor=dense_divisor, debug_pred_cap=debug_pred_cap)
     _check(lib.glp_run(handle, int(variant), int(max_iters), None if sd is None else sd.ctypes.data, ns,
                        ctypes.byref(prm), ctypes.byref(info)))
     return dict(iterations=info.iterations, stop_reason=info.stop_reason,

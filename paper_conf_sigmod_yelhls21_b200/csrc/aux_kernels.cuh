@@ -86,6 +86,17 @@ __global__ void k_relayout(const int64_t* __restrict__ off, const int32_t* __res
   }
 }
 
+// Predicted distinct labels of each row at t = 1 (performance hint only).
+__global__ void k_init_pred(const BinItem* __restrict__ rows, int32_t n_rows, unsigned* __restrict__ pred0,
+                            unsigned* __restrict__ pred1, unsigned seed_cap) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_rows; i += (int64_t)gridDim.x * blockDim.x) {
+    const unsigned d = (unsigned)rows[i].d;
+    const unsigned p = seed_cap ? max(1u, min(d, seed_cap)) : d;
+    pred0[i] = p;
+    pred1[i] = p;
+  }
+}
+
 // LLP: V[l] = #{w : L[w] = l} [P:119].
 __global__ void k_hist(const int32_t* __restrict__ L, int64_t n, int32_t* __restrict__ V) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {

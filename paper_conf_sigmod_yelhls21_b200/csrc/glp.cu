@@ -125,35 +125,34 @@ void free_graph(glp_graph* g) {
 }
 
 // ---------------------------------------------------------------- layout
-#define GLP_HIGH_KERNEL(VAR) mfl_block<VAR, kHighBlock, kHighSlots, false, kHighUnroll>
-#define GLP_HUGE_KERNEL(VAR) mfl_block<VAR, kHugeBlock, kHugeSlots, true, kHugeUnroll>
+#define GLP_M_KERNEL(VAR) mfl_block<VAR, kMBlock, kMSlots, false, kMUnroll, CLS_M>
+#define GLP_L_KERNEL(VAR) mfl_block<VAR, kLBlock, kLSlots, true, kLUnroll, CLS_L>
 
 // Degree bins, low-degree warp chunks and the bin-major arc copy col2
 // (DESIGN.md §Layout).  Host decides the order; a kernel moves the arcs.
 // off_h: host row offsets; off_d/col_d: the caller's CSR on the device.
 void build_layout(glp_graph* g, const int64_t* off_h, const int64_t* off_d, const int32_t* col_d) {
-  std::vector<int32_t> low, mid, high, huge;
+  std::vector<int32_t> low, rows;
   for (int b = 0; b < NBINS; ++b) g->bin_verts[b] = g->bin_arcs[b] = 0;
   int64_t maxd = 0;
   for (int64_t v = 0; v < g->nl; ++v) {
     const int64_t d = off_h[v + 1] - off_h[v];
     if (d >= ((int64_t)1 << 30)) fail(GLP_ERR_INVALID_GRAPH, "row degree >= 2^30 is not supported");
     maxd = std::max(maxd, d);
-    int b;
+    int b;  // reporting bins: 0 | 1-32 | 33-256 | 257-2048 | > 2048
     if (d == 0) b = BIN_ISO;
     else if (d <= kLowMax) { b = BIN_LOW; low.push_back((int32_t)v); }
-    else if (d <= kMidMax) { b = BIN_MID; mid.push_back((int32_t)v); }
-    else if (d <= kHighMax) { b = BIN_HIGH; high.push_back((int32_t)v); }
-    else { b = BIN_HUGE; huge.push_back((int32_t)v); }
+    else if (d <= 256) b = BIN_MID;
+    else if (d <= 2048) b = BIN_HIGH;
+    else b = BIN_HUGE;
+    if (d > kLowMax) rows.push_back((int32_t)v);
     g->bin_verts[b] += 1;
     g->bin_arcs[b] += d;
   }
   g->max_deg = maxd;
   auto deg = [&](int32_t v) { return off_h[v + 1] - off_h[v]; };
-  // largest rows first in the block-per-vertex bins (long rows start early)
-  auto by_deg = [&](int32_t a, int32_t b) { return deg(a) != deg(b) ? deg(a) > deg(b) : a < b; };
-  std::sort(huge.begin(), huge.end(), by_deg);
-  std::sort(high.begin(), high.end(), by_deg);
+  // degree-descending: long rows start first, and each row class is a prefix
+  std::sort(rows.begin(), rows.end(), [&](int32_t a, int32_t b) { return deg(a) != deg(b) ? deg(a) > deg(b) : a < b; });
   std::vector<int64_t> ioff(g->nl, 0);
   std::vector<int32_t> ideg(g->nl, 0);
   int64_t pos = 0;
@@ -193,22 +192,27 @@ void build_layout(glp_graph* g, const int64_t* off_h, const int64_t* off_d, cons
       pos += (deg(v) + 3) & ~(int64_t)3;
     }
   };
-  std::vector<BinItem> mid_i, high_i, huge_i;
-  place(mid, mid_i);
-  place(high, high_i);
-  place(huge, huge_i);
+  std::vector<BinItem> row_i;
+  place(rows, row_i);
   g->nnz2 = pos;
   if (pos >= ((int64_t)1 << 56)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
   g->n_low = (int32_t)low.size();
   g->n_chunks = (int32_t)chunks.size();
-  g->n_mid = (int32_t)mid_i.size();
-  g->n_high = (int32_t)high_i.size();
-  g->n_huge = (int32_t)huge_i.size();
+  g->n_rows = (int32_t)row_i.size();
+  g->n_gt256 = 0;
+  g->n_gt2048 = 0;
+  for (const BinItem& it : row_i) {
+    g->n_gt256 += it.d > 256;
+    g->n_gt2048 += it.d > 2048;
+  }
   g->low_list = upload(g, low);
   g->chunks = upload(g, chunks);
-  g->mid_items = upload(g, mid_i);
-  g->high_items = upload(g, high_i);
-  g->huge_items = upload(g, huge_i);
+  g->rows = upload(g, row_i);
+  g->pred[0] = dalloc<unsigned>(g, std::max<int32_t>(g->n_rows, 1));
+  g->pred[1] = dalloc<unsigned>(g, std::max<int32_t>(g->n_rows, 1));
+  g->redo_m = dalloc<int32_t>(g, std::max<int32_t>(g->n_rows, 1));
+  g->redo_l = dalloc<int32_t>(g, std::max<int32_t>(g->n_rows, 1));
+  g->d_sched = dalloc<Sched>(g, 1);
   g->ioff = upload(g, ioff);
   g->ideg = upload(g, ideg);
   g->col2 = dalloc<int32_t>(g, g->nnz2);
@@ -216,13 +220,6 @@ void build_layout(glp_graph* g, const int64_t* off_h, const int64_t* off_d, cons
   if (g->nl > 0 && g->nnz > 0) {
     k_relayout<<<g->sms * 8, 256, 0, g->stream>>>(off_d, col_d, g->ioff, g->nl, g->col2);
     CK(cudaGetLastError());
-  }
-  g->ovf_hint = dalloc<uint8_t>(g, std::max<int32_t>(g->n_huge, 1));
-  g->ovf_init.resize(g->n_huge);
-  for (int32_t i = 0; i < g->n_huge; ++i) {
-    // all-distinct estimate for t = 1: enough partitions for <= SLOTS/2 labels each
-    const int64_t p = (huge_i[i].d + kHugeSlots / 2 - 1) / (kHugeSlots / 2);
-    g->ovf_init[i] = (uint8_t)std::min<int64_t>(p, 255);
   }
 }
 
@@ -359,22 +356,22 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaEventCreate(&g->ev_b));
 
     const int sms = g->sms;
-    const int hs = kHighSlots * 8, us = kHugeSlots * 8;
-    CK(cudaFuncSetAttribute(GLP_HIGH_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, hs));
-    CK(cudaFuncSetAttribute(GLP_HIGH_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, hs));
-    CK(cudaFuncSetAttribute(GLP_HIGH_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, hs));
-    CK(cudaFuncSetAttribute(GLP_HUGE_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, us));
-    CK(cudaFuncSetAttribute(GLP_HUGE_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, us));
-    CK(cudaFuncSetAttribute(GLP_HUGE_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, us));
+    const int ms_ = kMSlots * 8, ls_ = kLSlots * 8;
+    CK(cudaFuncSetAttribute(GLP_M_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, ms_));
+    CK(cudaFuncSetAttribute(GLP_M_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, ms_));
+    CK(cudaFuncSetAttribute(GLP_M_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, ms_));
+    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, ls_));
+    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, ls_));
+    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, ls_));
     g->grid_low = grid_for(sms, (const void*)mfl_low<V_LLP>, kLowBlock, 0);
-    g->grid_mid = grid_for(sms, (const void*)mfl_mid<V_LLP>, kMidBlock, 0);
-    g->grid_high = grid_for(sms, (const void*)GLP_HIGH_KERNEL(V_LLP), kHighBlock, hs);
-    g->grid_huge = grid_for(sms, (const void*)GLP_HUGE_KERNEL(V_LLP), kHugeBlock, us);
+    g->grid_w = grid_for(sms, (const void*)mfl_warp<V_LLP>, kWBlock, 0);
+    g->grid_m = grid_for(sms, (const void*)GLP_M_KERNEL(V_LLP), kMBlock, ms_);
+    g->grid_l = grid_for(sms, (const void*)GLP_L_KERNEL(V_LLP), kLBlock, ls_);
     g->grid_aux = sms * 8;
-    if (g->n_huge > 0) {
-      g->grid_huge = std::min<int>(g->grid_huge, g->n_huge);
+    if (g->n_rows > 0) {
+      // L staging: two row-sized buffers per resident L block
       g->stage_stride = (g->max_deg + 3) & ~(int64_t)3;
-      g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 2 * g->grid_huge);
+      g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 2 * g->grid_l);
     }
     g->nnz_global = g->nnz;
     if (nranks > 1) nccl_init(g, dist->nccl_unique_id);
@@ -402,7 +399,7 @@ cudaEvent_t pool_event(glp_graph* g, size_t& used) {
   return g->ev_pool[used++];
 }
 
-const char* kKernelNames[] = {"mfl_low", "mfl_mid", "mfl_high", "mfl_huge", "push", "llp_hist", "exchange"};
+const char* kKernelNames[] = {"mfl_low", "mfl_warp", "mfl_block_m", "mfl_block_l", "push", "llp_hist", "exchange"};
 constexpr int kNumKernelNames = 7;
 
 template <class F>
@@ -422,36 +419,56 @@ void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t&
 
 // ---------------------------------------------------------------- run
 template <int VAR>
-void launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, size_t& used) {
+int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, size_t& used) {
   Counters* c = g->d_cnt;
-  if (g->n_huge) {
-    MflArgs b = a;
-    b.items = g->huge_items; b.n_items = g->n_huge; b.cnt = c + 3;
-    b.ovf_hint = g->ovf_hint; b.stage = g->stage; b.stage_stride = g->stage_stride;
-    timed(g, prof, 3, pend, used, [&] {
-      GLP_HUGE_KERNEL(VAR)<<<g->grid_huge, kHugeBlock, kHugeSlots * 8, g->stream>>>(b);
-    });
+  Sched* sc = g->d_sched;
+  int n = 0;
+  const size_t ms_ = kMSlots * 8, ls_ = kLSlots * 8;
+  MflArgs r = a;
+  r.items = g->rows; r.pred = g->pred[g->pb]; r.pred_next = g->pred[1 - g->pb];
+  r.stage = g->stage; r.stage_stride = g->stage_stride;
+  if (g->n_gt2048) {  // L, static: rows of class L (a prefix of deg > 2048)
+    MflArgs b = r;
+    b.n_items = g->n_gt2048; b.cnt = c + 3; b.work = &sc->work_l;
+    const int grid = std::min<int>(g->grid_l, g->n_gt2048);
+    timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<grid, kLBlock, ls_, g->stream>>>(b); });
+    ++n;
   }
-  if (g->n_high) {
-    MflArgs b = a;
-    b.items = g->high_items; b.n_items = g->n_high; b.cnt = c + 2;
-    const int grid = std::min<int>(g->grid_high, g->n_high);
-    timed(g, prof, 2, pend, used, [&] {
-      GLP_HIGH_KERNEL(VAR)<<<grid, kHighBlock, kHighSlots * 8, g->stream>>>(b);
-    });
+  if (g->n_gt256) {  // M, static; overflowing rows -> L redo list
+    MflArgs b = r;
+    b.n_items = g->n_gt256; b.cnt = c + 2; b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
+    const int grid = std::min<int>(g->grid_m, g->n_gt256);
+    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<grid, kMBlock, ms_, g->stream>>>(b); });
+    ++n;
   }
-  if (g->n_mid) {
-    MflArgs b = a;
-    b.items = g->mid_items; b.n_items = g->n_mid; b.cnt = c + 1;
-    const int grid = std::min<int>(g->grid_mid, (g->n_mid + kMidBlock / 32 - 1) / (kMidBlock / 32));
-    timed(g, prof, 1, pend, used, [&] { mfl_mid<VAR><<<grid, kMidBlock, 0, g->stream>>>(b); });
+  if (g->n_rows) {  // W: every row of class W; overflowing rows -> M redo list
+    MflArgs b = r;
+    b.n_items = g->n_rows; b.cnt = c + 1; b.redo_out = g->redo_m; b.redo_out_n = &sc->n_redo_m;
+    const int grid = std::min<int>(g->grid_w, (g->n_rows + kWBlock / 32 - 1) / (kWBlock / 32));
+    timed(g, prof, 1, pend, used, [&] { mfl_warp<VAR><<<grid, kWBlock, 0, g->stream>>>(b); });
+    ++n;
   }
   if (g->n_chunks) {
     MflArgs b = a;
     b.list = g->low_list; b.chunks = g->chunks; b.n_chunks = g->n_chunks; b.cnt = c + 0;
     const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock / 32 - 1) / (kLowBlock / 32));
     timed(g, prof, 0, pend, used, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, g->stream>>>(b); });
+    ++n;
   }
+  if (g->n_rows) {
+    // re-queued rows (their labels overflowed the smaller table): W -> M -> L.
+    // The redo launches read the queue length on the device and exit at once
+    // when it is empty.
+    MflArgs b = r;
+    b.mode = 1; b.cnt = c + 2; b.redo_in = g->redo_m; b.redo_in_n = &sc->n_redo_m;
+    b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
+    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<g->sms, kMBlock, ms_, g->stream>>>(b); });
+    MflArgs q = r;
+    q.mode = 1; q.cnt = c + 3; q.redo_in = g->redo_l; q.redo_in_n = &sc->n_redo_l; q.work = &sc->work_lr;
+    timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<g->grid_l, kLBlock, ls_, g->stream>>>(q); });
+    n += 2;
+  }
+  return n;
 }
 
 void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_t* seeds, int64_t n_seeds,
@@ -505,13 +522,14 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     g->init_launches += 1;
     CK(cudaGetLastError());
   }
-  if (g->n_huge) {
-    // t = 1 of CLASSIC/LLP has all-distinct labels: rows wider than the shared
-    // table start in the global table (performance hint only)
-    std::vector<uint8_t> h(g->ovf_init);
-    if (variant == GLP_VARIANT_SEEDED) std::fill(h.begin(), h.end(), 1);
-    CK(cudaMemcpyAsync(g->ovf_hint, h.data(), h.size(), cudaMemcpyHostToDevice, s));
-    CK(cudaStreamSynchronize(s));
+  if (g->n_rows) {
+    // predicted distinct labels per row for t = 1: deg (all labels distinct)
+    // for CLASSIC/LLP, at most the number of seeds for SEEDED
+    g->pb = 0;
+    k_init_pred<<<ga, 256, 0, s>>>(g->rows, g->n_rows, g->pred[0], g->pred[1],
+                                   variant == GLP_VARIANT_SEEDED ? (unsigned)std::min<int64_t>(n_seeds, 1 << 30) : 0u);
+    CK(cudaGetLastError());
+    g->init_launches += 1;
   }
   int rb = 0;  // R = L[rb], W = L[1-rb]
   int fb = 0;  // flags read this iteration
@@ -563,17 +581,18 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     cudaEvent_t e0 = pool_event(g, used), e1 = pool_event(g, used);
     CK(cudaEventRecord(e0, s));
     CK(cudaMemsetAsync(g->d_cnt, 0, 4 * sizeof(Counters), s));
+    CK(cudaMemsetAsync(g->d_sched, 0, sizeof(Sched), s));
     g->cur_t = t;
     MflArgs a;
     memset(&a, 0, sizeof(a));
     a.col = g->col2; a.R = g->L[rb]; a.W = g->L[1 - rb]; a.so = g->so;
     a.V = g->V; a.is_seed = g->is_seed; a.flag = g->flag[fb];
     a.vb = g->vb; a.gamma = p.gamma; a.t = t; a.dense = dense ? 1 : 0;
-    launches += (g->n_huge > 0) + (g->n_high > 0) + (g->n_mid > 0) + (g->n_chunks > 0);
+    a.pred_cap = p.debug_pred_cap > 0 ? (unsigned)p.debug_pred_cap : 0u;
     switch (variant) {
-      case GLP_VARIANT_CLASSIC: launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
-      case GLP_VARIANT_SEEDED: launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
-      default: launch_mfl<V_LLP>(g, a, prof, pend, used); break;
+      case GLP_VARIANT_CLASSIC: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
+      case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
+      default: launches += launch_mfl<V_LLP>(g, a, prof, pend, used); break;
     }
     if (g->nranks > 1) {
       timed(g, prof, 6, pend, used, [&] { nccl_exchange(g, g->L[1 - rb]); });
@@ -634,6 +653,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       });
     }
     g->iter_stats.push_back(st);
+    g->pb = 1 - g->pb;
     rb = 1 - rb;
     fb = nf;
     dense = next_dense;

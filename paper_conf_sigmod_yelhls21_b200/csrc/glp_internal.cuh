@@ -22,24 +22,44 @@
 
 namespace glp {
 
-// Degree bins (thresholds are compile-time: each kernel's shared-memory table
-// is sized for its bin).  low: packed warps (PAPER §4.2); mid: warp per vertex;
-// high/huge: block per vertex with a shared-memory hash table (PAPER §4.1).
-constexpr int kLowMax = 32;       // deg <= 32   -> mfl_low  (one warp, several vertices)
-constexpr int kMidMax = 256;      // deg <= 256  -> mfl_mid  (one warp, one vertex)
-constexpr int kHighMax = 2048;    // deg <= 2048 -> mfl_block<128 thr, 4096 slots>
-                                  // deg >  2048 -> mfl_block<1024 thr, 16384 slots,
-                                  //                 partitioned recount on overflow>
+// Degree bin of the packed-warp kernel (PAPER §4.2): deg <= 32.
+constexpr int kLowMax = 32;
 constexpr int kLowBlock = 256;
-constexpr int kMidBlock = 256;
-constexpr int kMidSlots = 2 * kMidMax;      // per-warp table slots (key+count u32), load <= 1/2
-constexpr int kHighBlock = 128;
-constexpr int kHighSlots = 2 * kHighMax;    // 32 KB table, load <= 1/2
-constexpr int kHighUnroll = 2;
-constexpr int kHugeBlock = 1024;
-constexpr int kHugeSlots = 16384;           // 128 KB table
-constexpr int kHugeUnroll = 2;
-constexpr int kHugeProbe = 32;              // probe limit before declaring overflow
+
+// Rows with deg > 32 are counted in shared-memory hash tables (PAPER §4.1).
+// Each iteration a row goes to one of three kernels by its *predicted*
+// distinct-label count `pred` (the exact count of its previous iteration;
+// deg at t = 1, when all labels are distinct) -- labels collapse as
+// communities form [P:130], so most rows migrate to the warp path:
+//   W  pred <= 256,  deg <= 16384 : one warp per row, 512-slot table per warp
+//   M  pred <= 2048, deg <= 65536 : one 128-thread block per row, 4096 slots
+//   L  otherwise                  : one 1024-thread block per row, 16384
+//                                   slots, hash-partitioned passes
+// A row whose labels overflow its table is re-queued to the next class in the
+// same iteration (exact recount), so `pred` only steers performance.
+constexpr unsigned kWPred = 256, kMPred = 2048;
+constexpr int kWMaxDeg = 16384, kMMaxDeg = 65536;
+constexpr int kWBlock = 256;
+constexpr int kWSlots = 512;
+constexpr int kMBlock = 128;
+constexpr int kMSlots = 4096;
+constexpr int kMUnroll = 2;
+constexpr int kLBlock = 1024;
+constexpr int kLSlots = 16384;
+constexpr int kLUnroll = 2;
+constexpr int kLProbe = 32;  // probe limit before declaring a partition overflowed
+enum RowClass { CLS_W = 0, CLS_M = 1, CLS_L = 2 };
+__host__ __device__ __forceinline__ int row_class(unsigned pred, int d) {
+  if (pred <= kWPred && d <= kWMaxDeg) return CLS_W;
+  if (pred <= kMPred && d <= kMMaxDeg) return CLS_M;
+  return CLS_L;
+}
+
+// Per-iteration scheduling state (reset with the counters).
+struct Sched {
+  unsigned n_redo_m, n_redo_l;      // rows re-queued to M / L this iteration
+  unsigned long long work_l, work_lr;  // dynamic work counters of L (static / redo)
+};
 
 // A low-degree chunk: up to 32 consecutive arcs of consecutive low-list
 // vertices.  st = arc start in col2 | (arc count << 56); bit i of segmask set
@@ -68,7 +88,7 @@ struct Counters {
   unsigned long long chdeg;     // sum of deg over changed vertices
   unsigned long long arcs;      // arcs scanned
   unsigned long long verts;     // vertices scanned
-  unsigned long long work_next; // dynamic work counter (huge bin)
+  unsigned long long pad0;
   unsigned long long pad[2];
 };
 
@@ -84,10 +104,18 @@ struct MflArgs {
   const int32_t* __restrict__ list;     // low bin: vertex list (local ids)
   const LowChunk* __restrict__ chunks;  // low bin
   int32_t n_chunks;
-  const BinItem* __restrict__ items;    // mid/high/huge bins
-  int32_t n_items;
-  uint8_t* __restrict__ ovf_hint;       // huge bin: hash partitions to start with
-  int32_t* __restrict__ stage;          // huge bin: per-block staged row labels
+  const BinItem* __restrict__ items;    // rows with deg > 32, degree-descending
+  int32_t n_items;                      // prefix of items this launch scans
+  const unsigned* __restrict__ pred;    // per row: predicted distinct labels (this iteration)
+  unsigned* __restrict__ pred_next;     // per row: distinct labels counted now (next iteration)
+  unsigned pred_cap;                    // testing: clamp predictions (0 = off)
+  int32_t mode;                         // 0: scan items by class, 1: redo list
+  const int32_t* __restrict__ redo_in;  // mode 1: rows to process
+  const unsigned* redo_in_n;
+  int32_t* __restrict__ redo_out;       // rows re-queued to the next class
+  unsigned* redo_out_n;
+  unsigned long long* work;             // dynamic fetch counter (L)
+  int32_t* __restrict__ stage;          // L: per-block staged row labels (2 x stride)
   int64_t stage_stride;
   Counters* cnt;
   int64_t vb;                           // global id of local row 0
@@ -134,11 +162,13 @@ struct glp_graph {
   int32_t* ideg = nullptr;  // [nl] degree of row v
   int32_t* low_list = nullptr;  int32_t n_low = 0;
   glp::LowChunk* chunks = nullptr;   int32_t n_chunks = 0;
-  glp::BinItem* mid_items = nullptr; int32_t n_mid = 0;
-  glp::BinItem* high_items = nullptr; int32_t n_high = 0;
-  glp::BinItem* huge_items = nullptr; int32_t n_huge = 0;
-  uint8_t* ovf_hint = nullptr;
-  std::vector<uint8_t> ovf_init;  // per-run initial hints (host)
+  glp::BinItem* rows = nullptr; int32_t n_rows = 0;  // deg > 32, degree-descending
+  int32_t n_gt256 = 0, n_gt2048 = 0;                 // prefixes with deg > 256 / > 2048
+  unsigned* pred[2] = {nullptr, nullptr};            // [n_rows], double-buffered per iteration
+  int pb = 0;                                        // pred[pb] is read this iteration
+  int32_t* redo_m = nullptr;                         // [n_rows]
+  int32_t* redo_l = nullptr;                         // [n_rows]
+  glp::Sched* d_sched = nullptr;
   int64_t bin_verts[glp::NBINS] = {0}, bin_arcs[glp::NBINS] = {0};
 
   // per-rank row bounds (all ranks), for the exchange
@@ -159,7 +189,7 @@ struct glp_graph {
   int64_t seeds_cap = 0;
 
   // launch geometry
-  int grid_low = 0, grid_mid = 0, grid_high = 0, grid_huge = 0, grid_aux = 0;
+  int grid_low = 0, grid_w = 0, grid_m = 0, grid_l = 0, grid_aux = 0;
 
   int cur = 0;  // index of L holding the result of the last run
   int cur_t = 0;  // iteration being launched (profiling)

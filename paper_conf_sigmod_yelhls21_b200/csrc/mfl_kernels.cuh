@@ -16,11 +16,13 @@
 //             32 lanes ("one-warp-multi-vertices" [P:227-234 §4.2]): lane
 //             masks from the chunk's segment-start bitmap, label frequency per
 //             segment, shuffle-tree arg-max per segment.
-//   mfl_mid   deg <= 256: one warp per vertex, per-warp shared-memory table.
-//   mfl_block deg > 256: one block per vertex with a shared-memory hash table
-//             ("SharedMemBigNodes" HT [P:132-182 §4.1]); the largest bin
-//             recounts rows whose distinct labels overflow the table in hash
-//             partitions (replacing GlobalInsert/GHT [P:166, P:182]).
+//   deg > 32: a row goes to one of three kernels by its predicted
+//             distinct-label count (glp_internal.cuh row_class):
+//   mfl_warp  W: one warp per row, per-warp shared-memory table;
+//   mfl_block M/L: one block per row with a shared-memory hash table
+//             ("SharedMemBigNodes" HT [P:132-182 §4.1]); L recounts rows whose
+//             distinct labels overflow the table in hash partitions
+//             (replacing GlobalInsert/GHT [P:166, P:182]).
 //
 // Exactness of the running arg-max (the paper's ht_score taken from the
 // atomicAdd return value [P:150-156]): a label's count only grows, and its
@@ -288,38 +290,55 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
 }
 
 // ---------------------------------------------------------------------------
-// mfl_mid: one warp per vertex (33..256 arcs, padded to a multiple of 4), one
-// or two 128-bit loads per lane cover the row; per-warp shared table of
-// pow2 >= 2*deg slots.
+// mfl_warp: one warp per row of class W (few distinct labels): per-warp shared
+// table of pow2 >= 2*pred slots (<= 512), two 128-bit loads per lane per
+// round (256 arcs in flight per warp), no block barriers.  Rows whose labels
+// overflow the table are re-queued to the block kernel M.
 template <int VAR>
-__global__ void __launch_bounds__(kMidBlock) mfl_mid(MflArgs a) {
-  __shared__ __align__(16) unsigned long long tabs[kMidBlock / 32][kMidSlots];
-  __shared__ int s_never;  // mid tables never overflow
+__global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
+  __shared__ __align__(16) unsigned long long tabs[kWBlock / 32][kWSlots];
+  __shared__ int s_over[kWBlock / 32];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  if (threadIdx.x == 0) s_never = 0;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
   Tally ty;
   for (int i = gw; i < a.n_items; i += nwarps) {
     const BinItem it = a.items[i];
+    const unsigned pred = a.pred_cap ? min(a.pred[i], a.pred_cap) : a.pred[i];
+    if (row_class(pred, it.d) != CLS_W) continue;
     if (!a.dense && !a.flag[a.vb + it.v]) continue;
-    const unsigned tsz = max(64u, 1u << (32 - __clz(2u * (unsigned)it.d - 1u)));
+    const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * max(pred, 1u) - 1u))), (unsigned)kWSlots);
     const Table tab{tabs[wid], tsz};
     tab.clear(lane, 32);
-    int4 u0 = make_int4(-1, -1, -1, -1), u1 = u0;
-    if (4 * lane < it.d) u0 = ld_stream4(a.col + it.start + 4 * lane);
-    if (128 + 4 * lane < it.d) u1 = ld_stream4(a.col + it.start + 128 + 4 * lane);
-    int l[8];
-    l[0] = gather(a, u0.x); l[1] = gather(a, u0.y); l[2] = gather(a, u0.z); l[3] = gather(a, u0.w);
-    l[4] = gather(a, u1.x); l[5] = gather(a, u1.y); l[6] = gather(a, u1.z); l[7] = gather(a, u1.w);
+    if (lane == 0) s_over[wid] = 0;
     __syncwarp();
     Best<VAR> b;
-    const int nj = it.d > 128 ? 8 : 4;  // warp-uniform
+    unsigned fresh = 0;
+    bool over = false;
+    for (int base = 0; base < it.d && !over; base += 256) {
+      int4 u0 = make_int4(-1, -1, -1, -1), u1 = u0;
+      if (base + 4 * lane < it.d) u0 = ld_stream4(a.col + it.start + base + 4 * lane);
+      if (base + 128 + 4 * lane < it.d) u1 = ld_stream4(a.col + it.start + base + 128 + 4 * lane);
+      int l[8];
+      l[0] = gather(a, u0.x); l[1] = gather(a, u0.y); l[2] = gather(a, u0.z); l[3] = gather(a, u0.w);
+      l[4] = gather(a, u1.x); l[5] = gather(a, u1.y); l[6] = gather(a, u1.z); l[7] = gather(a, u1.w);
+      const int nj = (it.d - base) > 128 ? 8 : 4;  // warp-uniform
 #pragma unroll
-    for (int j = 0; j < 8; ++j)
-      if (j < nj) warp_insert<VAR, false>(a, tab, tsz, l[j], l[j] >= 0, b, &s_never);
+      for (int j = 0; j < 8; ++j)
+        if (j < nj) fresh += warp_insert<VAR, true>(a, tab, tsz, l[j], l[j] >= 0, b, &s_over[wid]);
+      __syncwarp();
+      over = s_over[wid] != 0;
+    }
+    if (over) {
+      if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = i;
+      __syncwarp();
+      continue;
+    }
     b.warp_reduce();
-    if (lane == 0) update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
+    if (lane == 0) {
+      a.pred_next[i] = max(fresh, 1u);
+      update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
+    }
     __syncwarp();
   }
   tally_flush(ty, a.cnt);
@@ -411,63 +430,80 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
   if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
 }
 
-// mfl_block: one block per vertex.  SLOTS = shared table capacity (pow2).
-// OVF = the bin may hold rows with more distinct labels than the table holds
-// (largest bin).  Such rows are radix-partitioned by a hash of the label into
-// P parts (gather pass -> per-block staging buffer + shared histogram,
-// scatter pass -> partition-contiguous copy), then each part is counted
-// exactly in the shared table; the best over the parts is the row's MFL.  A
-// part whose labels still overflow (probe limit) restarts the row with 2P.
-// P comes from the row's distinct-label count of the previous iteration
-// (performance hint only; t = 1 of CLASSIC/LLP starts from the all-distinct
-// estimate).  This replaces the paper's global-memory fallback table [P:166]:
-// on B200 re-streaming a staged row costs less than clearing and probing a
-// per-row global table.
-template <int VAR, int BLOCK, int SLOTS, bool OVF, int UNROLL>
+// mfl_block: one block per row of class CLS (M or L).  mode 0 scans the
+// degree-sorted row prefix and takes the rows of its class; mode 1 takes the
+// rows another kernel re-queued this iteration.
+//   M (PART = false): table of pow2 >= 4*pred slots (<= SLOTS); a row whose
+//     labels overflow it is re-queued to L.
+//   L (PART = true): rows with more distinct labels than the table holds are
+//     radix-partitioned by a hash of the label into P parts (gather pass ->
+//     per-block staging buffer + shared histogram, scatter pass ->
+//     partition-contiguous copy), then each part is counted exactly in the
+//     shared table; the best over the parts is the row's MFL.  A part that
+//     still overflows (probe limit) restarts the row with 2P.  This replaces
+//     the paper's global-memory fallback table [P:166]: on B200 re-streaming a
+//     staged row costs less than clearing and probing a per-row global table.
+// Both record the row's exact distinct-label count as the next `pred`.
+template <int VAR, int BLOCK, int SLOTS, bool PART, int UNROLL, int CLS>
 __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
   extern __shared__ __align__(16) unsigned long long smem_tab[];  // SLOTS
   __shared__ int s_i, s_over, s_distinct;
-  __shared__ int s_hist[OVF ? 256 : 1], s_cur[OVF ? 256 : 1];
+  __shared__ int s_hist[PART ? 256 : 1], s_cur[PART ? 256 : 1];
   Tally ty;
-  int32_t* stageA = OVF ? a.stage + (int64_t)blockIdx.x * 2 * a.stage_stride : nullptr;
-  int32_t* stageB = OVF ? stageA + a.stage_stride : nullptr;
+  int32_t* stageA = PART ? a.stage + (int64_t)blockIdx.x * 2 * a.stage_stride : nullptr;
+  int32_t* stageB = PART ? stageA + a.stage_stride : nullptr;
+  const int n_redo = a.mode ? (int)*a.redo_in_n : 0;
   for (int i0 = blockIdx.x;; i0 += gridDim.x) {
-    if (OVF) {
-      if (threadIdx.x == 0) s_i = (int)atomicAdd(&a.cnt->work_next, 1ull);
+    int i;
+    if (PART) {  // dynamic fetch: row costs vary by orders of magnitude
+      if (threadIdx.x == 0) s_i = (int)atomicAdd(a.work, 1ull);
       __syncthreads();
+      const int k = s_i;
+      __syncthreads();
+      if (a.mode ? k >= n_redo : k >= a.n_items) break;
+      i = a.mode ? a.redo_in[k] : k;
+    } else {
+      if (a.mode ? i0 >= n_redo : i0 >= a.n_items) break;
+      i = a.mode ? a.redo_in[i0] : i0;
     }
-    const int i = OVF ? s_i : i0;
-    if (i >= a.n_items) break;
     const BinItem it = a.items[i];
-    if (!a.dense && !a.flag[a.vb + it.v]) {
-      if (OVF) __syncthreads();
-      continue;
+    const unsigned pred = a.pred_cap ? min(a.pred[i], a.pred_cap) : a.pred[i];
+    if (!a.mode) {
+      if (row_class(pred, it.d) != CLS) continue;              // block-uniform
+      if (!a.dense && !a.flag[a.vb + it.v]) continue;
     }
     const int d = it.d;
     Best<VAR> b;
-    unsigned nparts = OVF ? max(1u, (unsigned)a.ovf_hint[i]) : 1u;
+    if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; }
+    // a re-queued row overflowed a smaller table: its pred is stale
+    const unsigned est = a.mode ? (unsigned)d : max(pred, 1u);
+    unsigned nparts = PART ? max(1u, (min(est, (unsigned)d) + SLOTS / 2 - 1) / (SLOTS / 2)) : 1u;
     bool staged = false;  // stageA holds the row's gathered labels
-    if (OVF && threadIdx.x == 0) s_distinct = 0;
+    bool over = false;
     if (nparts == 1u) {
-      // single pass: gather + count (stage the labels if an overflow is possible)
-      const unsigned tsz = min(1u << (32 - __clz(2u * (unsigned)d - 1u)), (unsigned)SLOTS);
+      // single pass: gather + count (L: stage the labels if an overflow is possible)
+      const unsigned want = PART ? 2u * (unsigned)d : 4u * est;
+      const unsigned tsz = min(max(64u, 1u << (32 - __clz(want - 1u))), (unsigned)SLOTS);
       const Table tab{smem_tab, tsz};
-      if (threadIdx.x == 0) s_over = 0;
       tab.clear(threadIdx.x, BLOCK);
       __syncthreads();
-      const bool may_over = OVF && 2u * (unsigned)d > (unsigned)SLOTS;
-      block_count<VAR, BLOCK, UNROLL, OVF>(a, it.start, d, tab, may_over ? kHugeProbe : tsz, 0u, 1u, nullptr,
-                                           may_over ? stageA : nullptr, &s_over, &s_distinct, b);
+      const bool may_over = PART && 2u * (unsigned)d > (unsigned)SLOTS;
+      block_count<VAR, BLOCK, UNROLL, true>(a, it.start, d, tab, may_over ? kLProbe : tsz, 0u, 1u, nullptr,
+                                            may_over ? stageA : nullptr, &s_over, &s_distinct, b);
       __syncthreads();
-      const bool over = s_over != 0;
+      over = s_over != 0;
       __syncthreads();
-      if (over) {
-        nparts = max(2u, ((unsigned)d + SLOTS / 2 - 1) / (SLOTS / 2));
-        nparts = min(nparts, 255u);
-        b = Best<VAR>();
+      if (over && PART) {
+        nparts = min(max(2u, ((unsigned)d + SLOTS / 2 - 1) / (SLOTS / 2)), 255u);
+        over = false;
       }
     }
-    if (OVF) {
+    if (!PART && over) {
+      if (threadIdx.x == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = i;
+      continue;
+    }
+    if (PART) {
+      nparts = min(nparts, 255u);
       while (nparts > 1u) {
         // (a) histogram of partitions (gathering + staging the row if needed)
         if (threadIdx.x < 256) s_hist[threadIdx.x] = 0;
@@ -523,32 +559,29 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
         __syncthreads();
         // (d) count each partition exactly (s_cur[p] now = end of part p)
         b = Best<VAR>();
-        bool over = false;
-        for (unsigned p = 0; p < nparts && !over; ++p) {
+        bool pover = false;
+        for (unsigned p = 0; p < nparts && !pover; ++p) {
           const int end = s_cur[p];
           const int cnt = s_hist[p];
           const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * (unsigned)max(cnt, 1) - 1u))), (unsigned)SLOTS);
           const Table tab{smem_tab, tsz};
           tab.clear(threadIdx.x, BLOCK);
           __syncthreads();
-          const unsigned probe = 2u * (unsigned)cnt <= (unsigned)SLOTS ? tsz : kHugeProbe;
+          const unsigned probe = 2u * (unsigned)cnt <= (unsigned)SLOTS ? tsz : kLProbe;
           count_staged<VAR, BLOCK>(a, stageB + (end - cnt), cnt, tab, probe, &s_over, &s_distinct, b);
           __syncthreads();
-          over = s_over != 0;
+          pover = s_over != 0;
           __syncthreads();
         }
-        if (!over) break;
+        if (!pover) break;
         nparts = min(nparts * 2u, 255u);  // a part overflowed: finer partitions (exact recount)
-      }
-      if (threadIdx.x == 0) {
-        // next iteration starts from the partitions this row's distinct labels
-        // need at load <= 1/2 (labels collapse over iterations [P:130])
-        const unsigned need = ((unsigned)s_distinct + SLOTS / 2 - 1) / (SLOTS / 2);
-        a.ovf_hint[i] = (uint8_t)min(max(need, 1u), 255u);
       }
     }
     b = block_best<VAR, BLOCK>(b);
-    if (threadIdx.x == 0) update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty);
+    if (threadIdx.x == 0) {
+      a.pred_next[i] = max((unsigned)s_distinct, 1u);
+      update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty);
+    }
     __syncthreads();
   }
   tally_flush(ty, a.cnt);

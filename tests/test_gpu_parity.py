@@ -22,11 +22,12 @@ glp = pytest.importorskip("paper_conf_sigmod_yelhls21_b200")
 
 
 def gpu(csr, variant=0, max_iters=20, seeds=None, gamma=0.0, frontier=-1, on_device=True,
-        stop_on_2cycle=True, dense_divisor=0):
+        stop_on_2cycle=True, dense_divisor=0, debug_pred_cap=0):
     c = csr.to("cuda") if on_device else csr
     with glp.Graph(c) as g:
         info = g.run(variant, max_iters, seeds, gamma=gamma, frontier=frontier,
-                     stop_on_2cycle=stop_on_2cycle, dense_divisor=dense_divisor)
+                     stop_on_2cycle=stop_on_2cycle, dense_divisor=dense_divisor,
+                     debug_pred_cap=debug_pred_cap)
         lab = g.labels("cpu").numpy().copy()
         st = g.iter_stats()
     return lab, info, st
@@ -135,6 +136,16 @@ def test_bin_boundaries(degrees):
     assert_same_run(csr, 0, 15)
     assert_same_run(csr, 2, 6, gamma=0.5)
     assert_same_run(csr, 1, 15, seeds=[0, len(degrees) + 3])
+
+
+@pytest.mark.parametrize("cap", [1, 40, 300])
+def test_requeue_paths_exact(cap):
+    """Under-predicted distinct counts force every overflow / re-queue path
+    (W -> M -> L, partition retries); results must not change."""
+    for csr in [_degree_mix([70000, 20000, 5000, 3000, 1500, 600, 300, 100, 40], seed=3, extra_pairs=60000),
+                graphs.rmat(14, seed=5)]:
+        assert_same_run(csr, 0, 12, debug_pred_cap=cap)
+        assert_same_run(csr, 2, 5, gamma=0.25, debug_pred_cap=cap)
 
 
 def test_hub_with_few_labels_and_ties():

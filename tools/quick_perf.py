@@ -21,7 +21,7 @@ for k in g.kernel_stats():
               round(k['arcs'] / max(k['ms'], 1e-9) / 1e6, 2), 'Garcs/s')
 # per-iteration kernel breakdown (profiled runs of 1..4 iterations, differences)
 prev = {}
-for t in range(1, 5):
+for t in range(1, int(sys.argv[2]) + 1 if len(sys.argv) > 2 else 5):
     g.run('classic', t, profile=True)
     cur = {k['name']: k['ms'] for k in g.kernel_stats()}
     print('iter', t, {k: round(cur[k] - prev.get(k, 0), 3) for k in cur if cur[k] - prev.get(k, 0) > 0})
