@@ -74,6 +74,19 @@ __global__ void k_push(const int64_t* __restrict__ ioff, const int32_t* __restri
   }
 }
 
+// Sparse iterations: a low-degree chunk is active if any of its vertices is.
+__global__ void k_chunk_flags(const LowChunk* __restrict__ chunks, int32_t n_chunks,
+                              const int32_t* __restrict__ list, const uint8_t* __restrict__ flag, int64_t vb,
+                              uint8_t* __restrict__ cflag) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n_chunks; c += (int64_t)gridDim.x * blockDim.x) {
+    const LowChunk ch = chunks[c];
+    const int nv = __popc(ch.segmask);
+    uint8_t act = 0;
+    for (int j = 0; j < nv && !act; ++j) act = flag[vb + list[ch.vbase + j]];
+    cflag[c] = act ? 1 : 0;
+  }
+}
+
 // Build the bin-major arc copy: row v of the caller's CSR -> col2[ioff[v]...].
 __global__ void k_relayout(const int64_t* __restrict__ off, const int32_t* __restrict__ col,
                            const int64_t* __restrict__ ioff, int64_t nl, int32_t* __restrict__ col2) {

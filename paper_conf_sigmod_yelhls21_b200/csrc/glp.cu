@@ -204,9 +204,11 @@ void build_layout(glp_graph* g, const int64_t* off_h, const int64_t* off_d, cons
   for (const BinItem& it : row_i) {
     g->n_gt256 += it.d > 256;
     g->n_gt2048 += it.d > 2048;
+    g->n_ge8k += it.d >= 8192;
   }
   g->low_list = upload(g, low);
   g->chunks = upload(g, chunks);
+  g->cflag = dalloc<uint8_t>(g, std::max<int32_t>(g->n_chunks, 1));
   g->rows = upload(g, row_i);
   g->pred[0] = dalloc<unsigned>(g, std::max<int32_t>(g->n_rows, 1));
   g->pred[1] = dalloc<unsigned>(g, std::max<int32_t>(g->n_rows, 1));
@@ -425,33 +427,34 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   int n = 0;
   const size_t ms_ = kMSlots * 8, ls_ = kLSlots * 8;
   MflArgs r = a;
-  r.items = g->rows; r.pred = g->pred[g->pb]; r.pred_next = g->pred[1 - g->pb];
+  r.items = g->rows; r.big_prefix = g->n_ge8k; r.pred = g->pred[g->pb]; r.pred_next = g->pred[1 - g->pb];
   r.stage = g->stage; r.stage_stride = g->stage_stride;
   if (g->n_gt2048) {  // L, static: rows of class L (a prefix of deg > 2048)
     MflArgs b = r;
     b.n_items = g->n_gt2048; b.cnt = c + 3; b.work = &sc->work_l;
-    const int grid = std::min<int>(g->grid_l, g->n_gt2048);
+    const int grid = std::min<int>(g->grid_l, g->n_ge8k + (g->n_gt2048 - g->n_ge8k + 31) / 32);
     timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<grid, kLBlock, ls_, g->stream>>>(b); });
     ++n;
   }
   if (g->n_gt256) {  // M, static; overflowing rows -> L redo list
     MflArgs b = r;
     b.n_items = g->n_gt256; b.cnt = c + 2; b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
-    const int grid = std::min<int>(g->grid_m, g->n_gt256);
+    b.work = &sc->work_m;
+    const int grid = std::min<int>(g->grid_m, g->n_ge8k + (g->n_gt256 - g->n_ge8k + 31) / 32);
     timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<grid, kMBlock, ms_, g->stream>>>(b); });
     ++n;
   }
   if (g->n_rows) {  // W: every row of class W; overflowing rows -> M redo list
     MflArgs b = r;
     b.n_items = g->n_rows; b.cnt = c + 1; b.redo_out = g->redo_m; b.redo_out_n = &sc->n_redo_m;
-    const int grid = std::min<int>(g->grid_w, (g->n_rows + kWBlock / 32 - 1) / (kWBlock / 32));
+    const int grid = std::min<int>(g->grid_w, (g->n_rows + kWBlock - 1) / kWBlock);
     timed(g, prof, 1, pend, used, [&] { mfl_warp<VAR><<<grid, kWBlock, 0, g->stream>>>(b); });
     ++n;
   }
   if (g->n_chunks) {
     MflArgs b = a;
-    b.list = g->low_list; b.chunks = g->chunks; b.n_chunks = g->n_chunks; b.cnt = c + 0;
-    const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock / 32 - 1) / (kLowBlock / 32));
+    b.list = g->low_list; b.chunks = g->chunks; b.cflag = g->cflag; b.n_chunks = g->n_chunks; b.cnt = c + 0;
+    const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock - 1) / kLowBlock);
     timed(g, prof, 0, pend, used, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, g->stream>>>(b); });
     ++n;
   }
@@ -460,7 +463,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     // The redo launches read the queue length on the device and exit at once
     // when it is empty.
     MflArgs b = r;
-    b.mode = 1; b.cnt = c + 2; b.redo_in = g->redo_m; b.redo_in_n = &sc->n_redo_m;
+    b.mode = 1; b.cnt = c + 2; b.redo_in = g->redo_m; b.redo_in_n = &sc->n_redo_m; b.work = &sc->work_mr;
     b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
     timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<g->sms, kMBlock, ms_, g->stream>>>(b); });
     MflArgs q = r;
@@ -542,6 +545,10 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       CK(cudaGetLastError());
       g->flag_clean[fb] = false;
       if (g->nranks > 1) nccl_merge_flags(g, g->flag[fb]);
+      if (g->n_chunks) {
+        k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_list, g->flag[fb], g->vb, g->cflag);
+        g->init_launches += 1;
+      }
       dense = false;
     }
   }
@@ -638,7 +645,10 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       timed(g, prof, 4, pend, used, [&] {
         k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, g->flag[nf]);
         if (g->nranks > 1) nccl_merge_flags(g, g->flag[nf]);
+        if (g->n_chunks)
+          k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_list, g->flag[nf], g->vb, g->cflag);
       });
+      launches += g->n_chunks ? 1 : 0;
       g->flag_clean[nf] = false;
     }
     if (!dense && !g->flag_clean[fb]) {

@@ -58,7 +58,7 @@ __host__ __device__ __forceinline__ int row_class(unsigned pred, int d) {
 // Per-iteration scheduling state (reset with the counters).
 struct Sched {
   unsigned n_redo_m, n_redo_l;      // rows re-queued to M / L this iteration
-  unsigned long long work_l, work_lr;  // dynamic work counters of L (static / redo)
+  unsigned long long work_m, work_mr, work_l, work_lr;  // dynamic fetch counters (static / redo)
 };
 
 // A low-degree chunk: up to 32 consecutive arcs of consecutive low-list
@@ -103,9 +103,11 @@ struct MflArgs {
   const uint8_t* __restrict__ flag;     // [npad] frontier marks by global id (sparse)
   const int32_t* __restrict__ list;     // low bin: vertex list (local ids)
   const LowChunk* __restrict__ chunks;  // low bin
+  const uint8_t* __restrict__ cflag;    // low bin: chunk has an active vertex (sparse)
   int32_t n_chunks;
   const BinItem* __restrict__ items;    // rows with deg > 32, degree-descending
   int32_t n_items;                      // prefix of items this launch scans
+  int32_t big_prefix;                   // rows fetched one per ticket (longest rows)
   const unsigned* __restrict__ pred;    // per row: predicted distinct labels (this iteration)
   unsigned* __restrict__ pred_next;     // per row: distinct labels counted now (next iteration)
   unsigned pred_cap;                    // testing: clamp predictions (0 = off)
@@ -162,8 +164,10 @@ struct glp_graph {
   int32_t* ideg = nullptr;  // [nl] degree of row v
   int32_t* low_list = nullptr;  int32_t n_low = 0;
   glp::LowChunk* chunks = nullptr;   int32_t n_chunks = 0;
+  uint8_t* cflag = nullptr;          // [n_chunks] chunk activity (sparse iterations)
   glp::BinItem* rows = nullptr; int32_t n_rows = 0;  // deg > 32, degree-descending
   int32_t n_gt256 = 0, n_gt2048 = 0;                 // prefixes with deg > 256 / > 2048
+  int32_t n_ge8k = 0;                                // prefix with deg >= 8192
   unsigned* pred[2] = {nullptr, nullptr};            // [n_rows], double-buffered per iteration
   int pb = 0;                                        // pred[pb] is read this iteration
   int32_t* redo_m = nullptr;                         // [n_rows]

@@ -244,16 +244,28 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
   const unsigned le = kFull >> (31 - lane);  // lanes 0..lane
   Tally ty;
-  for (int c = gw; c < a.n_chunks; c += nwarps) {
-    const LowChunk ch = a.chunks[c];
+  // each warp takes 32 consecutive chunks at a time; in sparse iterations the
+  // inactive ones are skipped with one coalesced read of their chunk flags
+  for (int c0 = gw * 32; c0 < a.n_chunks; c0 += nwarps * 32) {
+    const int cl = c0 + lane;
+    LowChunk mine;
+    mine.st = 0ull; mine.vbase = 0; mine.segmask = 0u;
+    bool act = cl < a.n_chunks;
+    if (act) {
+      mine = a.chunks[cl];
+      if (!a.dense) act = a.cflag[cl] != 0;
+    }
+    unsigned todo = __ballot_sync(kFull, act);
+    while (todo) {
+    const int j = __ffs(todo) - 1;
+    todo &= todo - 1;
+    LowChunk ch;
+    ch.st = __shfl_sync(kFull, mine.st, j);
+    ch.vbase = __shfl_sync(kFull, mine.vbase, j);
+    ch.segmask = __shfl_sync(kFull, mine.segmask, j);
     const int64_t start = (int64_t)(ch.st & ((1ull << 56) - 1));
     const int total = (int)(ch.st >> 56);
     const unsigned segs = ch.segmask;
-    if (!a.dense) {
-      const int nv = __popc(segs);
-      const bool act = lane < nv && a.flag[a.vb + a.list[ch.vbase + lane]];
-      if (__ballot_sync(kFull, act) == 0) continue;  // whole chunk inactive
-    }
     const bool valid = lane < total;
     const unsigned below = segs & le;
     const int seg = __popc(below) - 1;                   // vertex index in chunk
@@ -285,6 +297,7 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       const int v = a.list[ch.vbase + seg];
       update_vertex<VAR>(a, v, vd, b.have(), b.label(), ty);
     }
+    }  // todo
   }
   tally_flush(ty, a.cnt);
 }
@@ -302,11 +315,36 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
   Tally ty;
-  for (int i = gw; i < a.n_items; i += nwarps) {
-    const BinItem it = a.items[i];
-    const unsigned pred = a.pred_cap ? min(a.pred[i], a.pred_cap) : a.pred[i];
-    if (row_class(pred, it.d) != CLS_W) continue;
-    if (!a.dense && !a.flag[a.vb + it.v]) continue;
+  // 32 rows per warp at a time: the class / frontier test of the batch is
+  // lane-parallel, then the warp processes the selected rows one by one
+  // rows are degree-sorted, so a warp's batch is strided across the list
+  // (lane l of warp w takes row base + l * nwarps + w) to balance long rows
+  for (int base = 0; base < a.n_items; base += nwarps * 32) {
+    const int il = base + lane * nwarps + gw;
+    BinItem mine;
+    mine.start = 0; mine.v = 0; mine.d = 0;
+    unsigned mpred = 0;
+    bool ok = il < a.n_items;
+    if (ok) {
+      mine = a.items[il];
+      const unsigned raw = a.pred[il];
+      mpred = a.pred_cap ? min(raw, a.pred_cap) : raw;
+      ok = row_class(mpred, mine.d) == CLS_W;
+      if (ok && !a.dense && !a.flag[a.vb + mine.v]) {
+        ok = false;
+        a.pred_next[il] = raw;  // inactive: carry the prediction forward
+      }
+    }
+    unsigned todo = __ballot_sync(kFull, ok);
+    while (todo) {
+    const int jl = __ffs(todo) - 1;
+    todo &= todo - 1;
+    const int i = base + jl * nwarps + gw;
+    BinItem it;
+    it.start = __shfl_sync(kFull, mine.start, jl);
+    it.v = __shfl_sync(kFull, mine.v, jl);
+    it.d = __shfl_sync(kFull, mine.d, jl);
+    const unsigned pred = __shfl_sync(kFull, mpred, jl);
     const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * max(pred, 1u) - 1u))), (unsigned)kWSlots);
     const Table tab{tabs[wid], tsz};
     tab.clear(lane, 32);
@@ -340,6 +378,7 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
       update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
     }
     __syncwarp();
+    }  // todo
   }
   tally_flush(ty, a.cnt);
 }
@@ -447,31 +486,54 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
 template <int VAR, int BLOCK, int SLOTS, bool PART, int UNROLL, int CLS>
 __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
   extern __shared__ __align__(16) unsigned long long smem_tab[];  // SLOTS
-  __shared__ int s_i, s_over, s_distinct;
+  __shared__ int s_over, s_distinct;
   __shared__ int s_hist[PART ? 256 : 1], s_cur[PART ? 256 : 1];
   Tally ty;
   int32_t* stageA = PART ? a.stage + (int64_t)blockIdx.x * 2 * a.stage_stride : nullptr;
   int32_t* stageB = PART ? stageA + a.stage_stride : nullptr;
+  __shared__ int s_k0, s_nsel, s_sel[32];
   const int n_redo = a.mode ? (int)*a.redo_in_n : 0;
-  for (int i0 = blockIdx.x;; i0 += gridDim.x) {
-    int i;
-    if (PART) {  // dynamic fetch: row costs vary by orders of magnitude
-      if (threadIdx.x == 0) s_i = (int)atomicAdd(a.work, 1ull);
-      __syncthreads();
-      const int k = s_i;
-      __syncthreads();
-      if (a.mode ? k >= n_redo : k >= a.n_items) break;
-      i = a.mode ? a.redo_in[k] : k;
-    } else {
-      if (a.mode ? i0 >= n_redo : i0 >= a.n_items) break;
-      i = a.mode ? a.redo_in[i0] : i0;
+  const int lim = a.mode ? n_redo : a.n_items;
+  for (;;) {
+    // dynamic fetch of 32 rows (row costs vary by orders of magnitude); warp 0
+    // selects the rows of this class (and, in sparse iterations, the active
+    // ones) lane-parallel
+    // (tickets below big_prefix -- the longest rows, and every re-queued row --
+    // fetch one row each so long rows spread over blocks; later tickets 32)
+    if (threadIdx.x == 0) s_k0 = (int)atomicAdd(a.work, 1ull);
+    __syncthreads();
+    const int tk = s_k0;
+    const int big = a.mode ? lim : a.big_prefix;
+    const int k0 = tk < big ? tk : big + (tk - big) * 32;
+    const int kn = tk < big ? 1 : 32;
+    if (k0 >= lim) break;
+    if (threadIdx.x < 32) {
+      const int k = k0 + (int)threadIdx.x;
+      bool ok = (int)threadIdx.x < kn && k < lim;
+      int ik = -1;
+      if (ok) {
+        ik = a.mode ? a.redo_in[k] : k;
+        if (!a.mode) {
+          const BinItem itk = a.items[ik];
+          const unsigned raw = a.pred[ik];
+          const unsigned pk = a.pred_cap ? min(raw, a.pred_cap) : raw;
+          ok = row_class(pk, itk.d) == CLS;
+          if (ok && !a.dense && !a.flag[a.vb + itk.v]) {
+            ok = false;
+            a.pred_next[ik] = raw;  // inactive: carry the prediction forward
+          }
+        }
+      }
+      const unsigned m = __ballot_sync(kFull, ok);
+      if (ok) s_sel[__popc(m & ((1u << threadIdx.x) - 1u))] = ik;
+      if (threadIdx.x == 0) s_nsel = __popc(m);
     }
+    __syncthreads();
+    const int nsel = s_nsel;
+    for (int q = 0; q < nsel; ++q) {
+    const int i = s_sel[q];
     const BinItem it = a.items[i];
     const unsigned pred = a.pred_cap ? min(a.pred[i], a.pred_cap) : a.pred[i];
-    if (!a.mode) {
-      if (row_class(pred, it.d) != CLS) continue;              // block-uniform
-      if (!a.dense && !a.flag[a.vb + it.v]) continue;
-    }
     const int d = it.d;
     Best<VAR> b;
     if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; }
@@ -500,6 +562,7 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
     }
     if (!PART && over) {
       if (threadIdx.x == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = i;
+      __syncthreads();
       continue;
     }
     if (PART) {
@@ -583,6 +646,7 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
       update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty);
     }
     __syncthreads();
+    }  // selected rows
   }
   tally_flush(ty, a.cnt);
 }
