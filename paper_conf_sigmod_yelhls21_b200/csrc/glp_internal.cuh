@@ -31,14 +31,14 @@ constexpr int kLowBlock = 256;
 // distinct-label count `pred` (the exact count of its previous iteration;
 // deg at t = 1, when all labels are distinct) -- labels collapse as
 // communities form [P:130], so most rows migrate to the warp path:
-//   W  pred <= 256,  deg <= 16384 : one warp per row, 512-slot table per warp
-//   M  pred <= 2048, deg <= 65536 : one 128-thread block per row, 4096 slots
+//   W  pred <= 256,  deg <= 4096  : one warp per row, 512-slot table per warp
+//   M  pred <= 2048, deg <= 16384 : one 128-thread block per row, 4096 slots
 //   L  otherwise                  : one 1024-thread block per row, 16384
 //                                   slots, hash-partitioned passes
 // A row whose labels overflow its table is re-queued to the next class in the
 // same iteration (exact recount), so `pred` only steers performance.
 constexpr unsigned kWPred = 256, kMPred = 2048;
-constexpr int kWMaxDeg = 16384, kMMaxDeg = 65536;
+constexpr int kWMaxDeg = 4096, kMMaxDeg = 16384;
 constexpr int kWBlock = 256;
 constexpr int kWSlots = 512;
 constexpr int kMBlock = 128;

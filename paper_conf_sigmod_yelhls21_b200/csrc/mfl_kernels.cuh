@@ -173,6 +173,85 @@ __device__ __forceinline__ unsigned warp_insert(const MflArgs& a, const Table& t
   return COUNT_NEW ? (unsigned)__popc(__ballot_sync(kFull, fresh)) : 0u;
 }
 
+// Batched form of warp_insert for N labels per lane: the hot-label ballots of
+// all N slots first, then the N home-slot probes as independent shared loads,
+// then the N atomics, so their latencies overlap (a lane's inserts no longer
+// wait on each other); only labels whose home slot holds another label fall
+// back to the probing loop.  Returns this lane's count of newly claimed slots.
+template <bool POW2>
+__device__ __forceinline__ unsigned ht_probe_from(const Table& t, unsigned lab, unsigned c, unsigned h,
+                                                  unsigned max_probe, bool* fresh) {
+  for (unsigned p = 1; p < max_probe; ++p) {
+    h = (h + 1) & (t.tsz - 1);
+    unsigned long long e = *((volatile unsigned long long*)(t.slots + h));
+    if (e == kEmpty) {
+      const unsigned long long prev = atomicCAS(t.slots + h, kEmpty, ((unsigned long long)lab << 32) | c);
+      if (prev == kEmpty) {
+        *fresh = true;
+        return c;
+      }
+      e = prev;
+    }
+    if ((unsigned)(e >> 32) == lab) return atomicAdd((unsigned*)(t.slots + h), c) + c;
+  }
+  return 0u;
+}
+
+template <int VAR, int N>
+__device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
+                                                  const int (&lab)[N], Best<VAR>& b, volatile int* overflow) {
+  const int lane = threadIdx.x & 31;
+  unsigned c[N];
+  const int cand0 = b.have() ? (int)b.label() : -2;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    const bool vote = lab[j] >= 0;
+    const int hot = __shfl_sync(kFull, cand0 == -2 ? lab[j] : cand0, 0);
+    const unsigned m = __ballot_sync(kFull, vote && lab[j] == hot);
+    c[j] = vote ? (lab[j] != hot ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u)) : 0u;
+  }
+  unsigned h[N];
+  unsigned long long e[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    h[j] = slot_hash((unsigned)lab[j], t.tsz);
+    e[j] = c[j] ? *((volatile unsigned long long*)(t.slots + h[j])) : 0ull;
+  }
+  unsigned cnt[N];
+  unsigned nfresh = 0;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    cnt[j] = 0u;
+    if (c[j]) {
+      const unsigned l = (unsigned)lab[j];
+      if ((unsigned)(e[j] >> 32) == l) {
+        cnt[j] = atomicAdd((unsigned*)(t.slots + h[j]), c[j]) + c[j];
+      } else if (e[j] == kEmpty) {
+        const unsigned long long prev = atomicCAS(t.slots + h[j], kEmpty, ((unsigned long long)l << 32) | c[j]);
+        if (prev == kEmpty) {
+          cnt[j] = c[j];
+          ++nfresh;
+        } else if ((unsigned)(prev >> 32) == l) {
+          cnt[j] = atomicAdd((unsigned*)(t.slots + h[j]), c[j]) + c[j];
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    if (c[j] && cnt[j] == 0u) {
+      bool fr = false;
+      cnt[j] = ht_probe_from<true>(t, (unsigned)lab[j], c[j], h[j], max_probe, &fr);
+      nfresh += fr ? 1u : 0u;
+      if (cnt[j] == 0u) *overflow = 1;
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < N; ++j)
+    if (cnt[j]) b.observe(cnt[j], (unsigned)lab[j], a);
+  return nfresh;
+}
+
 // Per-thread iteration statistics, block-reduced once at kernel exit.
 struct Tally {
   unsigned long long changed = 0, d2 = 0, chdeg = 0, arcs = 0, verts = 0;
@@ -360,10 +439,12 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
       int l[8];
       l[0] = gather(a, u0.x); l[1] = gather(a, u0.y); l[2] = gather(a, u0.z); l[3] = gather(a, u0.w);
       l[4] = gather(a, u1.x); l[5] = gather(a, u1.y); l[6] = gather(a, u1.z); l[7] = gather(a, u1.w);
-      const int nj = (it.d - base) > 128 ? 8 : 4;  // warp-uniform
-#pragma unroll
-      for (int j = 0; j < 8; ++j)
-        if (j < nj) fresh += warp_insert<VAR, true>(a, tab, tsz, l[j], l[j] >= 0, b, &s_over[wid]);
+      if (it.d - base > 128) {  // warp-uniform
+        fresh += warp_insert_n<VAR, 8>(a, tab, tsz, l, b, &s_over[wid]);
+      } else {
+        const int l4[4] = {l[0], l[1], l[2], l[3]};
+        fresh += warp_insert_n<VAR, 4>(a, tab, tsz, l4, b, &s_over[wid]);
+      }
       __syncwarp();
       over = s_over[wid] != 0;
     }
@@ -373,6 +454,7 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
       continue;
     }
     b.warp_reduce();
+    fresh = __reduce_add_sync(kFull, fresh);
     if (lane == 0) {
       a.pred_next[i] = max(fresh, 1u);
       update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
@@ -426,14 +508,18 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
           __stcg((int4*)(stage_out + idx), make_int4(lab[4 * j], lab[4 * j + 1], lab[4 * j + 2], lab[4 * j + 3]));
       }
     }
+    if (nparts > 1u) {
 #pragma unroll
-    for (int j = 0; j < 4 * UNROLL; ++j) {
-      const bool vote = lab[j] >= 0 && (nparts == 1u || label_part((unsigned)lab[j], nparts) == part);
-      fresh += warp_insert<VAR, COUNT_NEW>(a, tab, max_probe, lab[j], vote, b, overflow);
+      for (int j = 0; j < 4 * UNROLL; ++j)
+        if (lab[j] >= 0 && label_part((unsigned)lab[j], nparts) != part) lab[j] = -1;
     }
+    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow);
     if (__any_sync(kFull, *overflow != 0)) break;  // warp-uniform exit
   }
-  if (COUNT_NEW && (threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
+  if (COUNT_NEW) {
+    fresh = __reduce_add_sync(kFull, fresh);
+    if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
+  }
 }
 
 template <int VAR, int BLOCK>
@@ -460,12 +546,17 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
                                              unsigned max_probe, volatile int* overflow, int* distinct,
                                              Best<VAR>& b) {
   unsigned fresh = 0;
-  for (int j0 = 0; j0 < cnt; j0 += BLOCK) {
-    const int j = j0 + (int)threadIdx.x;
-    const int lab = j < cnt ? __ldcg(stage + j) : -1;
-    fresh += warp_insert<VAR, true>(a, tab, max_probe, lab, lab >= 0, b, overflow);
+  for (int j0 = 0; j0 < cnt; j0 += 4 * BLOCK) {
+    int lab[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int j = j0 + k * BLOCK + (int)threadIdx.x;
+      lab[k] = j < cnt ? __ldcg(stage + j) : -1;
+    }
+    fresh += warp_insert_n<VAR, 4>(a, tab, max_probe, lab, b, overflow);
     if (__any_sync(kFull, *overflow != 0)) break;
   }
+  fresh = __reduce_add_sync(kFull, fresh);
   if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
 }
 
