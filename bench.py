@@ -168,19 +168,11 @@ def bench_gpu(args):
     stream = torch.cuda.current_stream()
 
     # ---- partition (1-D vertex ranges; equal vertex counts) ----
-    kw = {}
-    off, col = csr.row_offsets, csr.col_idx
-    vb, ve = 0, n
     if world > 1:
-        bounds = glp.glp_partition(n, world)
-        vb, ve = bounds[rank], bounds[rank + 1]
-        o0, o1 = int(off[vb]), int(off[ve])
-        off = (off[vb:ve + 1] - o0).contiguous()
-        col = col[o0:o1].contiguous()
-        uid = [glp.glp_nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0)
-        kw = dict(rank=rank, nranks=world, nccl_unique_id=uid[0], v_begin=vb, v_end=ve)
-    g = glp.Graph(n=n, row_offsets=off, col_idx=col, device=local, stream=stream, **kw)
+        from paper_conf_sigmod_yelhls21_b200 import dist as gdist
+        g = gdist.distributed_graph(csr, stream=stream)
+    else:
+        g = glp.Graph(csr, device=local, stream=stream)
     info = g.info()
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
 
@@ -340,7 +332,7 @@ def bench_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="glp", choices=["glp", "reference"])
     ap.add_argument("--workload", default="rmat24", choices=sorted(WORKLOADS))

@@ -1,0 +1,51 @@
+"""Multi-GPU plumbing for the 1-D vertex-range partition.
+
+One process per GPU.  Rank r owns rows [b_r, b_{r+1}) of the CSR (bounds from
+``glp_partition``: equal vertex counts, or equal arc counts), keeps the owned
+rows with GLOBAL column ids, and replicates the label array; the library
+exchanges labels each iteration with an in-place NCCL all-gather.  This module
+only slices the CSR and distributes the NCCL unique id through
+``torch.distributed``; all per-iteration work happens inside libglp.so.
+"""
+from __future__ import annotations
+
+import torch
+
+from . import Graph, glp_nccl_unique_id, glp_partition
+
+
+def shard_bounds(n: int, world: int, row_offsets=None, edge_balanced: bool = False):
+    """Row bounds [b_0 = 0, ..., b_world = n] of every rank."""
+    return glp_partition(n, world, row_offsets if edge_balanced else None, edge_balanced=edge_balanced)
+
+
+def local_rows(row_offsets: torch.Tensor, col_idx: torch.Tensor, v_begin: int, v_end: int):
+    """The owned rows of a global CSR: rebased offsets + their arcs (global ids)."""
+    o0 = int(row_offsets[v_begin])
+    o1 = int(row_offsets[v_end])
+    off = (row_offsets[v_begin:v_end + 1] - o0).contiguous()
+    col = col_idx[o0:o1].contiguous()
+    return off, col
+
+
+def broadcast_unique_id(group=None) -> bytes:
+    """Rank 0 creates the 128-byte NCCL id; every rank receives it."""
+    import torch.distributed as dist
+    obj = [glp_nccl_unique_id() if dist.get_rank(group) == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
+def distributed_graph(csr, group=None, edge_balanced: bool = False, stream=None) -> Graph:
+    """Create this rank's share of `csr` (full graph on every rank) as a
+    multi-GPU glp graph over the NCCL communicator of the process group."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    bounds = shard_bounds(csr.n, world, csr.row_offsets.cpu(), edge_balanced)
+    vb, ve = bounds[rank], bounds[rank + 1]
+    off, col = local_rows(csr.row_offsets, csr.col_idx, vb, ve)
+    uid = broadcast_unique_id(group) if world > 1 else None
+    dev = torch.cuda.current_device()
+    return Graph(n=csr.n, row_offsets=off, col_idx=col, rank=rank, nranks=world, nccl_unique_id=uid,
+                 v_begin=vb, v_end=ve, device=dev, stream=stream)
