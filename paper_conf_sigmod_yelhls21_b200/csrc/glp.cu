@@ -206,6 +206,39 @@ void build_layout(glp_graph* g, const int64_t* off_h, const int64_t* off_d, cons
     g->n_gt2048 += it.d > 2048;
     g->n_ge8k += it.d >= 8192;
   }
+  // giant rows: the prefix with deg > kGiantMin, split into segments
+  g->n_giant = 0;
+  for (const BinItem& it : row_i) g->n_giant += it.d > kGiantMin;
+  if (g->n_giant > 0) {
+    if (maxd >= ((int64_t)1 << kGCountBits))
+      fail(GLP_ERR_UNSUPPORTED, "a row has >= 2^25 arcs (giant-row table count field)");
+    std::vector<GiantSeg> segs;
+    std::vector<int32_t> first;
+    std::vector<int64_t> toff;
+    int64_t slots = 0;
+    for (int32_t r = 0; r < g->n_giant; ++r) {
+      first.push_back((int32_t)segs.size());
+      toff.push_back(slots);
+      for (int32_t b = 0; b < row_i[r].d; b += kGiantSeg) segs.push_back(GiantSeg{r, b});
+      int64_t tsz = 1;
+      while (tsz < 2 * (int64_t)row_i[r].d) tsz <<= 1;
+      slots += tsz;
+    }
+    first.push_back((int32_t)segs.size());
+    toff.push_back(slots);
+    g->n_gsegs = (int32_t)segs.size();
+    g->gsegs = upload(g, segs);
+    g->gseg_first = upload(g, first);
+    g->gtab_off = upload(g, toff);
+    g->gtab_slots = slots;
+    g->gtab = dalloc<unsigned long long>(g, slots);
+    CK(cudaMemsetAsync(g->gtab, 0, slots * sizeof(unsigned long long), g->stream));
+    g->gepoch = 0;
+    g->gcand_key = dalloc<unsigned long long>(g, segs.size());
+    g->gcand_lab = dalloc<unsigned>(g, segs.size());
+    g->gdistinct = dalloc<unsigned>(g, g->n_giant);
+    CK(cudaMemsetAsync(g->gdistinct, 0, g->n_giant * sizeof(unsigned), g->stream));
+  }
   g->low_list = upload(g, low);
   g->chunks = upload(g, chunks);
   g->cflag = dalloc<uint8_t>(g, std::max<int32_t>(g->n_chunks, 1));
@@ -352,8 +385,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->flag[1] = dalloc<uint8_t>(g, npad);
     CK(cudaMemsetAsync(g->flag[0], 0, std::max<int64_t>(npad, 1), g->stream));
     CK(cudaMemsetAsync(g->flag[1], 0, std::max<int64_t>(npad, 1), g->stream));
-    g->d_cnt = dalloc<Counters>(g, 4);
-    CK(cudaMallocHost(&g->h_cnt, 4 * sizeof(Counters)));
+    g->d_cnt = dalloc<Counters>(g, 5);
+    CK(cudaMallocHost(&g->h_cnt, 5 * sizeof(Counters)));
     CK(cudaEventCreate(&g->ev_a));
     CK(cudaEventCreate(&g->ev_b));
 
@@ -369,6 +402,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->grid_w = grid_for(sms, (const void*)mfl_warp<V_LLP>, kWBlock, 0);
     g->grid_m = grid_for(sms, (const void*)GLP_M_KERNEL(V_LLP), kMBlock, ms_);
     g->grid_l = grid_for(sms, (const void*)GLP_L_KERNEL(V_LLP), kLBlock, ls_);
+    g->grid_g = grid_for(sms, (const void*)mfl_giant_count<V_LLP>, kGBlock, 0);
     g->grid_aux = sms * 8;
     if (g->n_rows > 0) {
       // L staging: two row-sized buffers per resident L block
@@ -401,8 +435,9 @@ cudaEvent_t pool_event(glp_graph* g, size_t& used) {
   return g->ev_pool[used++];
 }
 
-const char* kKernelNames[] = {"mfl_low", "mfl_warp", "mfl_block_m", "mfl_block_l", "push", "llp_hist", "exchange"};
-constexpr int kNumKernelNames = 7;
+const char* kKernelNames[] = {"mfl_low", "mfl_warp", "mfl_block_m", "mfl_block_l", "push", "llp_hist", "exchange",
+                              "mfl_giant"};
+constexpr int kNumKernelNames = 8;
 
 template <class F>
 void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t& used, F f) {
@@ -429,6 +464,17 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   MflArgs r = a;
   r.items = g->rows; r.big_prefix = g->n_ge8k; r.pred = g->pred[g->pb]; r.pred_next = g->pred[1 - g->pb];
   r.stage = g->stage; r.stage_stride = g->stage_stride;
+  if (g->n_giant) {  // giant rows: all blocks count segments into per-row global tables
+    MflArgs b = r;
+    b.cnt = c + 4; b.work = &sc->work_g;
+    b.gsegs = g->gsegs; b.n_gsegs = g->n_gsegs; b.gtab = g->gtab; b.gtab_off = g->gtab_off;
+    b.gcand_key = g->gcand_key; b.gcand_lab = g->gcand_lab; b.gdistinct = g->gdistinct; b.epoch = g->gepoch;
+    timed(g, prof, 7, pend, used, [&] {
+      mfl_giant_count<VAR><<<std::min(g->grid_g, g->n_gsegs), kGBlock, 0, g->stream>>>(b);
+      mfl_giant_finish<VAR><<<g->n_giant, 256, 0, g->stream>>>(b, g->gseg_first);
+    });
+    n += 2;
+  }
   if (g->n_gt2048) {  // L, static: rows of class L (a prefix of deg > 2048)
     MflArgs b = r;
     b.n_items = g->n_gt2048; b.cnt = c + 3; b.work = &sc->work_l;
@@ -570,8 +616,8 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       KStat& ks = g->kstats[pe.kid];
       ks.launches += 1;
       ks.ms += kms;
-      if (with_counters && pe.kid < 4 && pe.t == cur_t) {
-        const Counters& c = g->h_cnt[pe.kid];
+      if (with_counters && (pe.kid < 4 || pe.kid == 7) && pe.t == cur_t) {
+        const Counters& c = g->h_cnt[pe.kid == 7 ? 4 : pe.kid];
         ks.arcs += (double)c.arcs;
         // 4 B/arc (col_idx) + 8 B/active vertex (row offsets) + 4 B/changed label
         ks.bytes += 4.0 * (double)c.arcs + 8.0 * (double)c.verts + 4.0 * (double)c.changed;
@@ -587,9 +633,16 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   for (int32_t t = 1; t <= max_iters; ++t) {
     cudaEvent_t e0 = pool_event(g, used), e1 = pool_event(g, used);
     CK(cudaEventRecord(e0, s));
-    CK(cudaMemsetAsync(g->d_cnt, 0, 4 * sizeof(Counters), s));
+    CK(cudaMemsetAsync(g->d_cnt, 0, 5 * sizeof(Counters), s));
     CK(cudaMemsetAsync(g->d_sched, 0, sizeof(Sched), s));
     g->cur_t = t;
+    if (g->n_giant) {
+      // giant-table epoch: slots of other epochs are free; clear on wrap
+      if (++g->gepoch >= (1ull << kGEpochBits)) {
+        CK(cudaMemsetAsync(g->gtab, 0, g->gtab_slots * sizeof(unsigned long long), s));
+        g->gepoch = 1;
+      }
+    }
     MflArgs a;
     memset(&a, 0, sizeof(a));
     a.col = g->col2; a.R = g->L[rb]; a.W = g->L[1 - rb]; a.so = g->so;
@@ -603,14 +656,14 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     }
     if (g->nranks > 1) {
       timed(g, prof, 6, pend, used, [&] { nccl_exchange(g, g->L[1 - rb]); });
-      nccl_sum_counters(g, g->d_cnt, 4 * sizeof(Counters) / sizeof(unsigned long long));
+      nccl_sum_counters(g, g->d_cnt, 5 * sizeof(Counters) / sizeof(unsigned long long));
     }
-    CK(cudaMemcpyAsync(g->h_cnt, g->d_cnt, 4 * sizeof(Counters), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(g->h_cnt, g->d_cnt, 5 * sizeof(Counters), cudaMemcpyDeviceToHost, s));
     CK(cudaEventRecord(e1, s));
     CK(cudaStreamSynchronize(s));
     Counters tot;
     memset(&tot, 0, sizeof(tot));
-    for (int b = 0; b < 4; ++b) {
+    for (int b = 0; b < 5; ++b) {
       tot.changed += g->h_cnt[b].changed; tot.d2 += g->h_cnt[b].d2; tot.chdeg += g->h_cnt[b].chdeg;
       tot.arcs += g->h_cnt[b].arcs; tot.verts += g->h_cnt[b].verts;
     }

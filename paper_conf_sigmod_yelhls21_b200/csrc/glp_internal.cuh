@@ -48,17 +48,35 @@ constexpr int kLBlock = 1024;
 constexpr int kLSlots = 16384;
 constexpr int kLUnroll = 2;
 constexpr int kLProbe = 32;  // probe limit before declaring a partition overflowed
-enum RowClass { CLS_W = 0, CLS_M = 1, CLS_L = 2 };
+// Giant rows (deg > kGiantMin) are split into segments of kGiantSeg arcs that
+// many blocks count concurrently into one global-memory table per row
+// (epoch-tagged slots, never cleared between iterations); a second kernel
+// reduces the per-segment candidates of each row.
+constexpr int kGiantMin = 65536;
+constexpr int kGiantSeg = 32768;
+constexpr int kGBlock = 512;
+constexpr int kGUnroll = 2;
+constexpr int kGCountBits = 25;  // count field of a giant-table slot (deg < 2^25)
+constexpr int kGEpochBits = 64 - 31 - kGCountBits;
+enum RowClass { CLS_W = 0, CLS_M = 1, CLS_L = 2, CLS_G = 3 };
 __host__ __device__ __forceinline__ int row_class(unsigned pred, int d) {
+  if (d > kGiantMin) return CLS_G;
   if (pred <= kWPred && d <= kWMaxDeg) return CLS_W;
   if (pred <= kMPred && d <= kMMaxDeg) return CLS_M;
   return CLS_L;
 }
 
+// One segment of a giant row.
+struct GiantSeg {
+  int32_t row;    // index into the giant prefix of `rows`
+  int32_t begin;  // arc offset within the row
+};
+
 // Per-iteration scheduling state (reset with the counters).
 struct Sched {
   unsigned n_redo_m, n_redo_l;      // rows re-queued to M / L this iteration
   unsigned long long work_m, work_mr, work_l, work_lr;  // dynamic fetch counters (static / redo)
+  unsigned long long work_g;
 };
 
 // A low-degree chunk: up to 32 consecutive arcs of consecutive low-list
@@ -119,6 +137,14 @@ struct MflArgs {
   unsigned long long* work;             // dynamic fetch counter (L)
   int32_t* __restrict__ stage;          // L: per-block staged row labels (2 x stride)
   int64_t stage_stride;
+  const GiantSeg* __restrict__ gsegs;   // giant rows: segments, tables, candidates
+  int32_t n_gsegs;
+  unsigned long long* __restrict__ gtab;
+  const int64_t* __restrict__ gtab_off; // per giant row: slot offset, table size = next - this
+  unsigned long long* __restrict__ gcand_key;  // per segment
+  unsigned* __restrict__ gcand_lab;
+  unsigned* __restrict__ gdistinct;     // per giant row
+  unsigned long long epoch;             // giant-table epoch of this iteration (1..2^kGEpochBits-1)
   Counters* cnt;
   int64_t vb;                           // global id of local row 0
   double gamma;
@@ -168,6 +194,15 @@ struct glp_graph {
   glp::BinItem* rows = nullptr; int32_t n_rows = 0;  // deg > 32, degree-descending
   int32_t n_gt256 = 0, n_gt2048 = 0;                 // prefixes with deg > 256 / > 2048
   int32_t n_ge8k = 0;                                // prefix with deg >= 8192
+  int32_t n_giant = 0;                               // prefix with deg > kGiantMin
+  glp::GiantSeg* gsegs = nullptr; int32_t n_gsegs = 0;
+  unsigned long long* gtab = nullptr; int64_t gtab_slots = 0;
+  int64_t* gtab_off = nullptr;
+  unsigned long long* gcand_key = nullptr;
+  unsigned* gcand_lab = nullptr;
+  unsigned* gdistinct = nullptr;
+  int32_t* gseg_first = nullptr;                     // [n_giant+1]
+  unsigned long long gepoch = 0;                     // last giant-table epoch used
   unsigned* pred[2] = {nullptr, nullptr};            // [n_rows], double-buffered per iteration
   int pb = 0;                                        // pred[pb] is read this iteration
   int32_t* redo_m = nullptr;                         // [n_rows]
@@ -193,7 +228,7 @@ struct glp_graph {
   int64_t seeds_cap = 0;
 
   // launch geometry
-  int grid_low = 0, grid_w = 0, grid_m = 0, grid_l = 0, grid_aux = 0;
+  int grid_low = 0, grid_w = 0, grid_m = 0, grid_l = 0, grid_g = 0, grid_aux = 0;
 
   int cur = 0;  // index of L holding the result of the last run
   int cur_t = 0;  // iteration being launched (profiling)

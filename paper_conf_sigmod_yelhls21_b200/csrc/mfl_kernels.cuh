@@ -742,4 +742,114 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
   tally_flush(ty, a.cnt);
 }
 
+// ---------------------------------------------------------------------------
+// Giant rows (deg > kGiantMin): one global-memory table per row, shared by all
+// blocks that count the row's segments.  Slot = [epoch | label | count]; a slot
+// whose epoch is not this iteration's is free, so tables are never cleared
+// between iterations (only when the epoch counter wraps).
+__device__ __forceinline__ unsigned giant_add(unsigned long long* tab, unsigned long long tsz, unsigned lab,
+                                              unsigned c, unsigned long long epoch, bool* fresh) {
+  constexpr int kShift = 31 + kGCountBits;
+  const unsigned long long tag = (epoch << kShift) | ((unsigned long long)lab << kGCountBits);
+  const unsigned long long keymask = ~((1ull << kGCountBits) - 1ull);
+  const unsigned long long cmask = (1ull << kGCountBits) - 1ull;
+  unsigned long long h = (unsigned long long)((lab * 0x9E3779B97F4A7C15ull) >> 20) & (tsz - 1ull);
+  for (;;) {
+    unsigned long long e = *((volatile unsigned long long*)(tab + h));
+    for (;;) {
+      if ((e & keymask) == tag) return (unsigned)((atomicAdd(tab + h, (unsigned long long)c) & cmask) + c);
+      if ((e >> kShift) != epoch) {  // stale slot: claim it
+        const unsigned long long prev = atomicCAS(tab + h, e, tag | c);
+        if (prev == e) {
+          *fresh = true;
+          return c;
+        }
+        e = prev;  // re-examine the same slot
+        continue;
+      }
+      break;  // another label of this iteration
+    }
+    h = (h + 1ull) & (tsz - 1ull);
+  }
+}
+
+// Phase 1: blocks take segments (dynamic tickets) and count them into their
+// row's table; each segment leaves its best observation as a candidate.
+template <int VAR>
+__global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
+  __shared__ int s_k;
+  const int lane = threadIdx.x & 31;
+  for (;;) {
+    if (threadIdx.x == 0) s_k = (int)atomicAdd(a.work, 1ull);
+    __syncthreads();
+    const int k = s_k;
+    __syncthreads();
+    if (k >= a.n_gsegs) break;
+    const GiantSeg sg = a.gsegs[k];
+    const BinItem it = a.items[sg.row];
+    if (!a.dense && !a.flag[a.vb + it.v]) continue;  // block-uniform
+    unsigned long long* tab = a.gtab + a.gtab_off[sg.row];
+    const unsigned long long tsz = (unsigned long long)(a.gtab_off[sg.row + 1] - a.gtab_off[sg.row]);
+    const int end = min(sg.begin + kGiantSeg, it.d);
+    Best<VAR> b;
+    unsigned fresh = 0;
+    for (int base = sg.begin; base < end; base += kGBlock * 4 * kGUnroll) {
+      int lab[4 * kGUnroll];
+#pragma unroll
+      for (int j = 0; j < kGUnroll; ++j) {
+        const int idx = base + (j * kGBlock + (int)threadIdx.x) * 4;
+        const int4 u = idx < end ? ld_stream4(a.col + it.start + idx) : make_int4(-1, -1, -1, -1);
+        lab[4 * j + 0] = gather(a, u.x);
+        lab[4 * j + 1] = gather(a, u.y);
+        lab[4 * j + 2] = gather(a, u.z);
+        lab[4 * j + 3] = gather(a, u.w);
+      }
+      const int cand0 = b.have() ? (int)b.label() : -2;
+#pragma unroll
+      for (int j = 0; j < 4 * kGUnroll; ++j) {
+        const bool vote = lab[j] >= 0;
+        const int hot = __shfl_sync(kFull, cand0 == -2 ? lab[j] : cand0, 0);
+        const unsigned m = __ballot_sync(kFull, vote && lab[j] == hot);
+        const unsigned c = vote ? (lab[j] != hot ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u)) : 0u;
+        if (c) {
+          bool fr = false;
+          const unsigned cnt = giant_add(tab, tsz, (unsigned)lab[j], c, a.epoch, &fr);
+          fresh += fr ? 1u : 0u;
+          b.observe(cnt, (unsigned)lab[j], a);
+        }
+      }
+    }
+    fresh = __reduce_add_sync(kFull, fresh);
+    if (lane == 0 && fresh) atomicAdd(a.gdistinct + sg.row, fresh);
+    b = block_best<VAR, kGBlock>(b);
+    if (threadIdx.x == 0) {
+      a.gcand_key[k] = b.key;
+      a.gcand_lab[k] = b.lab;
+    }
+  }
+}
+
+// Phase 2: one block per giant row reduces its segments' candidates (the best
+// over all observations is exact, see the header) and updates the vertex.
+template <int VAR>
+__global__ void __launch_bounds__(256) mfl_giant_finish(MflArgs a, const int32_t* __restrict__ seg_first) {
+  Tally ty;
+  const int i = blockIdx.x;
+  const BinItem it = a.items[i];
+  const bool active = a.dense || a.flag[a.vb + it.v];
+  if (active) {
+    Best<VAR> b;
+    for (int k = seg_first[i] + (int)threadIdx.x; k < seg_first[i + 1]; k += 256) b.merge(a.gcand_key[k], a.gcand_lab[k]);
+    b = block_best<VAR, 256>(b);
+    if (threadIdx.x == 0) {
+      a.pred_next[i] = max(a.gdistinct[i], 1u);
+      a.gdistinct[i] = 0u;
+      update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
+    }
+  } else if (threadIdx.x == 0) {
+    a.pred_next[i] = a.pred[i];
+  }
+  tally_flush(ty, a.cnt);
+}
+
 }  // namespace glp

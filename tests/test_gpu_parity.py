@@ -148,6 +148,20 @@ def test_requeue_paths_exact(cap):
         assert_same_run(csr, 2, 5, gamma=0.25, debug_pred_cap=cap)
 
 
+def test_giant_rows_epoch_wrap():
+    """Giant rows (deg > 65536) use epoch-tagged global tables that are only
+    cleared when the 8-bit epoch wraps: run past several wraps."""
+    csr = graphs.star(70000)
+    ref = oracle.run(csr, 0, 600, stop_on_2cycle=False)
+    lab, info, st = gpu(csr, 0, 600, stop_on_2cycle=False)
+    assert info.iterations == 600 and (lab == ref.labels).all()
+    csr = _degree_mix([200000, 90000, 70000, 66000, 3000], seed=5, extra_pairs=300000)
+    for _ in range(2):
+        assert_same_run(csr, 0, 20)
+        assert_same_run(csr, 1, 20, seeds=[0, 1, 7, 400000])
+        assert_same_run(csr, 2, 6, gamma=1.0)
+
+
 def test_hub_with_few_labels_and_ties():
     # a hub whose neighbours carry a handful of labels: hot keys (warp
     # aggregation) and an exact tie resolved to the smaller label
