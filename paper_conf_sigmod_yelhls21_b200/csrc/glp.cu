@@ -22,6 +22,7 @@
 
 #include "aux_kernels.cuh"
 #include "glp_internal.cuh"
+#include "layout.cuh"
 #include "mfl_kernels.cuh"
 #include "nccl_dyn.cuh"
 
@@ -129,88 +130,126 @@ void free_graph(glp_graph* g) {
 #define GLP_L_KERNEL(VAR) mfl_block<VAR, kLBlock, kLSlots, true, kLUnroll, CLS_L>
 
 // Degree bins, low-degree warp chunks and the bin-major arc copy col2
-// (DESIGN.md §Layout).  Host decides the order; a kernel moves the arcs.
-// off_h: host row offsets; off_d/col_d: the caller's CSR on the device.
-void build_layout(glp_graph* g, const int64_t* off_h, const int64_t* off_d, const int32_t* col_d) {
-  std::vector<int32_t> low, rows;
-  for (int b = 0; b < NBINS; ++b) g->bin_verts[b] = g->bin_arcs[b] = 0;
-  int64_t maxd = 0;
-  for (int64_t v = 0; v < g->nl; ++v) {
-    const int64_t d = off_h[v + 1] - off_h[v];
-    if (d >= ((int64_t)1 << 30)) fail(GLP_ERR_INVALID_GRAPH, "row degree >= 2^30 is not supported");
-    maxd = std::max(maxd, d);
-    int b;  // reporting bins: 0 | 1-32 | 33-256 | 257-2048 | > 2048
-    if (d == 0) b = BIN_ISO;
-    else if (d <= kLowMax) { b = BIN_LOW; low.push_back((int32_t)v); }
-    else if (d <= 256) b = BIN_MID;
-    else if (d <= 2048) b = BIN_HIGH;
-    else b = BIN_HUGE;
-    if (d > kLowMax) rows.push_back((int32_t)v);
-    g->bin_verts[b] += 1;
-    g->bin_arcs[b] += d;
-  }
-  g->max_deg = maxd;
-  auto deg = [&](int32_t v) { return off_h[v + 1] - off_h[v]; };
-  // degree-descending: long rows start first, and each row class is a prefix
-  std::sort(rows.begin(), rows.end(), [&](int32_t a, int32_t b) { return deg(a) != deg(b) ? deg(a) > deg(b) : a < b; });
-  std::vector<int64_t> ioff(g->nl, 0);
-  std::vector<int32_t> ideg(g->nl, 0);
-  int64_t pos = 0;
-  // low bin: greedy chunks of consecutive low vertices with sum(deg) <= 32
-  std::vector<LowChunk> chunks;
-  {
-    size_t k = 0;
-    while (k < low.size()) {
-      LowChunk c;
-      c.vbase = (int32_t)k;
-      c.segmask = 0;
-      int total = 0;
-      const int64_t cstart = pos;
-      while (k < low.size() && total + deg(low[k]) <= 32) {
-        const int32_t v = low[k];
-        c.segmask |= 1u << total;
-        ioff[v] = pos;
-        ideg[v] = (int32_t)deg(v);
-        pos += deg(v);
-        total += (int)deg(v);
-        ++k;
-      }
-      c.st = (unsigned long long)cstart | ((unsigned long long)total << 56);
-      chunks.push_back(c);
+// (DESIGN.md §Layout), built on the device (layout.cuh).  off_d/col_d: the
+// caller's CSR on the device (borrowed or staged).
+void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
+  cudaStream_t s = g->stream;
+  auto pol = thrust::cuda::par.on(s);
+  const int64_t nl = g->nl;
+  std::vector<void*> tmp;
+  auto talloc = [&](size_t bytes) {
+    void* p = nullptr;
+    if (cudaMalloc(&p, std::max<size_t>(bytes, 16)) != cudaSuccess) {
+      cudaGetLastError();
+      for (void* q : tmp) cudaFree(q);
+      fail(GLP_ERR_OUT_OF_MEMORY, "layout scratch allocation failed");
     }
-  }
-  auto place = [&](const std::vector<int32_t>& vs, std::vector<BinItem>& items) {
-    pos = (pos + 3) & ~(int64_t)3;
-    for (int32_t v : vs) {
-      BinItem it;
-      it.start = pos;
-      it.v = v;
-      it.d = (int32_t)deg(v);
-      ioff[v] = pos;
-      ideg[v] = it.d;
-      items.push_back(it);
-      pos += (deg(v) + 3) & ~(int64_t)3;
-    }
+    tmp.push_back(p);
+    return p;
   };
-  std::vector<BinItem> row_i;
-  place(rows, row_i);
-  g->nnz2 = pos;
-  if (pos >= ((int64_t)1 << 56)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
-  g->n_low = (int32_t)low.size();
-  g->n_chunks = (int32_t)chunks.size();
-  g->n_rows = (int32_t)row_i.size();
-  g->n_gt256 = 0;
-  g->n_gt2048 = 0;
+  struct Free {
+    std::vector<void*>& v;
+    cudaStream_t s;
+    ~Free() {
+      cudaStreamSynchronize(s);
+      for (void* p : v) cudaFree(p);
+    }
+  } fr{tmp, s};
+  int32_t* deg = (int32_t*)talloc(nl * sizeof(int32_t));
+  LayoutStats* dst = (LayoutStats*)talloc(sizeof(LayoutStats));
+  CK(cudaMemsetAsync(dst, 0, sizeof(LayoutStats), s));
+  const int gb = g->sms * 8;
+  if (nl) k_degree_stats<<<gb, 256, 0, s>>>(off_d, nl, deg, dst);
+  CK(cudaGetLastError());
+  LayoutStats st;
+  CK(cudaMemcpyAsync(&st, dst, sizeof(st), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  for (int b = 0; b < NBINS; ++b) {
+    g->bin_verts[b] = (int64_t)st.verts[b];
+    g->bin_arcs[b] = (int64_t)st.arcs[b];
+  }
+  g->max_deg = (int64_t)st.max_deg;
+  if (g->max_deg >= ((int64_t)1 << 30)) fail(GLP_ERR_INVALID_GRAPH, "row degree >= 2^30 is not supported");
+  const int64_t n_low = g->bin_verts[BIN_LOW];
+  const int64_t n_rows = nl - g->bin_verts[BIN_ISO] - n_low;
+  g->ioff = dalloc<int64_t>(g, nl);
+  g->ideg = dalloc<int32_t>(g, nl);
+  CK(cudaMemsetAsync(g->ioff, 0, std::max<int64_t>(nl, 1) * sizeof(int64_t), s));
+  CK(cudaMemsetAsync(g->ideg, 0, std::max<int64_t>(nl, 1) * sizeof(int32_t), s));
+  unsigned long long* keys = (unsigned long long*)talloc(std::max(n_low, n_rows) * sizeof(unsigned long long));
+  // ---- low rows: sorted by (deg, id), packed floor(32/deg) per chunk
+  g->low_list = dalloc<int32_t>(g, n_low);
+  LowGroups grp;
+  memset(&grp, 0, sizeof(grp));
+  int64_t vb = 0, cb = 0, ab = 0;
+  for (int d = 1; d <= 33; ++d) {
+    grp.vbase[d] = vb;
+    grp.cbase[d] = cb;
+    grp.abase[d] = ab;
+    if (d <= 32) {
+      const int64_t cnt = (int64_t)st.low_hist[d];
+      vb += cnt;
+      cb += (cnt + (32 / d) - 1) / (32 / d);
+      ab += cnt * d;
+    }
+  }
+  g->n_low = (int32_t)n_low;
+  g->n_chunks = (int32_t)cb;
+  g->chunks = dalloc<LowChunk>(g, cb);
+  g->cflag = dalloc<uint8_t>(g, std::max<int64_t>(cb, 1));
+  const int64_t low_arcs = ab;
+  if (n_low) {
+    thrust::copy_if(pol, thrust::counting_iterator<int32_t>(0), thrust::counting_iterator<int32_t>((int32_t)nl),
+                    thrust::device_pointer_cast(g->low_list), IsLow{deg});
+    k_make_keys<<<gb, 256, 0, s>>>(g->low_list, n_low, deg, 0, keys);
+    thrust::sort(pol, thrust::device_pointer_cast(keys), thrust::device_pointer_cast(keys) + n_low);
+    k_keys_to_ids<<<gb, 256, 0, s>>>(keys, n_low, g->low_list);
+    k_low_chunks<<<gb, 256, 0, s>>>(grp, cb, n_low, g->chunks);
+    k_low_place<<<gb, 256, 0, s>>>(grp, g->low_list, n_low, deg, g->ioff, g->ideg);
+    CK(cudaGetLastError());
+  }
+  // ---- other rows: (deg desc, id), 16-B aligned, padded to a multiple of 4
+  int32_t* rows = (int32_t*)talloc(n_rows * sizeof(int32_t));
+  int64_t* pstart = (int64_t*)talloc((n_rows + 1) * sizeof(int64_t));
+  const int64_t rows_base = (low_arcs + 3) & ~(int64_t)3;
+  g->n_rows = (int32_t)n_rows;
+  g->rows = dalloc<BinItem>(g, n_rows);
+  std::vector<BinItem> row_i(n_rows);
+  int64_t padded_total = 0;
+  if (n_rows) {
+    thrust::copy_if(pol, thrust::counting_iterator<int32_t>(0), thrust::counting_iterator<int32_t>((int32_t)nl),
+                    thrust::device_pointer_cast(rows), IsRow{deg});
+    k_make_keys<<<gb, 256, 0, s>>>(rows, n_rows, deg, 1, keys);
+    thrust::sort(pol, thrust::device_pointer_cast(keys), thrust::device_pointer_cast(keys) + n_rows);
+    k_keys_to_ids<<<gb, 256, 0, s>>>(keys, n_rows, rows);
+    k_padded_deg<<<gb, 256, 0, s>>>(rows, n_rows, deg, pstart);
+    CK(cudaGetLastError());
+    thrust::exclusive_scan(pol, thrust::device_pointer_cast(pstart), thrust::device_pointer_cast(pstart) + n_rows + 1,
+                           thrust::device_pointer_cast(pstart));
+    k_row_place<<<gb, 256, 0, s>>>(rows, n_rows, deg, pstart, rows_base, g->rows, g->ioff, g->ideg);
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(row_i.data(), g->rows, n_rows * sizeof(BinItem), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&padded_total, pstart + n_rows, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+  }
+  g->nnz2 = rows_base + padded_total;
+  if (g->nnz2 >= ((int64_t)1 << 56)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
+  g->n_gt256 = g->n_gt2048 = g->n_ge8k = 0;
   for (const BinItem& it : row_i) {
     g->n_gt256 += it.d > 256;
     g->n_gt2048 += it.d > 2048;
     g->n_ge8k += it.d >= 8192;
   }
+  g->pred[0] = dalloc<unsigned>(g, std::max<int64_t>(n_rows, 1));
+  g->pred[1] = dalloc<unsigned>(g, std::max<int64_t>(n_rows, 1));
+  g->redo_m = dalloc<int32_t>(g, std::max<int64_t>(n_rows, 1));
+  g->redo_l = dalloc<int32_t>(g, std::max<int64_t>(n_rows, 1));
+  g->d_sched = dalloc<Sched>(g, 1);
   // giant rows: the prefix with deg > kGiantMin, split into segments
   g->n_giant = 0;
   for (const BinItem& it : row_i) g->n_giant += it.d > kGiantMin;
   if (g->n_giant > 0) {
-    if (maxd >= ((int64_t)1 << kGCountBits))
+    if (g->max_deg >= ((int64_t)1 << kGCountBits))
       fail(GLP_ERR_UNSUPPORTED, "a row has >= 2^25 arcs (giant-row table count field)");
     std::vector<GiantSeg> segs;
     std::vector<int32_t> first;
@@ -232,30 +271,21 @@ void build_layout(glp_graph* g, const int64_t* off_h, const int64_t* off_d, cons
     g->gtab_off = upload(g, toff);
     g->gtab_slots = slots;
     g->gtab = dalloc<unsigned long long>(g, slots);
-    CK(cudaMemsetAsync(g->gtab, 0, slots * sizeof(unsigned long long), g->stream));
+    CK(cudaMemsetAsync(g->gtab, 0, slots * sizeof(unsigned long long), s));
     g->gepoch = 0;
     g->gcand_key = dalloc<unsigned long long>(g, segs.size());
     g->gcand_lab = dalloc<unsigned>(g, segs.size());
     g->gdistinct = dalloc<unsigned>(g, g->n_giant);
-    CK(cudaMemsetAsync(g->gdistinct, 0, g->n_giant * sizeof(unsigned), g->stream));
+    CK(cudaMemsetAsync(g->gdistinct, 0, g->n_giant * sizeof(unsigned), s));
   }
-  g->low_list = upload(g, low);
-  g->chunks = upload(g, chunks);
-  g->cflag = dalloc<uint8_t>(g, std::max<int32_t>(g->n_chunks, 1));
-  g->rows = upload(g, row_i);
-  g->pred[0] = dalloc<unsigned>(g, std::max<int32_t>(g->n_rows, 1));
-  g->pred[1] = dalloc<unsigned>(g, std::max<int32_t>(g->n_rows, 1));
-  g->redo_m = dalloc<int32_t>(g, std::max<int32_t>(g->n_rows, 1));
-  g->redo_l = dalloc<int32_t>(g, std::max<int32_t>(g->n_rows, 1));
-  g->d_sched = dalloc<Sched>(g, 1);
-  g->ioff = upload(g, ioff);
-  g->ideg = upload(g, ideg);
+  // ---- the arcs themselves
   g->col2 = dalloc<int32_t>(g, g->nnz2);
-  CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), g->stream));  // padding = -1
-  if (g->nl > 0 && g->nnz > 0) {
-    k_relayout<<<g->sms * 8, 256, 0, g->stream>>>(off_d, col_d, g->ioff, g->nl, g->col2);
+  CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), s));  // padding = -1
+  if (nl > 0 && g->nnz > 0) {
+    k_relayout<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, nl, g->col2);
     CK(cudaGetLastError());
   }
+  CK(cudaStreamSynchronize(s));
 }
 
 void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm, glp_graph** out) {
@@ -315,20 +345,13 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     if (g->nnz >= ((int64_t)1 << 40)) fail(GLP_ERR_INVALID_ARGUMENT, "nnz_local too large");
 
     g->sms = prop.multiProcessorCount;
-    std::vector<int64_t> off_h;
-    const int64_t* off_host = nullptr;
     const int64_t* off_d = nullptr;
     const int32_t* col_d = nullptr;
     std::vector<void*> temps;  // caller-CSR staging freed after the relayout
     if (csr->on_device) {
       off_d = csr->row_offsets;
       col_d = csr->col_idx;
-      off_h.resize(g->nl + 1);
-      CK(cudaMemcpyAsync(off_h.data(), off_d, (g->nl + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, g->stream));
-      CK(cudaStreamSynchronize(g->stream));
-      off_host = off_h.data();
     } else {
-      off_host = csr->row_offsets;
       void *po = nullptr, *pc = nullptr;
       if (cudaMalloc(&po, (g->nl + 1) * sizeof(int64_t)) != cudaSuccess ||
           cudaMalloc(&pc, std::max<int64_t>(g->nnz, 1) * sizeof(int32_t)) != cudaSuccess) {
@@ -354,23 +377,22 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
         for (void* p : v) cudaFree(p);
       }
     } tg{temps, g->stream};
-    // host-side structural checks on the offsets (cheap, always on)
-    if (off_host[0] != 0 || off_host[g->nl] != g->nnz)
-      fail(GLP_ERR_INVALID_GRAPH, "row_offsets[0] must be 0 and row_offsets[last] == nnz_local");
-    for (int64_t v = 0; v < g->nl; ++v)
-      if (off_host[v + 1] < off_host[v]) fail(GLP_ERR_INVALID_GRAPH, "row_offsets not non-decreasing");
-    if (p.validate && g->nnz) {
+    // structural checks on the device: off[0] == 0, off[nl] == nnz, monotone
+    // offsets (always); col in [0, n) (validate = 1)
+    {
       int* dbad = dalloc<int>(g, 1);
       CK(cudaMemsetAsync(dbad, 0, sizeof(int), g->stream));
-      k_validate_col<<<g->sms * 4, 256, 0, g->stream>>>(col_d, g->nnz, g->n, dbad);
+      k_validate_off<<<g->sms * 4, 256, 0, g->stream>>>(off_d, g->nl, g->nnz, dbad);
+      if (p.validate && g->nnz) k_validate_col<<<g->sms * 4, 256, 0, g->stream>>>(col_d, g->nnz, g->n, dbad);
       CK(cudaGetLastError());
       int bad = 0;
       CK(cudaMemcpyAsync(&bad, dbad, sizeof(int), cudaMemcpyDeviceToHost, g->stream));
       CK(cudaStreamSynchronize(g->stream));
-      if (bad) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
+      if (bad & 3) fail(GLP_ERR_INVALID_GRAPH, "row_offsets[0] must be 0 and row_offsets[last] == nnz_local");
+      if (bad & 4) fail(GLP_ERR_INVALID_GRAPH, "row_offsets not non-decreasing");
+      if (bad & 8) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
     }
-    build_layout(g, off_host, off_d, col_d);
-    CK(cudaStreamSynchronize(g->stream));
+    build_layout(g, off_d, col_d);
 
     // labels: replicated full arrays, padded to a multiple of nranks for the
     // in-place all-gather
