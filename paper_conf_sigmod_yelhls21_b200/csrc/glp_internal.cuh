@@ -59,6 +59,9 @@ constexpr int kGUnroll = 2;
 constexpr int kGCountBits = 25;  // count field of a giant-table slot (deg < 2^25)
 constexpr int kGEpochBits = 64 - 31 - kGCountBits;
 enum RowClass { CLS_W = 0, CLS_M = 1, CLS_L = 2, CLS_G = 3 };
+// pred word: low 31 bits = predicted distinct labels; bit 31 = the row took
+// the sorted-row fast path last time (do not retry it)
+constexpr unsigned kPredMask = 0x7fffffffu, kMonoTried = 0x80000000u;
 __host__ __device__ __forceinline__ int row_class(unsigned pred, int d) {
   if (d > kGiantMin) return CLS_G;
   if (pred <= kWPred && d <= kWMaxDeg) return CLS_W;

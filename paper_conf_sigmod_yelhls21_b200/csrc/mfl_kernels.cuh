@@ -34,6 +34,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <climits>
+
 #include "glp_internal.cuh"
 
 namespace glp {
@@ -382,6 +384,47 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
 }
 
 // ---------------------------------------------------------------------------
+// Sorted-row fast path.  If the labels of a row, read in arc order, are all
+// valid and strictly increasing, every label occurs exactly once: each count is
+// 1 and no table is needed (the scores are observed directly).  This is the
+// case at t = 1 (unique labels L0[u] = u [P:68]) whenever the CSR rows are
+// sorted, and is checked on the data, never assumed.  Rows only try it when
+// their predicted distinct count equals their degree.
+//
+// Lane-local part: labels x[0..3] at arcs idx0..idx0+3 (valid while < d).
+__device__ __forceinline__ bool quad_increasing(const int (&x)[4], int idx0, int d) {
+  bool ok = true;
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    if (idx0 + k < d) {
+      ok &= x[k] >= 0;
+      if (k > 0) ok &= x[k - 1] < x[k];
+    }
+  }
+  return ok;
+}
+
+// Warp-level check of one 128-arc quad row (lane l holds arcs base+4l..+3);
+// `prev` is the label of the arc just before `base` (-1 at the row start).
+// Returns the warp-uniform verdict and the last valid label in *last.
+__device__ __forceinline__ bool warp_quads_increasing(const int (&x)[4], int base, int d, int prev, int* last) {
+  const int lane = threadIdx.x & 31;
+  const int idx0 = base + 4 * lane;
+  bool ok = quad_increasing(x, idx0, d);
+  const int nxt = __shfl_down_sync(kFull, x[0], 1);
+  if (lane < 31 && idx0 + 4 < d) ok &= x[3] < nxt;   // lane boundary
+  const int first = __shfl_sync(kFull, x[0], 0);
+  if (base < d) ok &= prev < first;                   // boundary with the previous quad row
+  // last valid label of this quad row
+  const int lastidx = min(d, base + 128) - 1 - base;   // >= 0 when base < d
+  const int src = max(lastidx, 0) >> 2, k = max(lastidx, 0) & 3;
+  const int mine = k == 0 ? x[0] : k == 1 ? x[1] : k == 2 ? x[2] : x[3];
+  const int lv = __shfl_sync(kFull, mine, src);
+  *last = base < d ? lv : prev;
+  return __all_sync(kFull, ok);
+}
+
+// ---------------------------------------------------------------------------
 // mfl_warp: one warp per row of class W (few distinct labels): per-warp shared
 // table of pow2 >= 2*pred slots (<= 512), two 128-bit loads per lane per
 // round (256 arcs in flight per warp), no block barriers.  Rows whose labels
@@ -407,8 +450,8 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
     if (ok) {
       mine = a.items[il];
       const unsigned raw = a.pred[il];
-      mpred = a.pred_cap ? min(raw, a.pred_cap) : raw;
-      ok = row_class(mpred, mine.d) == CLS_W;
+      mpred = a.pred_cap ? min(raw & kPredMask, a.pred_cap) | (raw & kMonoTried) : raw;
+      ok = row_class(mpred & kPredMask, mine.d) == CLS_W;
       if (ok && !a.dense && !a.flag[a.vb + mine.v]) {
         ok = false;
         a.pred_next[il] = raw;  // inactive: carry the prediction forward
@@ -424,7 +467,7 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
     it.v = __shfl_sync(kFull, mine.v, jl);
     it.d = __shfl_sync(kFull, mine.d, jl);
     const unsigned pred = __shfl_sync(kFull, mpred, jl);
-    const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * max(pred, 1u) - 1u))), (unsigned)kWSlots);
+    const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
     const Table tab{tabs[wid], tsz};
     tab.clear(lane, 32);
     if (lane == 0) s_over[wid] = 0;
@@ -432,6 +475,9 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
     Best<VAR> b;
     unsigned fresh = 0;
     bool over = false;
+    bool mono = VAR != V_SEEDED && !(pred & kMonoTried) && pred >= (unsigned)it.d;  // sorted-row candidate
+    const bool tried = mono;
+    int prev = -1;
     for (int base = 0; base < it.d && !over; base += 256) {
       int4 u0 = make_int4(-1, -1, -1, -1), u1 = u0;
       if (base + 4 * lane < it.d) u0 = ld_stream4(a.col + it.start + base + 4 * lane);
@@ -439,6 +485,31 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
       int l[8];
       l[0] = gather(a, u0.x); l[1] = gather(a, u0.y); l[2] = gather(a, u0.z); l[3] = gather(a, u0.w);
       l[4] = gather(a, u1.x); l[5] = gather(a, u1.y); l[6] = gather(a, u1.z); l[7] = gather(a, u1.w);
+      if (mono) {
+        const int q0[4] = {l[0], l[1], l[2], l[3]}, q1[4] = {l[4], l[5], l[6], l[7]};
+        int mid = -1, end = -1;
+        bool ok = warp_quads_increasing(q0, base, it.d, prev, &mid);
+        ok = ok && warp_quads_increasing(q1, base + 128, it.d, mid, &end);
+        if (ok) {  // every label of this round occurs once in the row so far
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            if (l[j] >= 0) { b.observe(1u, (unsigned)l[j], a); ++fresh; }
+          prev = end;
+          continue;
+        }
+        // not sorted: count this row with the table, re-inserting the rounds
+        // already observed (their count-1 observations stay valid lower bounds)
+        mono = false;
+        fresh = 0;
+        for (int b2 = 0; b2 < base; b2 += 256) {
+          int4 v0 = make_int4(-1, -1, -1, -1), v1 = v0;
+          if (b2 + 4 * lane < it.d) v0 = ld_stream4(a.col + it.start + b2 + 4 * lane);
+          if (b2 + 128 + 4 * lane < it.d) v1 = ld_stream4(a.col + it.start + b2 + 128 + 4 * lane);
+          const int m8[8] = {gather(a, v0.x), gather(a, v0.y), gather(a, v0.z), gather(a, v0.w),
+                             gather(a, v1.x), gather(a, v1.y), gather(a, v1.z), gather(a, v1.w)};
+          fresh += warp_insert_n<VAR, 8>(a, tab, tsz, m8, b, &s_over[wid]);
+        }
+      }
       if (it.d - base > 128) {  // warp-uniform
         fresh += warp_insert_n<VAR, 8>(a, tab, tsz, l, b, &s_over[wid]);
       } else {
@@ -456,7 +527,8 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
     b.warp_reduce();
     fresh = __reduce_add_sync(kFull, fresh);
     if (lane == 0) {
-      a.pred_next[i] = max(fresh, 1u);
+      // a row that just took the sorted fast path is not retried next time
+      a.pred_next[i] = max(fresh, 1u) | (tried && mono ? kMonoTried : 0u);
       update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
     }
     __syncwarp();
@@ -520,6 +592,51 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
     fresh = __reduce_add_sync(kFull, fresh);
     if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
   }
+}
+
+// Block-level sorted-row fast path (see warp_quads_increasing): one 128-bit
+// load per thread per 4*BLOCK arcs; warps check their own 128-arc quad rows,
+// thread 0 chains the warp boundaries.  Returns the block-uniform verdict; on
+// success every label has been observed with count 1 and *fresh counts them.
+template <int VAR, int BLOCK>
+__device__ __forceinline__ bool block_mono(const MflArgs& a, int64_t start, int d, Best<VAR>& b, unsigned* fresh) {
+  constexpr int NW = BLOCK / 32;
+  __shared__ int s_first[NW], s_last[NW], s_ok, s_prev;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  int prev_round = -1;
+  for (int base = 0; base < d; base += 4 * BLOCK) {
+    const int wb = base + 128 * wid;
+    int x[4] = {-1, -1, -1, -1};
+    if (wb + 4 * lane < d) {
+      const int4 u = ld_stream4(a.col + start + wb + 4 * lane);
+      x[0] = gather(a, u.x); x[1] = gather(a, u.y); x[2] = gather(a, u.z); x[3] = gather(a, u.w);
+    }
+    int lastw = -1;
+    const bool okw = warp_quads_increasing(x, wb, d, INT_MIN, &lastw);
+    if (lane == 0) {
+      s_first[wid] = x[0];
+      s_last[wid] = lastw;
+    }
+    const int ok_all = __syncthreads_and(okw ? 1 : 0);
+    if (threadIdx.x == 0) {
+      bool ok = ok_all != 0;
+      int p = prev_round;
+      for (int w = 0; w < NW; ++w)
+        if (base + 128 * w < d) {
+          ok = ok && p < s_first[w];
+          p = s_last[w];
+        }
+      s_ok = ok ? 1 : 0;
+      s_prev = p;
+    }
+    __syncthreads();
+    if (!s_ok) return false;
+    prev_round = s_prev;
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+      if (wb + 4 * lane + k < d) { b.observe(1u, (unsigned)x[k], a); ++*fresh; }
+  }
+  return true;
 }
 
 template <int VAR, int BLOCK>
@@ -607,7 +724,7 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
         if (!a.mode) {
           const BinItem itk = a.items[ik];
           const unsigned raw = a.pred[ik];
-          const unsigned pk = a.pred_cap ? min(raw, a.pred_cap) : raw;
+          const unsigned pk = a.pred_cap ? min(raw & kPredMask, a.pred_cap) : (raw & kPredMask);
           ok = row_class(pk, itk.d) == CLS;
           if (ok && !a.dense && !a.flag[a.vb + itk.v]) {
             ok = false;
@@ -624,10 +741,26 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
     for (int q = 0; q < nsel; ++q) {
     const int i = s_sel[q];
     const BinItem it = a.items[i];
-    const unsigned pred = a.pred_cap ? min(a.pred[i], a.pred_cap) : a.pred[i];
+    const unsigned praw = a.pred[i];
+    const bool tried_before = (praw & kMonoTried) != 0;
+    const unsigned pred = a.pred_cap ? min(praw & kPredMask, a.pred_cap) : (praw & kPredMask);
     const int d = it.d;
     Best<VAR> b;
     if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; }
+    bool mono_done = false;
+    if (!a.mode && VAR != V_SEEDED && !tried_before && pred >= (unsigned)d) {
+      __syncthreads();
+      unsigned fr = 0;
+      mono_done = block_mono<VAR, BLOCK>(a, it.start, d, b, &fr);
+      if (mono_done) {
+        fr = __reduce_add_sync(kFull, fr);
+        if ((threadIdx.x & 31) == 0 && fr) atomicAdd(&s_distinct, (int)fr);
+        __syncthreads();
+      } else {
+        b = Best<VAR>();
+      }
+    }
+    if (!mono_done) {
     // a re-queued row overflowed a smaller table: its pred is stale
     const unsigned est = a.mode ? (unsigned)d : max(pred, 1u);
     unsigned nparts = PART ? max(1u, (min(est, (unsigned)d) + SLOTS / 2 - 1) / (SLOTS / 2)) : 1u;
@@ -731,9 +864,10 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
         nparts = min(nparts * 2u, 255u);  // a part overflowed: finer partitions (exact recount)
       }
     }
+    }  // !mono_done
     b = block_best<VAR, BLOCK>(b);
     if (threadIdx.x == 0) {
-      a.pred_next[i] = max((unsigned)s_distinct, 1u);
+      a.pred_next[i] = max((unsigned)s_distinct, 1u) | (mono_done ? kMonoTried : 0u);
       update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty);
     }
     __syncthreads();

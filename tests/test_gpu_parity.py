@@ -162,6 +162,38 @@ def test_giant_rows_epoch_wrap():
         assert_same_run(csr, 2, 6, gamma=1.0)
 
 
+def _perturb_rows(csr, mode, seed=0):
+    """Same graph, different arc order inside rows: 'shuffle' every row, or
+    'tail' = swap the last two arcs of every row (sorted until the very end)."""
+    off, col = csr.numpy()
+    col = col.copy()
+    g = np.random.default_rng(seed)
+    for v in range(csr.n):
+        a, b = off[v], off[v + 1]
+        if b - a < 2:
+            continue
+        if mode == "shuffle":
+            col[a:b] = g.permutation(col[a:b])
+        else:
+            col[b - 2], col[b - 1] = col[b - 1], col[b - 2]
+    return from_arrays(csr.n, off, col)
+
+
+@pytest.mark.parametrize("mode", ["shuffle", "tail"])
+def test_unsorted_rows_sorted_fast_path(mode):
+    """The sorted-row fast path (t = 1) must agree with the table path on any
+    arc order, including rows that stop being sorted in their last round."""
+    base = _degree_mix([70000, 9000, 3000, 1500, 600, 300, 130, 40], seed=2, extra_pairs=40000)
+    for csr in [base, graphs.rmat(13, seed=3)]:
+        pert = _perturb_rows(csr, mode)
+        for variant, gamma in [(0, 0.0), (2, 0.5)]:
+            a = gpu(csr, variant, 6, gamma=gamma)
+            b = gpu(pert, variant, 6, gamma=gamma)
+            assert (a[0] == b[0]).all()
+            ref = oracle.run(pert, variant, 6, gamma=gamma, threads=8)
+            assert (b[0] == ref.labels).all()
+
+
 def test_hub_with_few_labels_and_ties():
     # a hub whose neighbours carry a handful of labels: hot keys (warp
     # aggregation) and an exact tie resolved to the smaller label
