@@ -432,7 +432,9 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 2 * g->grid_l);
     }
     g->nnz_global = g->nnz;
-    if (nranks > 1) nccl_init(g, dist->nccl_unique_id);
+    // NCCL exchange for nranks > 1; with nranks == 1 a unique id still selects
+    // the NCCL path (a one-rank communicator), which tests its plumbing on one GPU
+    if (nranks > 1 || (dist && dist->nccl_unique_id)) nccl_init(g, dist->nccl_unique_id);
     CK(cudaStreamSynchronize(g->stream));
   } catch (...) {
     free_graph(g);
@@ -612,7 +614,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       g->init_launches += 1;
       CK(cudaGetLastError());
       g->flag_clean[fb] = false;
-      if (g->nranks > 1) nccl_merge_flags(g, g->flag[fb]);
+      if (g->nccl) nccl_merge_flags(g, g->flag[fb]);
       if (g->n_chunks) {
         k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_list, g->flag[fb], g->vb, g->cflag);
         g->init_launches += 1;
@@ -676,7 +678,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
       default: launches += launch_mfl<V_LLP>(g, a, prof, pend, used); break;
     }
-    if (g->nranks > 1) {
+    if (g->nccl) {
       timed(g, prof, 6, pend, used, [&] { nccl_exchange(g, g->L[1 - rb]); });
       nccl_sum_counters(g, g->d_cnt, 5 * sizeof(Counters) / sizeof(unsigned long long));
     }
@@ -719,7 +721,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       launches += 1;
       timed(g, prof, 4, pend, used, [&] {
         k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, g->flag[nf]);
-        if (g->nranks > 1) nccl_merge_flags(g, g->flag[nf]);
+        if (g->nccl) nccl_merge_flags(g, g->flag[nf]);
         if (g->n_chunks)
           k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_list, g->flag[nf], g->vb, g->cflag);
       });

@@ -311,19 +311,38 @@ __device__ __forceinline__ void update_vertex(const MflArgs& a, int v, int deg, 
 }
 
 // ---------------------------------------------------------------------------
-// mfl_low: one warp per chunk = up to 32 consecutive arcs of several low-degree
-// vertices.  Fig. 3 / [P:229-232]: activemask = lanes holding a valid label;
-// vmask = lanes of the same vertex (from the chunk's segment-start bitmap);
-// frequency = number of lanes of vmask with the same label (a shuffle loop as
-// long as the chunk's longest segment: match.any.sync costs ~60 SM cycles per
-// warp on distinct keys on sm_100, tools/ubench); arg-max = shuffle tree over
-// the segment.
+// mfl_low: one warp per chunk = floor(32/deg) low-degree vertices of one
+// degree `deg`, their arcs filling lanes [j*deg, (j+1)*deg) ("one-warp-multi-
+// vertices" [P:227-234 §4.2]).  activemask = lanes holding a valid label;
+// vmask = the deg lanes of a vertex; frequency of a lane's label = number of
+// vmask lanes with the same label (a shuffle loop of deg steps: match.any.sync
+// costs ~60 SM cycles per warp on distinct keys on sm_100, tools/ubench);
+// arg-max = shuffle tree toward the segment head, then lane j updates vertex
+// j.  Loads of the next chunk (arcs, vertex ids) are issued before the current
+// chunk is counted (software pipelining across the warp's chunks).
+template <int VAR>
+__device__ __forceinline__ void update_vertex_pre(const MflArgs& a, int v, int deg, bool have, unsigned best, int r,
+                                                  int2 so, Tally& ty) {
+  const int64_t gv = a.vb + v;
+  int nw = have ? (int)best : r;
+  if (VAR == V_SEEDED && a.is_seed[v]) nw = r;  // clamped seed (R12)
+  const int l2 = (so.x == a.t - 1) ? so.y : r;  // L_{t-2}[v]
+  a.W[gv] = nw;
+  ty.verts += 1;
+  ty.arcs += (unsigned long long)deg;
+  ty.d2 += (nw != l2);
+  if (nw != r) {
+    ty.changed += 1;
+    ty.chdeg += (unsigned long long)deg;
+    a.so[v] = make_int2(a.t, r);
+  }
+}
+
 template <int VAR>
 __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
   const int lane = threadIdx.x & 31;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
-  const unsigned le = kFull >> (31 - lane);  // lanes 0..lane
   Tally ty;
   // each warp takes 32 consecutive chunks at a time; in sparse iterations the
   // inactive ones are skipped with one coalesced read of their chunk flags
@@ -337,48 +356,74 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       if (!a.dense) act = a.cflag[cl] != 0;
     }
     unsigned todo = __ballot_sync(kFull, act);
-    while (todo) {
-    const int j = __ffs(todo) - 1;
+    if (!todo) continue;
+    // issue the arc and vertex-id loads of chunk j
+    auto issue = [&](int j, int& u, int& v, int& total, int& nv) {
+      const unsigned long long st = __shfl_sync(kFull, mine.st, j);
+      const int vbase = __shfl_sync(kFull, mine.vbase, j);
+      const unsigned segs = __shfl_sync(kFull, mine.segmask, j);
+      total = (int)(st >> 56);
+      nv = __popc(segs);
+      const int64_t start = (int64_t)(st & ((1ull << 56) - 1));
+      u = lane < total ? ld_stream(a.col + start + lane) : -1;
+      v = lane < nv ? a.list[vbase + lane] : -1;
+    };
+    int j = __ffs(todo) - 1;
     todo &= todo - 1;
-    LowChunk ch;
-    ch.st = __shfl_sync(kFull, mine.st, j);
-    ch.vbase = __shfl_sync(kFull, mine.vbase, j);
-    ch.segmask = __shfl_sync(kFull, mine.segmask, j);
-    const int64_t start = (int64_t)(ch.st & ((1ull << 56) - 1));
-    const int total = (int)(ch.st >> 56);
-    const unsigned segs = ch.segmask;
-    const bool valid = lane < total;
-    const unsigned below = segs & le;
-    const int seg = __popc(below) - 1;                   // vertex index in chunk
-    const int vstart = 31 - __clz(below | 1u);           // first lane of my vertex
-    const unsigned above = segs & ~le;
-    const int vend = above ? __ffs(above) - 1 : total;   // one past my last lane
-    const int vd = vend - vstart;
-    int lab = -1;
-    if (valid) lab = gather(a, ld_stream(a.col + start + lane));
-    const bool vote = valid && lab >= 0;
-    if (!vote) lab = -1;
-    // label frequency inside the vertex's lanes [P:231-232]
-    const unsigned maxlen = __reduce_max_sync(kFull, valid ? (unsigned)vd : 0u);
-    unsigned k = 0;
-    for (unsigned j = 0; j < maxlen; ++j) {
-      const int other = __shfl_sync(kFull, lab, (vstart + (int)j) & 31);
-      k += (j < (unsigned)vd && other == lab) ? 1u : 0u;
-    }
-    // segmented arg-max toward the segment's first lane
-    Best<VAR> b;
-    if (vote) b.observe(k, (unsigned)lab, a);
+    int u, v, total, nv;
+    issue(j, u, v, total, nv);
+    for (;;) {
+      // prefetch the next chunk while this one is counted
+      int nu = -1, nvid = -1, ntotal = 0, nnv = 0;
+      const bool more = todo != 0;
+      if (more) {
+        const int nj = __ffs(todo) - 1;
+        todo &= todo - 1;
+        issue(nj, nu, nvid, ntotal, nnv);
+      }
+      const int d = total / nv;  // every vertex of the chunk has degree d
+      int lab = gather(a, u);
+      int r = 0;
+      int2 so = make_int2(0, 0);
+      if (lane < nv) {
+        r = ld_label(a.R + a.vb + v);
+        so = a.so[v];
+      }
+      const bool vote = lane < total && lab >= 0;
+      if (!vote) lab = -1;
+      const int sstart = (lane / d) * d, send = sstart + d;
+      // label frequency inside the vertex's lanes [P:231-232]
+      unsigned k = 0;
+      for (int i = 0; i < d; ++i) {
+        const int other = __shfl_sync(kFull, lab, (sstart + i) & 31);
+        k += other == lab ? 1u : 0u;
+      }
+      Best<VAR> b;
+      if (vote) b.observe(k, (unsigned)lab, a);
+      if (d > 1) {  // warp-uniform: segmented arg-max toward the segment head
 #pragma unroll
-    for (int s = 1; s < 32; s <<= 1) {
-      const unsigned long long ok = __shfl_down_sync(kFull, b.key, s);
-      const unsigned ol = VAR == V_LLP ? __shfl_down_sync(kFull, b.lab, s) : 0u;
-      if (lane + s < vend) b.merge(ok, ol);
+        for (int s2 = 1; s2 < 32; s2 <<= 1) {
+          const unsigned long long ok = __shfl_down_sync(kFull, b.key, s2);
+          const unsigned ol = VAR == V_LLP ? __shfl_down_sync(kFull, b.lab, s2) : 0u;
+          if (s2 < d && lane + s2 < send) b.merge(ok, ol);
+        }
+      }
+      // lane jv takes the result of segment jv (head lane jv*d)
+      const int head = (lane < nv ? lane * d : 0) & 31;
+      const unsigned long long bk = __shfl_sync(kFull, b.key, head);
+      const unsigned bl = VAR == V_LLP ? __shfl_sync(kFull, b.lab, head) : 0u;
+      if (lane < nv) {
+        Best<VAR> h;
+        h.key = bk;
+        h.lab = bl;
+        update_vertex_pre<VAR>(a, v, d, h.have(), h.label(), r, so, ty);
+      }
+      if (!more) break;
+      u = nu;
+      v = nvid;
+      total = ntotal;
+      nv = nnv;
     }
-    if (valid && lane == vstart) {
-      const int v = a.list[ch.vbase + seg];
-      update_vertex<VAR>(a, v, vd, b.have(), b.label(), ty);
-    }
-    }  // todo
   }
   tally_flush(ty, a.cnt);
 }

@@ -309,3 +309,25 @@ def test_error_codes():
     with pytest.raises(glp.GlpError) as e:
         glp.Graph(bad)
     assert e.value.status == 2
+
+
+def test_nccl_exchange_path_single_rank():
+    """A one-rank NCCL communicator drives the multi-GPU exchange code
+    (all-gather of labels, counter all-reduce, frontier-mark reduce-scatter)
+    on one GPU; results must equal the single-GPU path and the oracle."""
+    for csr, variant, seeds, gamma in [(graphs.rmat(14, seed=8), "classic", None, 0.0),
+                                       (graphs.rmat(13, seed=9), "llp", None, 1.0)]:
+        uid = glp.glp_nccl_unique_id()
+        c = csr.to("cuda")
+        with glp.Graph(c, rank=0, nranks=1, nccl_unique_id=uid, device=0) as g:
+            info = g.run(variant, 12, seeds, gamma=gamma)
+            lab = g.labels("cpu").numpy()
+        ref = oracle.run(csr, glp.VARIANTS[variant], 12, gamma=gamma, threads=8)
+        assert info.iterations == ref.iterations and (lab == ref.labels).all()
+    csr, seeds = graphs.taobao(users=40_000, items=10_000, pairs=200_000, rings=40, seed=5)
+    uid = glp.glp_nccl_unique_id()
+    with glp.Graph(csr.to("cuda"), rank=0, nranks=1, nccl_unique_id=uid, device=0) as g:
+        info = g.run("seeded", 30, seeds.numpy())
+        lab = g.labels("cpu").numpy()
+    ref = oracle.run(csr, oracle.SEEDED, 30, seeds=seeds.numpy(), threads=8)
+    assert info.iterations == ref.iterations and (lab == ref.labels).all()
