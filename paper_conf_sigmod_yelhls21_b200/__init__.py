@@ -19,7 +19,8 @@ import torch
 from . import _build
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = _build.LIB
+# GLP_LIB: load another in-tree build of the same library (kernel A/B experiments)
+LIB_PATH = os.environ.get("GLP_LIB") or _build.LIB
 
 CLASSIC, SEEDED, LLP = 0, 1, 2
 VARIANTS = {"classic": CLASSIC, "seeded": SEEDED, "llp": LLP}
@@ -192,8 +193,15 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
         d.cuda_stream = stream.cuda_stream if stream is not None else None
     h = ctypes.c_void_p()
     prm = make_params(validate=validate)
-    _check(lib.glp_graph_create(ctypes.byref(c), None if d is None else ctypes.byref(d),
-                                ctypes.byref(prm), ctypes.byref(h)))
+    st = lib.glp_graph_create(ctypes.byref(c), None if d is None else ctypes.byref(d), ctypes.byref(prm),
+                              ctypes.byref(h))
+    if st == 3 and torch.cuda.is_available():
+        # GLP_ERR_OUT_OF_MEMORY: the library allocates with cudaMalloc, so
+        # return torch's cached blocks to the driver and try once more
+        torch.cuda.empty_cache()
+        st = lib.glp_graph_create(ctypes.byref(c), None if d is None else ctypes.byref(d), ctypes.byref(prm),
+                                  ctypes.byref(h))
+    _check(st)
     return h
 
 

@@ -31,14 +31,16 @@ def needs_build() -> bool:
     return any(os.path.getmtime(s) > t for s in sources())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, out: str = LIB, defines=()) -> str:
+    """Compile csrc/glp.cu -> `out` (default: the in-tree libglp.so).  `defines`
+    (-D flags) are only used for kernel A/B variants built under build/."""
+    if out == LIB and not force and not needs_build():
         return LIB
-    cmd = [NVCC] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + [
-        "-o", LIB + ".tmp", os.path.join(CSRC, "glp.cu"), "-ldl"]
+    cmd = [NVCC] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + [f"-D{d}" for d in defines] + [
+        "-o", out + ".tmp", os.path.join(CSRC, "glp.cu"), "-ldl"]
     subprocess.check_call(cmd)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(out + ".tmp", out)
+    return out
 
 
 if __name__ == "__main__":

@@ -24,27 +24,38 @@ __global__ void k_validate_col(const int32_t* __restrict__ col, int64_t nnz, int
 }
 
 // PickLabel [P:99, P:109]: L[v] = v (CLASSIC, LLP) or UNLABELED (SEEDED, R12).
-__global__ void k_init_labels(int32_t* __restrict__ L0, int32_t* __restrict__ L1, int64_t n, int seeded) {
-  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t x = seeded ? -1 : (int32_t)v;
-    L0[v] = x;
-    L1[v] = x;
+// Arrays are indexed by internal id q (layout.cuh); the label value is the
+// original id orig[q].
+__global__ void k_init_labels(int32_t* __restrict__ L0, int32_t* __restrict__ L1, const int32_t* __restrict__ orig,
+                              int64_t n, int seeded) {
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t x = seeded ? -1 : orig[q];
+    L0[q] = x;
+    L1[q] = x;
   }
+}
+
+// glp_labels_get: out[v] = L[pos[v]] (original order)
+__global__ void k_unpermute(const int32_t* __restrict__ L, const int32_t* __restrict__ pos, int64_t n,
+                            int32_t* __restrict__ out) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    out[v] = L[pos[v]];
 }
 
 // Seeds carry their own id; owned seeds are marked and recorded as "changed at
 // t = 0" so that the first frontier is N(S) (exact: every other vertex has no
 // labelled neighbour and keeps -1, R5).
-__global__ void k_init_seeds(const int32_t* __restrict__ seeds, int64_t ns, int32_t* __restrict__ L0,
-                             int32_t* __restrict__ L1, uint8_t* __restrict__ is_seed, int2* __restrict__ so,
-                             int64_t vb, int64_t ve) {
+__global__ void k_init_seeds(const int32_t* __restrict__ seeds, int64_t ns, const int32_t* __restrict__ pos,
+                             int32_t* __restrict__ L0, int32_t* __restrict__ L1, uint8_t* __restrict__ is_seed,
+                             int2* __restrict__ so, int64_t vb, int64_t ve) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < ns; i += (int64_t)gridDim.x * blockDim.x) {
     const int32_t s = seeds[i];
-    L0[s] = s;
-    L1[s] = s;
-    if (s >= vb && s < ve) {
-      is_seed[s - vb] = 1;
-      so[s - vb] = make_int2(0, s);
+    const int32_t q = pos[s];
+    L0[q] = s;
+    L1[q] = s;
+    if (q >= vb && q < ve) {
+      is_seed[q - vb] = 1;
+      so[q - vb] = make_int2(0, s);
     }
   }
 }
@@ -75,27 +86,29 @@ __global__ void k_push(const int64_t* __restrict__ ioff, const int32_t* __restri
 }
 
 // Sparse iterations: a low-degree chunk is active if any of its vertices is.
-__global__ void k_chunk_flags(const LowChunk* __restrict__ chunks, int32_t n_chunks,
-                              const int32_t* __restrict__ list, const uint8_t* __restrict__ flag, int64_t vb,
-                              uint8_t* __restrict__ cflag) {
+__global__ void k_chunk_flags(const LowChunk* __restrict__ chunks, int32_t n_chunks, int64_t low_base,
+                              const uint8_t* __restrict__ flag, int64_t vb, uint8_t* __restrict__ cflag) {
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n_chunks; c += (int64_t)gridDim.x * blockDim.x) {
     const LowChunk ch = chunks[c];
     const int nv = __popc(ch.segmask);
     uint8_t act = 0;
-    for (int j = 0; j < nv && !act; ++j) act = flag[vb + list[ch.vbase + j]];
+    for (int j = 0; j < nv && !act; ++j) act = flag[vb + low_base + ch.vbase + j];
     cflag[c] = act ? 1 : 0;
   }
 }
 
-// Build the bin-major arc copy: row v of the caller's CSR -> col2[ioff[v]...].
+// Build the bin-major arc copy: row v of the caller's CSR (local original id)
+// -> col2[ioff[pos[vb + v] - vb] ...], each arc renamed to its internal id.
+// Arc order within a row is kept.
 __global__ void k_relayout(const int64_t* __restrict__ off, const int32_t* __restrict__ col,
-                           const int64_t* __restrict__ ioff, int64_t nl, int32_t* __restrict__ col2) {
+                           const int64_t* __restrict__ ioff, const int32_t* __restrict__ pos, int64_t nl, int64_t vb,
+                           int32_t* __restrict__ col2) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t v = gw; v < nl; v += nw) {
-    const int64_t s = off[v], d = off[v + 1] - s, o = ioff[v];
-    for (int64_t j = lane; j < d; j += 32) col2[o + j] = col[s + j];
+    const int64_t s = off[v], d = off[v + 1] - s, o = ioff[pos[vb + v] - vb];
+    for (int64_t j = lane; j < d; j += 32) col2[o + j] = pos[col[s + j]];
   }
 }
 

@@ -177,8 +177,11 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
   CK(cudaMemsetAsync(g->ioff, 0, std::max<int64_t>(nl, 1) * sizeof(int64_t), s));
   CK(cudaMemsetAsync(g->ideg, 0, std::max<int64_t>(nl, 1) * sizeof(int32_t), s));
   unsigned long long* keys = (unsigned long long*)talloc(std::max(n_low, n_rows) * sizeof(unsigned long long));
+  // orig_local[p] = local original id of internal vertex p: rows, low rows,
+  // isolated vertices (layout.cuh, internal vertex order)
+  int32_t* orig_local = (int32_t*)talloc(std::max<int64_t>(nl, 1) * sizeof(int32_t));
   // ---- low rows: sorted by (deg, id), packed floor(32/deg) per chunk
-  g->low_list = dalloc<int32_t>(g, n_low);
+  int32_t* low_list = orig_local + n_rows;
   LowGroups grp;
   memset(&grp, 0, sizeof(grp));
   int64_t vb = 0, cb = 0, ab = 0;
@@ -194,22 +197,23 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     }
   }
   g->n_low = (int32_t)n_low;
+  g->low_base = n_rows;
   g->n_chunks = (int32_t)cb;
   g->chunks = dalloc<LowChunk>(g, cb);
   g->cflag = dalloc<uint8_t>(g, std::max<int64_t>(cb, 1));
   const int64_t low_arcs = ab;
   if (n_low) {
     thrust::copy_if(pol, thrust::counting_iterator<int32_t>(0), thrust::counting_iterator<int32_t>((int32_t)nl),
-                    thrust::device_pointer_cast(g->low_list), IsLow{deg});
-    k_make_keys<<<gb, 256, 0, s>>>(g->low_list, n_low, deg, 0, keys);
+                    thrust::device_pointer_cast(low_list), IsLow{deg});
+    k_make_keys<<<gb, 256, 0, s>>>(low_list, n_low, deg, 0, keys);
     thrust::sort(pol, thrust::device_pointer_cast(keys), thrust::device_pointer_cast(keys) + n_low);
-    k_keys_to_ids<<<gb, 256, 0, s>>>(keys, n_low, g->low_list);
+    k_keys_to_ids<<<gb, 256, 0, s>>>(keys, n_low, low_list);
     k_low_chunks<<<gb, 256, 0, s>>>(grp, cb, n_low, g->chunks);
-    k_low_place<<<gb, 256, 0, s>>>(grp, g->low_list, n_low, deg, g->ioff, g->ideg);
+    k_low_place<<<gb, 256, 0, s>>>(grp, low_list, n_low, deg, n_rows, g->ioff, g->ideg);
     CK(cudaGetLastError());
   }
   // ---- other rows: (deg desc, id), 16-B aligned, padded to a multiple of 4
-  int32_t* rows = (int32_t*)talloc(n_rows * sizeof(int32_t));
+  int32_t* rows = orig_local;
   int64_t* pstart = (int64_t*)talloc((n_rows + 1) * sizeof(int64_t));
   const int64_t rows_base = (low_arcs + 3) & ~(int64_t)3;
   g->n_rows = (int32_t)n_rows;
@@ -233,7 +237,7 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     CK(cudaStreamSynchronize(s));
   }
   g->nnz2 = rows_base + padded_total;
-  if (g->nnz2 >= ((int64_t)1 << 56)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
+  if (g->nnz2 >= ((int64_t)1 << 48)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
   g->n_gt256 = g->n_gt2048 = g->n_ge8k = 0;
   for (const BinItem& it : row_i) {
     g->n_gt256 += it.d > 256;
@@ -278,11 +282,27 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     g->gdistinct = dalloc<unsigned>(g, g->n_giant);
     CK(cudaMemsetAsync(g->gdistinct, 0, g->n_giant * sizeof(unsigned), s));
   }
+  // ---- internal vertex order: isolated vertices last, then pos/orig of the
+  // owned slice; with several ranks the slices are all-gathered (every rank
+  // renames the global column ids of its arcs)
+  const int64_t n_iso = nl - n_rows - n_low;
+  if (n_iso)
+    thrust::copy_if(pol, thrust::counting_iterator<int32_t>(0), thrust::counting_iterator<int32_t>((int32_t)nl),
+                    thrust::device_pointer_cast(orig_local + n_rows + n_low), IsIso{deg});
+  g->pos = dalloc<int32_t>(g, std::max<int64_t>(g->npad, 1));
+  g->orig = dalloc<int32_t>(g, std::max<int64_t>(g->npad, 1));
+  if (nl) k_perm<<<gb, 256, 0, s>>>(orig_local, nl, g->vb, g->pos, g->orig);
+  if (g->npad > g->n) k_iota2<<<1, 256, 0, s>>>(g->pos, g->orig, g->n, g->npad);
+  CK(cudaGetLastError());
+  if (g->nccl) {
+    nccl_exchange(g, g->pos);
+    nccl_exchange(g, g->orig);
+  }
   // ---- the arcs themselves
   g->col2 = dalloc<int32_t>(g, g->nnz2);
   CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), s));  // padding = -1
   if (nl > 0 && g->nnz > 0) {
-    k_relayout<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, nl, g->col2);
+    k_relayout<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, g->pos, nl, g->vb, g->col2);
     CK(cudaGetLastError());
   }
   CK(cudaStreamSynchronize(s));
@@ -392,12 +412,16 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       if (bad & 4) fail(GLP_ERR_INVALID_GRAPH, "row_offsets not non-decreasing");
       if (bad & 8) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
     }
-    build_layout(g, off_d, col_d);
-
     // labels: replicated full arrays, padded to a multiple of nranks for the
     // in-place all-gather
     const int64_t npad = ((n + nranks - 1) / nranks) * nranks;
     g->npad = npad;
+    g->nnz_global = g->nnz;
+    // NCCL exchange for nranks > 1; with nranks == 1 a unique id still selects
+    // the NCCL path (a one-rank communicator), which tests its plumbing on one GPU
+    if (nranks > 1 || (dist && dist->nccl_unique_id)) nccl_init(g, dist->nccl_unique_id);
+    build_layout(g, off_d, col_d);
+
     g->L[0] = dalloc<int32_t>(g, npad);
     g->L[1] = dalloc<int32_t>(g, npad);
     g->so = dalloc<int2>(g, g->nl);
@@ -431,10 +455,6 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       g->stage_stride = (g->max_deg + 3) & ~(int64_t)3;
       g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 2 * g->grid_l);
     }
-    g->nnz_global = g->nnz;
-    // NCCL exchange for nranks > 1; with nranks == 1 a unique id still selects
-    // the NCCL path (a one-rank communicator), which tests its plumbing on one GPU
-    if (nranks > 1 || (dist && dist->nccl_unique_id)) nccl_init(g, dist->nccl_unique_id);
     CK(cudaStreamSynchronize(g->stream));
   } catch (...) {
     free_graph(g);
@@ -523,7 +543,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   }
   if (g->n_chunks) {
     MflArgs b = a;
-    b.list = g->low_list; b.chunks = g->chunks; b.cflag = g->cflag; b.n_chunks = g->n_chunks; b.cnt = c + 0;
+    b.low_base = g->low_base; b.chunks = g->chunks; b.cflag = g->cflag; b.n_chunks = g->n_chunks; b.cnt = c + 0;
     const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock - 1) / kLowBlock);
     timed(g, prof, 0, pend, used, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, g->stream>>>(b); });
     ++n;
@@ -569,7 +589,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   const int ga = g->grid_aux;
   // PickLabel
   g->init_launches = 1;
-  k_init_labels<<<ga, 256, 0, s>>>(g->L[0], g->L[1], g->npad, variant == GLP_VARIANT_SEEDED);
+  k_init_labels<<<ga, 256, 0, s>>>(g->L[0], g->L[1], g->orig, g->npad, variant == GLP_VARIANT_SEEDED);
   CK(cudaGetLastError());
   CK(cudaMemsetAsync(g->so, 0x80, std::max<int64_t>(g->nl, 1) * sizeof(int2), s));  // stamp = INT_MIN-ish
   CK(cudaMemsetAsync(g->is_seed, 0, std::max<int64_t>(g->nl, 1), s));
@@ -584,7 +604,8 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       g->seeds_cap = n_seeds;
     }
     CK(cudaMemcpyAsync(g->d_seeds, seeds, n_seeds * sizeof(int32_t), cudaMemcpyHostToDevice, s));
-    k_init_seeds<<<ga, 256, 0, s>>>(g->d_seeds, n_seeds, g->L[0], g->L[1], g->is_seed, g->so, g->vb, g->ve);
+    k_init_seeds<<<ga, 256, 0, s>>>(g->d_seeds, n_seeds, g->pos, g->L[0], g->L[1], g->is_seed, g->so, g->vb,
+                                     g->ve);
     g->init_launches += 1;
     CK(cudaGetLastError());
   }
@@ -616,7 +637,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       g->flag_clean[fb] = false;
       if (g->nccl) nccl_merge_flags(g, g->flag[fb]);
       if (g->n_chunks) {
-        k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_list, g->flag[fb], g->vb, g->cflag);
+        k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_base, g->flag[fb], g->vb, g->cflag);
         g->init_launches += 1;
       }
       dense = false;
@@ -723,7 +744,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
         k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, g->flag[nf]);
         if (g->nccl) nccl_merge_flags(g, g->flag[nf]);
         if (g->n_chunks)
-          k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_list, g->flag[nf], g->vb, g->cflag);
+          k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_base, g->flag[nf], g->vb, g->cflag);
       });
       launches += g->n_chunks ? 1 : 0;
       g->flag_clean[nf] = false;
@@ -789,8 +810,13 @@ glp_status glp_labels_get(const glp_graph* g, int32_t* out, int64_t out_len, int
     if (g->n == 0) return;
     if (!out) fail(GLP_ERR_INVALID_ARGUMENT, "out is NULL");
     CK(cudaSetDevice(g->device));
-    CK(cudaMemcpyAsync(out, g->L[g->cur], g->n * sizeof(int32_t),
-                       out_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, g->stream));
+    // back to original vertex order; the dead buffer L_{t-1} is the staging
+    // area of a host copy
+    int32_t* dst = out_on_device ? out : g->L[1 - g->cur];
+    k_unpermute<<<g->grid_aux, 256, 0, g->stream>>>(g->L[g->cur], g->pos, g->n, dst);
+    CK(cudaGetLastError());
+    if (!out_on_device)
+      CK(cudaMemcpyAsync(out, dst, g->n * sizeof(int32_t), cudaMemcpyDeviceToHost, g->stream));
     CK(cudaStreamSynchronize(g->stream));
   });
 }

@@ -10,7 +10,8 @@
 //                       label before it -> exact 2-cycle test (R8)
 //   flag[2] u8[n]       frontier marks by global id (sparse iterations only)
 //   V     int32[n]      LLP label histogram (LLP only)               [P:119]
-//   lists int32         degree-bin vertex lists + low-degree warp chunks
+//   pos/orig int32[n]   internal <-> original vertex ids (layout.cuh)
+//   chunks              low-degree warp chunks
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -83,7 +84,7 @@ struct Sched {
 };
 
 // A low-degree chunk: up to 32 consecutive arcs of consecutive low-list
-// vertices.  st = arc start in col2 | (arc count << 56); bit i of segmask set
+// vertices.  st = arc start in col2 | (degree << 48) | (arc count << 56); bit i of segmask set
 // iff a vertex's first arc is at lane i; vbase = index of its first vertex in
 // the low list.
 struct LowChunk {
@@ -122,7 +123,7 @@ struct MflArgs {
   const int32_t* __restrict__ V;        // LLP histogram [n] or null
   const uint8_t* __restrict__ is_seed;  // [nl] or null
   const uint8_t* __restrict__ flag;     // [npad] frontier marks by global id (sparse)
-  const int32_t* __restrict__ list;     // low bin: vertex list (local ids)
+  int64_t low_base;                     // low bin: internal id of low-list entry 0
   const LowChunk* __restrict__ chunks;  // low bin
   const uint8_t* __restrict__ cflag;    // low bin: chunk has an active vertex (sparse)
   int32_t n_chunks;
@@ -191,7 +192,10 @@ struct glp_graph {
   int32_t* col2 = nullptr;  int64_t nnz2 = 0;
   int64_t* ioff = nullptr;  // [nl] start of row v in col2
   int32_t* ideg = nullptr;  // [nl] degree of row v
-  int32_t* low_list = nullptr;  int32_t n_low = 0;
+  int32_t n_low = 0;
+  int64_t low_base = 0;     // internal id of the first low row (= n_rows)
+  int32_t* pos = nullptr;   // [npad] internal id of original vertex v (global)
+  int32_t* orig = nullptr;  // [npad] original id of internal vertex q (global)
   glp::LowChunk* chunks = nullptr;   int32_t n_chunks = 0;
   uint8_t* cflag = nullptr;          // [n_chunks] chunk activity (sparse iterations)
   glp::BinItem* rows = nullptr; int32_t n_rows = 0;  // deg > 32, degree-descending

@@ -6,7 +6,20 @@
 //    and its arcs are contiguous in col2;
 //  * rows with deg > 32 are sorted by (deg desc, id); each starts 16-B aligned
 //    and is padded with -1 to a multiple of 4;
-//  * ioff/ideg give every vertex's row in col2 (frontier push).
+//  * ioff/ideg give every vertex's row in col2 (frontier push);
+//  * vertices are renumbered into this layout order (internal ids, below).
+//
+// Internal vertex order.  The library numbers the owned vertices of a rank
+// by their layout position: rows with deg > 32 in (deg desc, id) order, then
+// the low rows in (deg, id) order, then the isolated vertices.  Row i of
+// `rows` is internal vertex i and low-list entry q is internal vertex
+// n_rows + q, so the kernels need no vertex-id tables, and the most gathered
+// labels (hubs: an arc's target is a hub with probability proportional to
+// its degree) sit together at the start of each rank's label slice, where
+// their 32-B sectors are shared and stay cached.  Only ids are permuted:
+// label VALUES remain original vertex ids (L0[pos[v]] = v), so scores, the
+// min-label tie-break (R4) and every result are unchanged; glp_labels_get
+// maps back.  A rank's owned range [vb, ve) maps onto itself.
 // Sorting and scans use thrust (a library primitive, the CUDA analogue of the
 // qsort the oracle uses); everything else is plain kernels.
 #pragma once
@@ -53,6 +66,10 @@ struct IsRow {
   const int32_t* deg;
   __host__ __device__ bool operator()(int64_t v) const { return deg[v] > kLowMax; }
 };
+struct IsIso {
+  const int32_t* deg;
+  __host__ __device__ bool operator()(int64_t v) const { return deg[v] == 0; }
+};
 
 // sort keys: low rows by (deg, id); other rows by (deg desc, id)
 __global__ void k_make_keys(const int32_t* __restrict__ ids, int64_t n, const int32_t* __restrict__ deg, int desc,
@@ -88,22 +105,25 @@ __global__ void k_low_chunks(LowGroups grp, int64_t n_chunks, int64_t n_low, Low
     unsigned mask = 0;
     for (int j = 0; j < nv; ++j) mask |= 1u << (j * d);
     LowChunk ch;
-    ch.st = (unsigned long long)(grp.abase[d] + q * (int64_t)k * d) | ((unsigned long long)(nv * d) << 56);
+    ch.st = (unsigned long long)(grp.abase[d] + q * (int64_t)k * d) | ((unsigned long long)d << 48) |
+            ((unsigned long long)(nv * d) << 56);
     ch.vbase = (int32_t)v0;
     ch.segmask = mask;
     chunks[c] = ch;
   }
 }
 
+// ioff/ideg of low-list entry q = internal vertex low_base + q
 __global__ void k_low_place(LowGroups grp, const int32_t* __restrict__ low, int64_t n_low,
-                            const int32_t* __restrict__ deg, int64_t* __restrict__ ioff, int32_t* __restrict__ ideg) {
+                            const int32_t* __restrict__ deg, int64_t low_base, int64_t* __restrict__ ioff,
+                            int32_t* __restrict__ ideg) {
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n_low; q += (int64_t)gridDim.x * blockDim.x) {
     const int32_t v = low[q];
     const int d = deg[v];
     const int k = 32 / d;
     const int64_t p = q - grp.vbase[d];
-    ioff[v] = grp.abase[d] + (p / k) * (int64_t)k * d + (p % k) * d;
-    ideg[v] = d;
+    ioff[low_base + q] = grp.abase[d] + (p / k) * (int64_t)k * d + (p % k) * d;
+    ideg[low_base + q] = d;
   }
 }
 
@@ -120,11 +140,30 @@ __global__ void k_row_place(const int32_t* __restrict__ rows, int64_t n, const i
     const int32_t v = rows[i];
     BinItem it;
     it.start = base + pstart[i];
-    it.v = v;
+    it.v = (int32_t)i;  // internal id of row i
     it.d = deg[v];
     items[i] = it;
-    ioff[v] = it.start;
-    ideg[v] = it.d;
+    ioff[i] = it.start;
+    ideg[i] = it.d;
+  }
+}
+
+// orig_local[p] -> pos/orig of the owned slice (global ids):
+//   orig[vb + p] = vb + orig_local[p],  pos[vb + orig_local[p]] = vb + p
+__global__ void k_perm(const int32_t* __restrict__ orig_local, int64_t nl, int64_t vb, int32_t* __restrict__ pos,
+                       int32_t* __restrict__ orig) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < nl; p += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = orig_local[p];
+    orig[vb + p] = (int32_t)(vb + v);
+    pos[vb + v] = (int32_t)(vb + p);
+  }
+}
+
+// identity on [a, b) (label-array padding beyond n_global)
+__global__ void k_iota2(int32_t* __restrict__ x, int32_t* __restrict__ y, int64_t a, int64_t b) {
+  for (int64_t i = a + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < b; i += (int64_t)gridDim.x * blockDim.x) {
+    x[i] = (int32_t)i;
+    y[i] = (int32_t)i;
   }
 }
 

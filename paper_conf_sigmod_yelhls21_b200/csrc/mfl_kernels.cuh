@@ -45,18 +45,60 @@ constexpr unsigned kNoLabel = 0xffffffffu;
 
 enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 
+// L2 policy of the two access streams: the arcs `col2`
+// are read once per iteration and must not evict the label array L_{t-1},
+// which every arc gathers from (64 MiB at RMAT-24, < 126 MB of L2), so arc
+// loads carry an L2 evict_first hint.  GLP_GATHER_POLICY selects the gathers'
+// hint: 0 none, 1 evict_last.
+#ifndef GLP_STREAM_POLICY
+#define GLP_STREAM_POLICY 1
+#endif
+#ifndef GLP_GATHER_POLICY
+#define GLP_GATHER_POLICY 0
+#endif
+// kernel A/B switches (tools/build_variants.py)
+#ifndef GLP_LOW_REDUX
+#define GLP_LOW_REDUX 1
+#endif
+#ifndef GLP_L_OPT
+#define GLP_L_OPT 1
+#endif
+#ifndef GLP_XROW
+#define GLP_XROW 1
+#endif
 __device__ __forceinline__ int ld_stream(const int32_t* p) {
   int r;
+#if GLP_STREAM_POLICY
+  asm volatile("{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_first.b64 pol, 1.0;\n\t"
+               "ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], pol;\n\t}"
+               : "=r"(r) : "l"(p));
+#else
   asm volatile("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(r) : "l"(p));
+#endif
   return r;
 }
 __device__ __forceinline__ int4 ld_stream4(const int32_t* p) {
   int4 r;
+#if GLP_STREAM_POLICY
+  asm volatile("{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_first.b64 pol, 1.0;\n\t"
+               "ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], pol;\n\t}"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+#else
   asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+#endif
   return r;
 }
-__device__ __forceinline__ int ld_label(const int32_t* p) { return __ldg(p); }
+__device__ __forceinline__ int ld_label(const int32_t* p) {
+#if GLP_GATHER_POLICY
+  int r;
+  asm volatile("{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
+               "ld.global.nc.L2::cache_hint.b32 %0, [%1], pol;\n\t}" : "=r"(r) : "l"(p));
+  return r;
+#else
+  return __ldg(p);
+#endif
+}
 __device__ __forceinline__ int gather(const MflArgs& a, int u) { return u >= 0 ? ld_label(a.R + u) : -1; }
 
 // LLP score val = k - gamma * (v - k) [P:119], double, no contraction (R11).
@@ -151,36 +193,16 @@ __device__ __forceinline__ unsigned ht_add(const Table& t, unsigned lab, unsigne
   }
 }
 
-// Insert one label per voting lane.  The warp's "hot" label -- lane 0's best
-// label so far (its own label on a fresh row) -- is merged with one ballot
-// first, so a collapsed neighbourhood (most neighbours share a community label
-// [P:130]) costs one shared atomic instead of 32 same-address atomics; the
-// other voting lanes insert individually (distinct-label regime, e.g. t = 1).
-// Returns the number of newly claimed slots in the warp when COUNT_NEW.
-template <int VAR, bool COUNT_NEW>
-__device__ __forceinline__ unsigned warp_insert(const MflArgs& a, const Table& t, unsigned max_probe, int lab,
-                                                bool vote, Best<VAR>& b, volatile int* overflow) {
-  const int lane = threadIdx.x & 31;
-  const int cand = b.have() ? (int)b.label() : lab;
-  const int hot = __shfl_sync(kFull, cand, 0);
-  const unsigned m = __ballot_sync(kFull, vote && lab == hot);
-  unsigned c = 0;
-  if (vote) c = (lab != hot) ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u);
-  bool fresh = false;
-  if (c) {
-    const unsigned cnt = ht_add(t, (unsigned)lab, c, max_probe, &fresh);
-    if (cnt == 0u) *overflow = 1;
-    else b.observe(cnt, (unsigned)lab, a);
-  }
-  return COUNT_NEW ? (unsigned)__popc(__ballot_sync(kFull, fresh)) : 0u;
-}
-
-// Batched form of warp_insert for N labels per lane: the hot-label ballots of
-// all N slots first, then the N home-slot probes as independent shared loads,
-// then the N atomics, so their latencies overlap (a lane's inserts no longer
-// wait on each other); only labels whose home slot holds another label fall
-// back to the probing loop.  Returns this lane's count of newly claimed slots.
-template <bool POW2>
+// Batched insert of N labels per lane (-1 = no vote).  First the warp's
+// "hot" label -- lane 0's best label so far, else its first label of this
+// batch -- is taken out: every lane counts its copies locally, one warp
+// reduction sums them and lane 0 adds the sum with a single shared atomic, so a
+// collapsed neighbourhood (most neighbours share a community label [P:130])
+// costs a few ALU ops per arc instead of same-address atomics.  The remaining
+// labels are inserted one by one: the N home-slot probes are issued as
+// independent shared loads, then the N atomics, so their latencies overlap;
+// only labels whose home slot holds another label fall back to the probing
+// loop.  Returns this lane's count of newly claimed slots.
 __device__ __forceinline__ unsigned ht_probe_from(const Table& t, unsigned lab, unsigned c, unsigned h,
                                                   unsigned max_probe, bool* fresh) {
   for (unsigned p = 1; p < max_probe; ++p) {
@@ -201,49 +223,65 @@ __device__ __forceinline__ unsigned ht_probe_from(const Table& t, unsigned lab, 
 
 template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
-                                                  const int (&lab)[N], Best<VAR>& b, volatile int* overflow) {
+                                                  const int (&labin)[N], Best<VAR>& b, volatile int* overflow) {
   const int lane = threadIdx.x & 31;
-  unsigned c[N];
-  const int cand0 = b.have() ? (int)b.label() : -2;
+  int lab[N];
 #pragma unroll
-  for (int j = 0; j < N; ++j) {
-    const bool vote = lab[j] >= 0;
-    const int hot = __shfl_sync(kFull, cand0 == -2 ? lab[j] : cand0, 0);
-    const unsigned m = __ballot_sync(kFull, vote && lab[j] == hot);
-    c[j] = vote ? (lab[j] != hot ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u)) : 0u;
+  for (int j = 0; j < N; ++j) lab[j] = labin[j];
+  unsigned nfresh = 0;
+  int cand = b.have() ? (int)b.label() : -1;
+#pragma unroll
+  for (int j = N - 1; j >= 0; --j)
+    if (cand < 0 && lab[j] >= 0) cand = lab[j];
+  const int hot = __shfl_sync(kFull, cand, 0);
+  if (hot >= 0) {  // warp-uniform
+    unsigned hc = 0;
+#pragma unroll
+    for (int j = 0; j < N; ++j)
+      if (lab[j] == hot) {
+        ++hc;
+        lab[j] = -1;
+      }
+    const unsigned tot = __reduce_add_sync(kFull, hc);
+    if (lane == 0 && tot) {
+      bool fr = false;
+      const unsigned cnt = ht_add(t, (unsigned)hot, tot, max_probe, &fr);
+      nfresh += fr ? 1u : 0u;
+      if (cnt == 0u) *overflow = 1;
+      else b.observe(cnt, (unsigned)hot, a);
+    }
   }
   unsigned h[N];
   unsigned long long e[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     h[j] = slot_hash((unsigned)lab[j], t.tsz);
-    e[j] = c[j] ? *((volatile unsigned long long*)(t.slots + h[j])) : 0ull;
+    e[j] = lab[j] >= 0 ? *((volatile unsigned long long*)(t.slots + h[j])) : 0ull;
   }
   unsigned cnt[N];
-  unsigned nfresh = 0;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     cnt[j] = 0u;
-    if (c[j]) {
+    if (lab[j] >= 0) {
       const unsigned l = (unsigned)lab[j];
       if ((unsigned)(e[j] >> 32) == l) {
-        cnt[j] = atomicAdd((unsigned*)(t.slots + h[j]), c[j]) + c[j];
+        cnt[j] = atomicAdd((unsigned*)(t.slots + h[j]), 1u) + 1u;
       } else if (e[j] == kEmpty) {
-        const unsigned long long prev = atomicCAS(t.slots + h[j], kEmpty, ((unsigned long long)l << 32) | c[j]);
+        const unsigned long long prev = atomicCAS(t.slots + h[j], kEmpty, ((unsigned long long)l << 32) | 1u);
         if (prev == kEmpty) {
-          cnt[j] = c[j];
+          cnt[j] = 1u;
           ++nfresh;
         } else if ((unsigned)(prev >> 32) == l) {
-          cnt[j] = atomicAdd((unsigned*)(t.slots + h[j]), c[j]) + c[j];
+          cnt[j] = atomicAdd((unsigned*)(t.slots + h[j]), 1u) + 1u;
         }
       }
     }
   }
 #pragma unroll
   for (int j = 0; j < N; ++j) {
-    if (c[j] && cnt[j] == 0u) {
+    if (lab[j] >= 0 && cnt[j] == 0u) {
       bool fr = false;
-      cnt[j] = ht_probe_from<true>(t, (unsigned)lab[j], c[j], h[j], max_probe, &fr);
+      cnt[j] = ht_probe_from(t, (unsigned)lab[j], 1u, h[j], max_probe, &fr);
       nfresh += fr ? 1u : 0u;
       if (cnt[j] == 0u) *overflow = 1;
     }
@@ -317,9 +355,12 @@ __device__ __forceinline__ void update_vertex(const MflArgs& a, int v, int deg, 
 // vmask = the deg lanes of a vertex; frequency of a lane's label = number of
 // vmask lanes with the same label (a shuffle loop of deg steps: match.any.sync
 // costs ~60 SM cycles per warp on distinct keys on sm_100, tools/ubench);
-// arg-max = shuffle tree toward the segment head, then lane j updates vertex
-// j.  Loads of the next chunk (arcs, vertex ids) are issued before the current
-// chunk is counted (software pipelining across the warp's chunks).
+// arg-max = two segmented warp reductions (redux.sync over the vmask: max
+// count, then min label among the maximal ones; LLP: a shuffle tree over the
+// double scores toward the segment head), then lane j updates vertex j.  Loads
+// of the next chunk are issued before the current chunk is counted (software
+// pipelining across the warp's chunks).  Chunk rows are consecutive internal
+// ids, so no vertex table is read.
 template <int VAR>
 __device__ __forceinline__ void update_vertex_pre(const MflArgs& a, int v, int deg, bool have, unsigned best, int r,
                                                   int2 so, Tally& ty) {
@@ -358,30 +399,33 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
     unsigned todo = __ballot_sync(kFull, act);
     if (!todo) continue;
     // issue the arc and vertex-id loads of chunk j
-    auto issue = [&](int j, int& u, int& v, int& total, int& nv) {
+    auto issue = [&](int j, int& u, int& v, int& total, int& d, unsigned& segs) {
       const unsigned long long st = __shfl_sync(kFull, mine.st, j);
       const int vbase = __shfl_sync(kFull, mine.vbase, j);
-      const unsigned segs = __shfl_sync(kFull, mine.segmask, j);
+      segs = __shfl_sync(kFull, mine.segmask, j);
       total = (int)(st >> 56);
-      nv = __popc(segs);
-      const int64_t start = (int64_t)(st & ((1ull << 56) - 1));
+      d = (int)((st >> 48) & 0xffull);
+      const int64_t start = (int64_t)(st & ((1ull << 48) - 1));
       u = lane < total ? ld_stream(a.col + start + lane) : -1;
-      v = lane < nv ? a.list[vbase + lane] : -1;
+      v = lane < __popc(segs) ? (int)(a.low_base + vbase + lane) : -1;
     };
     int j = __ffs(todo) - 1;
     todo &= todo - 1;
-    int u, v, total, nv;
-    issue(j, u, v, total, nv);
+    int u, v, total, d;
+    unsigned segs;
+    issue(j, u, v, total, d, segs);
     for (;;) {
       // prefetch the next chunk while this one is counted
-      int nu = -1, nvid = -1, ntotal = 0, nnv = 0;
+      int nu = -1, nvid = -1, ntotal = 0, nd = 1;
+      unsigned nsegs = 0u;
       const bool more = todo != 0;
       if (more) {
         const int nj = __ffs(todo) - 1;
         todo &= todo - 1;
-        issue(nj, nu, nvid, ntotal, nnv);
+        issue(nj, nu, nvid, ntotal, nd, nsegs);
       }
-      const int d = total / nv;  // every vertex of the chunk has degree d
+      // every vertex of the chunk has degree d; nv vertices, lanes [0, total)
+      const int nv = __popc(segs);
       int lab = gather(a, u);
       int r = 0;
       int2 so = make_int2(0, 0);
@@ -391,38 +435,49 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       }
       const bool vote = lane < total && lab >= 0;
       if (!vote) lab = -1;
-      const int sstart = (lane / d) * d, send = sstart + d;
+      // first lane of this lane's segment (vmask [P:230])
+      const int sstart = 31 - __clz(segs & ((2u << lane) - 1u));
       // label frequency inside the vertex's lanes [P:231-232]
       unsigned k = 0;
       for (int i = 0; i < d; ++i) {
         const int other = __shfl_sync(kFull, lab, (sstart + i) & 31);
         k += other == lab ? 1u : 0u;
       }
-      Best<VAR> b;
-      if (vote) b.observe(k, (unsigned)lab, a);
-      if (d > 1) {  // warp-uniform: segmented arg-max toward the segment head
+      const int head = (lane < nv ? lane * d : 0) & 31;  // lane jv takes segment jv
+      Best<VAR> h;
+      if (VAR == V_LLP || !GLP_LOW_REDUX) {
+        Best<VAR> b;
+        if (vote) b.observe(k, (unsigned)lab, a);
+        if (d > 1) {  // warp-uniform: segmented arg-max toward the segment head
+          const int send = sstart + d;
 #pragma unroll
-        for (int s2 = 1; s2 < 32; s2 <<= 1) {
-          const unsigned long long ok = __shfl_down_sync(kFull, b.key, s2);
-          const unsigned ol = VAR == V_LLP ? __shfl_down_sync(kFull, b.lab, s2) : 0u;
-          if (s2 < d && lane + s2 < send) b.merge(ok, ol);
+          for (int s2 = 1; s2 < 32; s2 <<= 1) {
+            const unsigned long long ok = __shfl_down_sync(kFull, b.key, s2);
+            const unsigned ol = __shfl_down_sync(kFull, b.lab, s2);
+            if (s2 < d && lane + s2 < send) b.merge(ok, ol);
+          }
         }
+        h.key = __shfl_sync(kFull, b.key, head);
+        h.lab = __shfl_sync(kFull, b.lab, head);
+      } else {
+        // segmented arg-max with two warp reductions over the segment's lanes
+        // (max count, then min label among the maximal ones: R4); lanes past
+        // the last segment form their own group
+        const unsigned segm = lane < total ? (d >= 32 ? kFull : ((1u << d) - 1u) << sstart)
+                                           : (kFull << (total & 31));
+        const unsigned kmax = __reduce_max_sync(segm, vote ? k : 0u);
+        const unsigned lmin = __reduce_min_sync(segm, (vote && k == kmax) ? (unsigned)lab : kNoLabel);
+        const unsigned hk = __shfl_sync(kFull, kmax, head);
+        const unsigned hl = __shfl_sync(kFull, lmin, head);
+        h.key = hk ? (((unsigned long long)hk << 32) | (unsigned long long)(~hl)) : 0ull;
       }
-      // lane jv takes the result of segment jv (head lane jv*d)
-      const int head = (lane < nv ? lane * d : 0) & 31;
-      const unsigned long long bk = __shfl_sync(kFull, b.key, head);
-      const unsigned bl = VAR == V_LLP ? __shfl_sync(kFull, b.lab, head) : 0u;
-      if (lane < nv) {
-        Best<VAR> h;
-        h.key = bk;
-        h.lab = bl;
-        update_vertex_pre<VAR>(a, v, d, h.have(), h.label(), r, so, ty);
-      }
+      if (lane < nv) update_vertex_pre<VAR>(a, v, d, h.have(), h.label(), r, so, ty);
       if (!more) break;
       u = nu;
       v = nvid;
       total = ntotal;
-      nv = nnv;
+      d = nd;
+      segs = nsegs;
     }
   }
   tally_flush(ty, a.cnt);
@@ -472,20 +527,35 @@ __device__ __forceinline__ bool warp_quads_increasing(const int (&x)[4], int bas
 // ---------------------------------------------------------------------------
 // mfl_warp: one warp per row of class W (few distinct labels): per-warp shared
 // table of pow2 >= 2*pred slots (<= 512), two 128-bit loads per lane per
-// round (256 arcs in flight per warp), no block barriers.  Rows whose labels
-// overflow the table are re-queued to the block kernel M.
+// round (256 arcs per warp), no block barriers.  Rows whose labels overflow the
+// table are re-queued to the block kernel M.
+//   * 32 rows per warp at a time: the class / frontier test of the batch is
+//     lane-parallel; rows are degree-sorted, so a warp's batch is strided
+//     across the list (lane l of warp w takes row base + l * nwarps + w);
+//   * software pipeline: the arcs of the next round -- of this row, or the
+//     first round of the next selected row -- are loaded while the current
+//     round is gathered and counted;
+//   * lane j keeps the result of batch row j, and the batch's vertices are
+//     updated lane-parallel at the end.
+__device__ __forceinline__ void load_round(const int32_t* col, int64_t start, int off, int d, int4& u0, int4& u1) {
+  const int lane = threadIdx.x & 31;
+  u0 = make_int4(-1, -1, -1, -1);
+  u1 = u0;
+  if (off + 4 * lane < d) u0 = ld_stream4(col + start + off + 4 * lane);
+  if (off + 128 + 4 * lane < d) u1 = ld_stream4(col + start + off + 128 + 4 * lane);
+}
+
 template <int VAR>
-__global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
+#ifndef GLP_W_MINB
+#define GLP_W_MINB 3
+#endif
+__global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
   __shared__ __align__(16) unsigned long long tabs[kWBlock / 32][kWSlots];
   __shared__ int s_over[kWBlock / 32];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
   Tally ty;
-  // 32 rows per warp at a time: the class / frontier test of the batch is
-  // lane-parallel, then the warp processes the selected rows one by one
-  // rows are degree-sorted, so a warp's batch is strided across the list
-  // (lane l of warp w takes row base + l * nwarps + w) to balance long rows
   for (int base = 0; base < a.n_items; base += nwarps * 32) {
     const int il = base + lane * nwarps + gw;
     BinItem mine;
@@ -503,81 +573,116 @@ __global__ void __launch_bounds__(kWBlock) mfl_warp(MflArgs a) {
       }
     }
     unsigned todo = __ballot_sync(kFull, ok);
-    while (todo) {
-    const int jl = __ffs(todo) - 1;
+    if (!todo) continue;
+    // per-lane result of batch row `lane`
+    bool rdone = false;
+    unsigned long long rkey = 0ull;
+    unsigned rlab = kNoLabel, rpred = 0u;
+    int jl = __ffs(todo) - 1;
     todo &= todo - 1;
-    const int i = base + jl * nwarps + gw;
-    BinItem it;
-    it.start = __shfl_sync(kFull, mine.start, jl);
-    it.v = __shfl_sync(kFull, mine.v, jl);
-    it.d = __shfl_sync(kFull, mine.d, jl);
-    const unsigned pred = __shfl_sync(kFull, mpred, jl);
-    const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
-    const Table tab{tabs[wid], tsz};
-    tab.clear(lane, 32);
-    if (lane == 0) s_over[wid] = 0;
-    __syncwarp();
-    Best<VAR> b;
-    unsigned fresh = 0;
-    bool over = false;
-    bool mono = VAR != V_SEEDED && !(pred & kMonoTried) && pred >= (unsigned)it.d;  // sorted-row candidate
-    const bool tried = mono;
-    int prev = -1;
-    for (int base = 0; base < it.d && !over; base += 256) {
-      int4 u0 = make_int4(-1, -1, -1, -1), u1 = u0;
-      if (base + 4 * lane < it.d) u0 = ld_stream4(a.col + it.start + base + 4 * lane);
-      if (base + 128 + 4 * lane < it.d) u1 = ld_stream4(a.col + it.start + base + 128 + 4 * lane);
-      int l[8];
-      l[0] = gather(a, u0.x); l[1] = gather(a, u0.y); l[2] = gather(a, u0.z); l[3] = gather(a, u0.w);
-      l[4] = gather(a, u1.x); l[5] = gather(a, u1.y); l[6] = gather(a, u1.z); l[7] = gather(a, u1.w);
-      if (mono) {
-        const int q0[4] = {l[0], l[1], l[2], l[3]}, q1[4] = {l[4], l[5], l[6], l[7]};
-        int mid = -1, end = -1;
-        bool ok = warp_quads_increasing(q0, base, it.d, prev, &mid);
-        ok = ok && warp_quads_increasing(q1, base + 128, it.d, mid, &end);
-        if (ok) {  // every label of this round occurs once in the row so far
+    int64_t start = __shfl_sync(kFull, mine.start, jl);
+    int d = __shfl_sync(kFull, mine.d, jl);
+    unsigned pred = __shfl_sync(kFull, mpred, jl);
+    int4 x0, x1;
+    load_round(a.col, start, 0, d, x0, x1);
+    for (;;) {
+      // the next selected row of the batch (its first round is prefetched)
+      const int njl = todo ? __ffs(todo) - 1 : -1;
+      if (todo) todo &= todo - 1;
+      int64_t nstart = 0;
+      int nd = 0;
+      unsigned npred = 0u;
+      if (njl >= 0) {
+        nstart = __shfl_sync(kFull, mine.start, njl);
+        nd = __shfl_sync(kFull, mine.d, njl);
+        npred = __shfl_sync(kFull, mpred, njl);
+      }
+      const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
+      const Table tab{tabs[wid], tsz};
+      tab.clear(lane, 32);
+      if (lane == 0) s_over[wid] = 0;
+      __syncwarp();
+      Best<VAR> b;
+      unsigned fresh = 0;
+      bool over = false;
+      bool mono = VAR != V_SEEDED && !(pred & kMonoTried) && pred >= (unsigned)d;  // sorted-row candidate
+      const bool tried = mono;
+      int prev = -1;
+      bool next_loaded = false;  // x0/x1 hold the next row's first round
+      for (int off = 0; off < d && !over; off += 256) {
+        int4 p0, p1;
+        if (off + 256 < d) {
+          load_round(a.col, start, off + 256, d, p0, p1);
+        } else {
+          load_round(a.col, nstart, 0, nd, p0, p1);  // nd == 0: no loads
+          next_loaded = true;
+        }
+        int l[8];
+        l[0] = gather(a, x0.x); l[1] = gather(a, x0.y); l[2] = gather(a, x0.z); l[3] = gather(a, x0.w);
+        l[4] = gather(a, x1.x); l[5] = gather(a, x1.y); l[6] = gather(a, x1.z); l[7] = gather(a, x1.w);
+        x0 = p0;
+        x1 = p1;
+        if (mono) {
+          const int q0[4] = {l[0], l[1], l[2], l[3]}, q1[4] = {l[4], l[5], l[6], l[7]};
+          int mid = -1, end = -1;
+          bool okm = warp_quads_increasing(q0, off, d, prev, &mid);
+          okm = okm && warp_quads_increasing(q1, off + 128, d, mid, &end);
+          if (okm) {  // every label of this round occurs once in the row so far
 #pragma unroll
-          for (int j = 0; j < 8; ++j)
-            if (l[j] >= 0) { b.observe(1u, (unsigned)l[j], a); ++fresh; }
-          prev = end;
-          continue;
+            for (int j = 0; j < 8; ++j)
+              if (l[j] >= 0) { b.observe(1u, (unsigned)l[j], a); ++fresh; }
+            prev = end;
+            continue;
+          }
+          // not sorted: count this row with the table, re-inserting the rounds
+          // already observed (their count-1 observations stay valid lower bounds)
+          mono = false;
+          fresh = 0;
+          for (int b2 = 0; b2 < off; b2 += 256) {
+            int4 v0, v1;
+            load_round(a.col, start, b2, d, v0, v1);
+            const int m8[8] = {gather(a, v0.x), gather(a, v0.y), gather(a, v0.z), gather(a, v0.w),
+                               gather(a, v1.x), gather(a, v1.y), gather(a, v1.z), gather(a, v1.w)};
+            fresh += warp_insert_n<VAR, 8>(a, tab, tsz, m8, b, &s_over[wid]);
+          }
         }
-        // not sorted: count this row with the table, re-inserting the rounds
-        // already observed (their count-1 observations stay valid lower bounds)
-        mono = false;
-        fresh = 0;
-        for (int b2 = 0; b2 < base; b2 += 256) {
-          int4 v0 = make_int4(-1, -1, -1, -1), v1 = v0;
-          if (b2 + 4 * lane < it.d) v0 = ld_stream4(a.col + it.start + b2 + 4 * lane);
-          if (b2 + 128 + 4 * lane < it.d) v1 = ld_stream4(a.col + it.start + b2 + 128 + 4 * lane);
-          const int m8[8] = {gather(a, v0.x), gather(a, v0.y), gather(a, v0.z), gather(a, v0.w),
-                             gather(a, v1.x), gather(a, v1.y), gather(a, v1.z), gather(a, v1.w)};
-          fresh += warp_insert_n<VAR, 8>(a, tab, tsz, m8, b, &s_over[wid]);
+        if (d - off > 128) {  // warp-uniform
+          fresh += warp_insert_n<VAR, 8>(a, tab, tsz, l, b, &s_over[wid]);
+        } else {
+          const int l4[4] = {l[0], l[1], l[2], l[3]};
+          fresh += warp_insert_n<VAR, 4>(a, tab, tsz, l4, b, &s_over[wid]);
         }
+        __syncwarp();
+        over = s_over[wid] != 0;
       }
-      if (it.d - base > 128) {  // warp-uniform
-        fresh += warp_insert_n<VAR, 8>(a, tab, tsz, l, b, &s_over[wid]);
+      if (over) {
+        if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = base + jl * nwarps + gw;
+        if (!next_loaded) load_round(a.col, nstart, 0, nd, x0, x1);
       } else {
-        const int l4[4] = {l[0], l[1], l[2], l[3]};
-        fresh += warp_insert_n<VAR, 4>(a, tab, tsz, l4, b, &s_over[wid]);
+        b.warp_reduce();
+        fresh = __reduce_add_sync(kFull, fresh);
+        if (lane == jl) {
+          rdone = true;
+          rkey = b.key;
+          rlab = b.lab;
+          // a row that just took the sorted fast path is not retried next time
+          rpred = max(fresh, 1u) | (tried && mono ? kMonoTried : 0u);
+        }
       }
       __syncwarp();
-      over = s_over[wid] != 0;
+      if (njl < 0) break;
+      jl = njl;
+      start = nstart;
+      d = nd;
+      pred = npred;
     }
-    if (over) {
-      if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = i;
-      __syncwarp();
-      continue;
+    if (rdone) {
+      Best<VAR> r;
+      r.key = rkey;
+      r.lab = rlab;
+      a.pred_next[il] = rpred;
+      update_vertex<VAR>(a, mine.v, mine.d, r.have(), r.label(), ty);
     }
-    b.warp_reduce();
-    fresh = __reduce_add_sync(kFull, fresh);
-    if (lane == 0) {
-      // a row that just took the sorted fast path is not retried next time
-      a.pred_next[i] = max(fresh, 1u) | (tried && mono ? kMonoTried : 0u);
-      update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
-    }
-    __syncwarp();
-    }  // todo
   }
   tally_flush(ty, a.cnt);
 }
@@ -591,95 +696,104 @@ __device__ __forceinline__ unsigned label_part(unsigned lab, unsigned nparts) {
   return __umulhi(lab * 0x85EBCA77u + 0x165667B1u, nparts);
 }
 
-template <int VAR, int BLOCK, int UNROLL, bool COUNT_NEW>
-__device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int d, const Table& tab,
-                                            unsigned max_probe, unsigned part, unsigned nparts,
-                                            const int32_t* stage_in, int32_t* stage_out,
-                                            volatile int* overflow, int* distinct, Best<VAR>& b) {
-  unsigned fresh = 0;
-  for (int base = 0; base < d; base += BLOCK * 4 * UNROLL) {
-    int lab[4 * UNROLL];
-    if (stage_in != nullptr) {
-      // labels of this row already gathered by an earlier pass (coalesced)
+// Round `base` of a row for the block kernels: UNROLL 128-bit loads per thread.
+template <int BLOCK, int UNROLL>
+__device__ __forceinline__ void block_load_round(const int32_t* col, int64_t start, int d, int base,
+                                                 int4 (&u)[UNROLL]) {
 #pragma unroll
-      for (int j = 0; j < UNROLL; ++j) {
-        const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
-        const int4 x = idx < d ? __ldcg((const int4*)(stage_in + idx)) : make_int4(-1, -1, -1, -1);
-        lab[4 * j + 0] = x.x; lab[4 * j + 1] = x.y; lab[4 * j + 2] = x.z; lab[4 * j + 3] = x.w;
-      }
-    } else {
-      int4 u[UNROLL];
-#pragma unroll
-      for (int j = 0; j < UNROLL; ++j) {
-        const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
-        u[j] = idx < d ? ld_stream4(a.col + start + idx) : make_int4(-1, -1, -1, -1);
-      }
-#pragma unroll
-      for (int j = 0; j < UNROLL; ++j) {
-        lab[4 * j + 0] = gather(a, u[j].x);
-        lab[4 * j + 1] = gather(a, u[j].y);
-        lab[4 * j + 2] = gather(a, u[j].z);
-        lab[4 * j + 3] = gather(a, u[j].w);
-        const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
-        if (stage_out != nullptr && idx < d)
-          __stcg((int4*)(stage_out + idx), make_int4(lab[4 * j], lab[4 * j + 1], lab[4 * j + 2], lab[4 * j + 3]));
-      }
-    }
-    if (nparts > 1u) {
-#pragma unroll
-      for (int j = 0; j < 4 * UNROLL; ++j)
-        if (lab[j] >= 0 && label_part((unsigned)lab[j], nparts) != part) lab[j] = -1;
-    }
-    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow);
-    if (__any_sync(kFull, *overflow != 0)) break;  // warp-uniform exit
-  }
-  if (COUNT_NEW) {
-    fresh = __reduce_add_sync(kFull, fresh);
-    if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
+  for (int j = 0; j < UNROLL; ++j) {
+    const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
+    u[j] = idx < d ? ld_stream4(col + start + idx) : make_int4(-1, -1, -1, -1);
   }
 }
 
-// Block-level sorted-row fast path (see warp_quads_increasing): one 128-bit
-// load per thread per 4*BLOCK arcs; warps check their own 128-arc quad rows,
-// thread 0 chains the warp boundaries.  Returns the block-uniform verdict; on
+// `u` holds round 0 of the row (loaded ahead by the caller); each round loads
+// the next one before gathering its own labels.
+template <int VAR, int BLOCK, int UNROLL>
+__device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int d, const Table& tab,
+                                            unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
+                                            volatile int* overflow, int* distinct, Best<VAR>& b) {
+  constexpr int STEP = BLOCK * 4 * UNROLL;
+  unsigned fresh = 0;
+  for (int base = 0; base < d; base += STEP) {
+    int4 un[UNROLL];
+    block_load_round<BLOCK, UNROLL>(a.col, start, d, base + STEP, un);
+    int lab[4 * UNROLL];
+#pragma unroll
+    for (int j = 0; j < UNROLL; ++j) {
+      lab[4 * j + 0] = gather(a, u[j].x);
+      lab[4 * j + 1] = gather(a, u[j].y);
+      lab[4 * j + 2] = gather(a, u[j].z);
+      lab[4 * j + 3] = gather(a, u[j].w);
+      const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
+      if (stage_out != nullptr && idx < d)
+        __stcg((int4*)(stage_out + idx), make_int4(lab[4 * j], lab[4 * j + 1], lab[4 * j + 2], lab[4 * j + 3]));
+    }
+#pragma unroll
+    for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
+    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow);
+    if (__any_sync(kFull, *overflow != 0)) break;  // warp-uniform exit
+  }
+  fresh = __reduce_add_sync(kFull, fresh);
+  if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
+}
+
+// Block-level sorted-row fast path (see warp_quads_increasing): rounds of
+// UNROLL 128-bit loads per thread (the block_load_round layout; `u` holds round
+// 0, loaded ahead by the caller, and each round loads the next before
+// gathering).  A round is a sequence of 128-arc quad rows q = j*NW + warp; each
+// warp checks its own, then warp 0 checks the NW*UNROLL boundaries between
+// consecutive quad rows lane-parallel.  Returns the block-uniform verdict; on
 // success every label has been observed with count 1 and *fresh counts them.
-template <int VAR, int BLOCK>
-__device__ __forceinline__ bool block_mono(const MflArgs& a, int64_t start, int d, Best<VAR>& b, unsigned* fresh) {
-  constexpr int NW = BLOCK / 32;
-  __shared__ int s_first[NW], s_last[NW], s_ok, s_prev;
+template <int VAR, int BLOCK, int UNROLL>
+__device__ __forceinline__ bool block_mono(const MflArgs& a, int64_t start, int d, int4 (&u)[UNROLL], Best<VAR>& b,
+                                           unsigned* fresh) {
+  constexpr int NW = BLOCK / 32, NQ = NW * UNROLL, STEP = 4 * BLOCK * UNROLL;
+  __shared__ int s_first[NQ], s_last[NQ], s_ok, s_prev;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   int prev_round = -1;
-  for (int base = 0; base < d; base += 4 * BLOCK) {
-    const int wb = base + 128 * wid;
-    int x[4] = {-1, -1, -1, -1};
-    if (wb + 4 * lane < d) {
-      const int4 u = ld_stream4(a.col + start + wb + 4 * lane);
-      x[0] = gather(a, u.x); x[1] = gather(a, u.y); x[2] = gather(a, u.z); x[3] = gather(a, u.w);
+  for (int base = 0; base < d; base += STEP) {
+    int4 un[UNROLL];
+    block_load_round<BLOCK, UNROLL>(a.col, start, d, base + STEP, un);
+    int x[UNROLL][4];
+#pragma unroll
+    for (int j = 0; j < UNROLL; ++j) {
+      x[j][0] = gather(a, u[j].x); x[j][1] = gather(a, u[j].y); x[j][2] = gather(a, u[j].z);
+      x[j][3] = gather(a, u[j].w);
+      u[j] = un[j];
     }
-    int lastw = -1;
-    const bool okw = warp_quads_increasing(x, wb, d, INT_MIN, &lastw);
-    if (lane == 0) {
-      s_first[wid] = x[0];
-      s_last[wid] = lastw;
+    bool okw = true;
+#pragma unroll
+    for (int j = 0; j < UNROLL; ++j) {
+      const int wb = base + j * 4 * BLOCK + 128 * wid;
+      int lastw = -1;
+      okw &= warp_quads_increasing(x[j], wb, d, INT_MIN, &lastw);
+      if (lane == 0) {
+        s_first[j * NW + wid] = x[j][0];
+        s_last[j * NW + wid] = lastw;
+      }
     }
     const int ok_all = __syncthreads_and(okw ? 1 : 0);
-    if (threadIdx.x == 0) {
+    if (wid == 0) {
+      const int nq = min(NQ, (d - base + 127) / 128);  // quad rows holding arcs
       bool ok = ok_all != 0;
-      int p = prev_round;
-      for (int w = 0; w < NW; ++w)
-        if (base + 128 * w < d) {
-          ok = ok && p < s_first[w];
-          p = s_last[w];
-        }
-      s_ok = ok ? 1 : 0;
-      s_prev = p;
+      for (int q = lane; q < nq; q += 32) ok &= (q == 0 ? prev_round : s_last[q - 1]) < s_first[q];
+      ok = __all_sync(kFull, ok);
+      if (lane == 0) {
+        s_ok = ok ? 1 : 0;
+        s_prev = s_last[nq - 1];
+      }
     }
     __syncthreads();
     if (!s_ok) return false;
     prev_round = s_prev;
 #pragma unroll
-    for (int k = 0; k < 4; ++k)
-      if (wb + 4 * lane + k < d) { b.observe(1u, (unsigned)x[k], a); ++*fresh; }
+    for (int j = 0; j < UNROLL; ++j) {
+      const int wb = base + j * 4 * BLOCK + 128 * wid;
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        if (wb + 4 * lane + k < d) { b.observe(1u, (unsigned)x[j][k], a); ++*fresh; }
+    }
   }
   return true;
 }
@@ -737,7 +851,10 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
 //     staged row costs less than clearing and probing a per-row global table.
 // Both record the row's exact distinct-label count as the next `pred`.
 template <int VAR, int BLOCK, int SLOTS, bool PART, int UNROLL, int CLS>
-__global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
+#ifndef GLP_M_MINB
+#define GLP_M_MINB 1
+#endif
+__global__ void __launch_bounds__(BLOCK, PART ? 1 : GLP_M_MINB) mfl_block(MflArgs a) {
   extern __shared__ __align__(16) unsigned long long smem_tab[];  // SLOTS
   __shared__ int s_over, s_distinct;
   __shared__ int s_hist[PART ? 256 : 1], s_cur[PART ? 256 : 1];
@@ -783,9 +900,26 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
     }
     __syncthreads();
     const int nsel = s_nsel;
+    // round 0 of the next selected row is loaded while the current row is
+    // counted (cross-row software pipeline)
+    BinItem nit;
+    nit.start = 0; nit.v = 0; nit.d = 0;
+    int4 pre[UNROLL];
+    if (nsel > 0) nit = a.items[s_sel[0]];
+    if (GLP_XROW) block_load_round<BLOCK, UNROLL>(a.col, nit.start, nit.d, 0, pre);
     for (int q = 0; q < nsel; ++q) {
     const int i = s_sel[q];
-    const BinItem it = a.items[i];
+    const BinItem it = nit;
+    int4 cur[UNROLL];
+#pragma unroll
+    for (int j = 0; j < UNROLL; ++j) cur[j] = pre[j];
+    nit.d = 0;
+    if (q + 1 < nsel) nit = a.items[s_sel[q + 1]];
+    if (GLP_XROW) {
+      block_load_round<BLOCK, UNROLL>(a.col, nit.start, nit.d, 0, pre);
+    } else {
+      block_load_round<BLOCK, UNROLL>(a.col, it.start, it.d, 0, cur);
+    }
     const unsigned praw = a.pred[i];
     const bool tried_before = (praw & kMonoTried) != 0;
     const unsigned pred = a.pred_cap ? min(praw & kPredMask, a.pred_cap) : (praw & kPredMask);
@@ -796,18 +930,22 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
     if (!a.mode && VAR != V_SEEDED && !tried_before && pred >= (unsigned)d) {
       __syncthreads();
       unsigned fr = 0;
-      mono_done = block_mono<VAR, BLOCK>(a, it.start, d, b, &fr);
+      mono_done = block_mono<VAR, BLOCK, UNROLL>(a, it.start, d, cur, b, &fr);
       if (mono_done) {
         fr = __reduce_add_sync(kFull, fr);
         if ((threadIdx.x & 31) == 0 && fr) atomicAdd(&s_distinct, (int)fr);
         __syncthreads();
       } else {
         b = Best<VAR>();
+        block_load_round<BLOCK, UNROLL>(a.col, it.start, d, 0, cur);  // table path restarts the row
       }
     }
     if (!mono_done) {
-    // a re-queued row overflowed a smaller table: its pred is stale
-    const unsigned est = a.mode ? (unsigned)d : max(pred, 1u);
+    // a re-queued row overflowed a smaller table: its pred is stale.  A row
+    // whose last count took the sorted fast path (all labels distinct then)
+    // tries one table-sized pass first: labels collapse after t = 1 [P:130]
+    const unsigned est = a.mode ? (unsigned)d : (GLP_L_OPT && tried_before && PART) ? min(max(pred, 1u), (unsigned)SLOTS / 2)
+                                                                         : max(pred, 1u);
     unsigned nparts = PART ? max(1u, (min(est, (unsigned)d) + SLOTS / 2 - 1) / (SLOTS / 2)) : 1u;
     bool staged = false;  // stageA holds the row's gathered labels
     bool over = false;
@@ -819,8 +957,8 @@ __global__ void __launch_bounds__(BLOCK, 1) mfl_block(MflArgs a) {
       tab.clear(threadIdx.x, BLOCK);
       __syncthreads();
       const bool may_over = PART && 2u * (unsigned)d > (unsigned)SLOTS;
-      block_count<VAR, BLOCK, UNROLL, true>(a, it.start, d, tab, may_over ? kLProbe : tsz, 0u, 1u, nullptr,
-                                            may_over ? stageA : nullptr, &s_over, &s_distinct, b);
+      block_count<VAR, BLOCK, UNROLL>(a, it.start, d, tab, may_over ? kLProbe : tsz, cur,
+                                      may_over ? stageA : nullptr, &s_over, &s_distinct, b);
       __syncthreads();
       over = s_over != 0;
       __syncthreads();
