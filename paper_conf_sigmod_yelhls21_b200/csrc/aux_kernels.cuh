@@ -114,12 +114,13 @@ __global__ void k_relayout(const int64_t* __restrict__ off, const int32_t* __res
 
 // Predicted distinct labels of each row at t = 1 (performance hint only).
 __global__ void k_init_pred(const BinItem* __restrict__ rows, int32_t n_rows, unsigned* __restrict__ pred0,
-                            unsigned* __restrict__ pred1, unsigned seed_cap) {
+                            unsigned* __restrict__ pred1, unsigned* __restrict__ pred2, unsigned seed_cap) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_rows; i += (int64_t)gridDim.x * blockDim.x) {
     const unsigned d = (unsigned)rows[i].d;
     const unsigned p = seed_cap ? max(1u, min(d, seed_cap)) : d;
     pred0[i] = p;
     pred1[i] = p;
+    pred2[i] = p;
   }
 }
 

@@ -244,8 +244,7 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     g->n_gt2048 += it.d > 2048;
     g->n_ge8k += it.d >= 8192;
   }
-  g->pred[0] = dalloc<unsigned>(g, std::max<int64_t>(n_rows, 1));
-  g->pred[1] = dalloc<unsigned>(g, std::max<int64_t>(n_rows, 1));
+  for (int k = 0; k < 3; ++k) g->pred[k] = dalloc<unsigned>(g, std::max<int64_t>(n_rows, 1));
   g->redo_m = dalloc<int32_t>(g, std::max<int64_t>(n_rows, 1));
   g->redo_l = dalloc<int32_t>(g, std::max<int64_t>(n_rows, 1));
   g->d_sched = dalloc<Sched>(g, 1);
@@ -452,7 +451,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->grid_aux = sms * 8;
     if (g->n_rows > 0) {
       // L staging: two row-sized buffers per resident L block
-      g->stage_stride = (g->max_deg + 3) & ~(int64_t)3;
+      // L never takes giant rows (deg > kGiantMin)
+      g->stage_stride = (std::min<int64_t>(g->max_deg, kGiantMin) + 3) & ~(int64_t)3;
       g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 2 * g->grid_l);
     }
     CK(cudaStreamSynchronize(g->stream));
@@ -506,7 +506,8 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   int n = 0;
   const size_t ms_ = kMSlots * 8, ls_ = kLSlots * 8;
   MflArgs r = a;
-  r.items = g->rows; r.big_prefix = g->n_ge8k; r.pred = g->pred[g->pb]; r.pred_next = g->pred[1 - g->pb];
+  r.items = g->rows; r.big_prefix = g->n_ge8k; r.pred = g->pred[g->pb]; r.pred_prev = g->pred[(g->pb + 2) % 3];
+  r.pred_next = g->pred[(g->pb + 1) % 3];
   r.stage = g->stage; r.stage_stride = g->stage_stride;
   if (g->n_giant) {  // giant rows: all blocks count segments into per-row global tables
     MflArgs b = r;
@@ -555,7 +556,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     MflArgs b = r;
     b.mode = 1; b.cnt = c + 2; b.redo_in = g->redo_m; b.redo_in_n = &sc->n_redo_m; b.work = &sc->work_mr;
     b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
-    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<g->sms, kMBlock, ms_, g->stream>>>(b); });
+    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<g->grid_m, kMBlock, ms_, g->stream>>>(b); });
     MflArgs q = r;
     q.mode = 1; q.cnt = c + 3; q.redo_in = g->redo_l; q.redo_in_n = &sc->n_redo_l; q.work = &sc->work_lr;
     timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<g->grid_l, kLBlock, ls_, g->stream>>>(q); });
@@ -620,7 +621,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     // predicted distinct labels per row for t = 1: deg (all labels distinct)
     // for CLASSIC/LLP, at most the number of seeds for SEEDED
     g->pb = 0;
-    k_init_pred<<<ga, 256, 0, s>>>(g->rows, g->n_rows, g->pred[0], g->pred[1],
+    k_init_pred<<<ga, 256, 0, s>>>(g->rows, g->n_rows, g->pred[0], g->pred[1], g->pred[2],
                                    variant == GLP_VARIANT_SEEDED ? (unsigned)std::min<int64_t>(n_seeds, 1 << 30) : 0u);
     CK(cudaGetLastError());
     g->init_launches += 1;
@@ -655,13 +656,15 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   // algorithmic bytes to the MFL kernels (SURVEY §8(d) model)
   auto drain = [&](bool with_counters) {
     const int cur_t = g->cur_t;
+    bool credited[kNumKernelNames] = {false};  // M and L launch twice (static + redo): credit once
     for (auto& pe : pend) {
       float kms = 0;
       CK(cudaEventElapsedTime(&kms, pe.a, pe.b));
       KStat& ks = g->kstats[pe.kid];
       ks.launches += 1;
       ks.ms += kms;
-      if (with_counters && (pe.kid < 4 || pe.kid == 7) && pe.t == cur_t) {
+      if (with_counters && (pe.kid < 4 || pe.kid == 7) && pe.t == cur_t && !credited[pe.kid]) {
+        credited[pe.kid] = true;
         const Counters& c = g->h_cnt[pe.kid == 7 ? 4 : pe.kid];
         ks.arcs += (double)c.arcs;
         // 4 B/arc (col_idx) + 8 B/active vertex (row offsets) + 4 B/changed label
@@ -761,7 +764,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       });
     }
     g->iter_stats.push_back(st);
-    g->pb = 1 - g->pb;
+    g->pb = (g->pb + 1) % 3;
     rb = 1 - rb;
     fb = nf;
     dense = next_dense;

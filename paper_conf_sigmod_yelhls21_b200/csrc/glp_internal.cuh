@@ -34,8 +34,9 @@ constexpr int kLowBlock = 256;
 // communities form [P:130], so most rows migrate to the warp path:
 //   W  pred <= 256,  deg <= 4096  : one warp per row, 512-slot table per warp
 //   M  pred <= 2048, deg <= 16384 : one 128-thread block per row, 4096 slots
-//   L  otherwise                  : one 1024-thread block per row, 16384
-//                                   slots, hash-partitioned passes
+//   L  otherwise                  : one 512-thread block per row (two per
+//                                   SM), 8192 slots, hash-partitioned passes
+// Sorted-row candidates (row_class `mono`) go to W whatever their size.
 // A row whose labels overflow its table is re-queued to the next class in the
 // same iteration (exact recount), so `pred` only steers performance.
 constexpr unsigned kWPred = 256, kMPred = 2048;
@@ -45,8 +46,14 @@ constexpr int kWSlots = 512;
 constexpr int kMBlock = 128;
 constexpr int kMSlots = 4096;
 constexpr int kMUnroll = 2;
-constexpr int kLBlock = 1024;
-constexpr int kLSlots = 16384;
+#ifndef GLP_LBLOCK
+#define GLP_LBLOCK 512
+#endif
+#ifndef GLP_LSLOTS
+#define GLP_LSLOTS 8192
+#endif
+constexpr int kLBlock = GLP_LBLOCK;
+constexpr int kLSlots = GLP_LSLOTS;
 constexpr int kLUnroll = 2;
 constexpr int kLProbe = 32;  // probe limit before declaring a partition overflowed
 // Giant rows (deg > kGiantMin) are split into segments of kGiantSeg arcs that
@@ -63,8 +70,12 @@ enum RowClass { CLS_W = 0, CLS_M = 1, CLS_L = 2, CLS_G = 3 };
 // pred word: low 31 bits = predicted distinct labels; bit 31 = the row took
 // the sorted-row fast path last time (do not retry it)
 constexpr unsigned kPredMask = 0x7fffffffu, kMonoTried = 0x80000000u;
-__host__ __device__ __forceinline__ int row_class(unsigned pred, int d) {
+// A sorted-row candidate (`mono`: its labels were all distinct last time and
+// it has not tried the fast path yet, e.g. every row at t = 1) needs no table:
+// it goes to the barrier-free warp kernel whatever its size.
+__host__ __device__ __forceinline__ int row_class(unsigned pred, int d, bool mono) {
   if (d > kGiantMin) return CLS_G;
+  if (mono) return CLS_W;
   if (pred <= kWPred && d <= kWMaxDeg) return CLS_W;
   if (pred <= kMPred && d <= kMMaxDeg) return CLS_M;
   return CLS_L;
@@ -131,6 +142,7 @@ struct MflArgs {
   int32_t n_items;                      // prefix of items this launch scans
   int32_t big_prefix;                   // rows fetched one per ticket (longest rows)
   const unsigned* __restrict__ pred;    // per row: predicted distinct labels (this iteration)
+  const unsigned* __restrict__ pred_prev;  // per row: distinct labels at t-2 (extrapolation)
   unsigned* __restrict__ pred_next;     // per row: distinct labels counted now (next iteration)
   unsigned pred_cap;                    // testing: clamp predictions (0 = off)
   int32_t mode;                         // 0: scan items by class, 1: redo list
@@ -210,7 +222,7 @@ struct glp_graph {
   unsigned* gdistinct = nullptr;
   int32_t* gseg_first = nullptr;                     // [n_giant+1]
   unsigned long long gepoch = 0;                     // last giant-table epoch used
-  unsigned* pred[2] = {nullptr, nullptr};            // [n_rows], double-buffered per iteration
+  unsigned* pred[3] = {nullptr, nullptr, nullptr};   // [n_rows], distinct counts of t-1, t-2 and t
   int pb = 0;                                        // pred[pb] is read this iteration
   int32_t* redo_m = nullptr;                         // [n_rows]
   int32_t* redo_l = nullptr;                         // [n_rows]

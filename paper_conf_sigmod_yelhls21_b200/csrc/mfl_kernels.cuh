@@ -58,13 +58,22 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #endif
 // kernel A/B switches (tools/build_variants.py)
 #ifndef GLP_LOW_REDUX
-#define GLP_LOW_REDUX 1
+#define GLP_LOW_REDUX 0
 #endif
 #ifndef GLP_L_OPT
-#define GLP_L_OPT 1
+#define GLP_L_OPT 0
 #endif
 #ifndef GLP_XROW
-#define GLP_XROW 1
+#define GLP_XROW 0
+#endif
+#ifndef GLP_L_IPF
+#define GLP_L_IPF 0
+#endif
+#ifndef GLP_L_EST
+#define GLP_L_EST 40
+#endif
+#ifndef GLP_W_LOAD
+#define GLP_W_LOAD 2
 #endif
 __device__ __forceinline__ int ld_stream(const int32_t* p) {
   int r;
@@ -292,6 +301,28 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
   return nfresh;
 }
 
+// Predicted distinct labels of a row this iteration (steers the row class and
+// table sizes only; overflow always triggers an exact recount).  Labels
+// collapse geometrically as communities form [P:130], so the count of t-1 is
+// extrapolated with the row's own ratio: p_{t-1}^2 / p_{t-2} (GLP_PRED_EXTRAP).
+#ifndef GLP_PRED_EXTRAP
+#define GLP_PRED_EXTRAP 1
+#endif
+__device__ __forceinline__ unsigned pred_est(unsigned raw, unsigned rawprev, unsigned cap) {
+  unsigned p = raw & kPredMask;
+  const unsigned q = rawprev & kPredMask;
+  if (GLP_PRED_EXTRAP && q > p) p = (unsigned)(((unsigned long long)p * p) / q);
+  if (cap) p = min(p, cap);
+  return max(p, 1u);
+}
+// Sorted-row candidate: all labels were distinct last time and the fast path
+// has not been tried on them (every row at t = 1); never for SEEDED (R12).
+template <int VAR>
+__device__ __forceinline__ bool mono_cand(unsigned raw, unsigned cap, int d) {
+  const unsigned p = cap ? min(raw & kPredMask, cap) : (raw & kPredMask);
+  return VAR != V_SEEDED && !(raw & kMonoTried) && p >= (unsigned)d;
+}
+
 // Per-thread iteration statistics, block-reduced once at kernel exit.
 struct Tally {
   unsigned long long changed = 0, d2 = 0, chdeg = 0, arcs = 0, verts = 0;
@@ -439,23 +470,20 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       const int sstart = 31 - __clz(segs & ((2u << lane) - 1u));
       // label frequency inside the vertex's lanes [P:231-232]
       unsigned k = 0;
-      for (int i = 0; i < d; ++i) {
-        const int other = __shfl_sync(kFull, lab, (sstart + i) & 31);
-        k += other == lab ? 1u : 0u;
-      }
+#pragma unroll 4
+      for (int i = 0; i < d; ++i) k += __shfl_sync(kFull, lab, sstart + i) == lab ? 1u : 0u;
       const int head = (lane < nv ? lane * d : 0) & 31;  // lane jv takes segment jv
       Best<VAR> h;
       if (VAR == V_LLP || !GLP_LOW_REDUX) {
         Best<VAR> b;
         if (vote) b.observe(k, (unsigned)lab, a);
-        if (d > 1) {  // warp-uniform: segmented arg-max toward the segment head
-          const int send = sstart + d;
-#pragma unroll
-          for (int s2 = 1; s2 < 32; s2 <<= 1) {
-            const unsigned long long ok = __shfl_down_sync(kFull, b.key, s2);
-            const unsigned ol = __shfl_down_sync(kFull, b.lab, s2);
-            if (s2 < d && lane + s2 < send) b.merge(ok, ol);
-          }
+        // segmented arg-max toward the segment head: ceil(log2 d) steps (d is
+        // warp-uniform)
+        const int send = sstart + d;
+        for (int s2 = 1; s2 < d; s2 <<= 1) {
+          const unsigned long long ok = __shfl_down_sync(kFull, b.key, s2);
+          const unsigned ol = VAR == V_LLP ? __shfl_down_sync(kFull, b.lab, s2) : 0u;
+          if (lane + s2 < send) b.merge(ok, ol);
         }
         h.key = __shfl_sync(kFull, b.key, head);
         h.lab = __shfl_sync(kFull, b.lab, head);
@@ -565,8 +593,10 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
     if (ok) {
       mine = a.items[il];
       const unsigned raw = a.pred[il];
-      mpred = a.pred_cap ? min(raw & kPredMask, a.pred_cap) | (raw & kMonoTried) : raw;
-      ok = row_class(mpred & kPredMask, mine.d) == CLS_W;
+      // in this kernel bit 31 of mpred marks a sorted-row candidate
+      const bool cand = mono_cand<VAR>(raw, a.pred_cap, mine.d);
+      mpred = pred_est(raw, a.pred_prev[il], a.pred_cap) | (cand ? kMonoTried : 0u);
+      ok = row_class(mpred & kPredMask, mine.d, cand) == CLS_W;
       if (ok && !a.dense && !a.flag[a.vb + mine.v]) {
         ok = false;
         a.pred_next[il] = raw;  // inactive: carry the prediction forward
@@ -597,7 +627,8 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
         nd = __shfl_sync(kFull, mine.d, njl);
         npred = __shfl_sync(kFull, mpred, njl);
       }
-      const unsigned tsz = min(max(64u, 1u << (32 - __clz(2u * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
+      const unsigned tsz =
+          min(max(64u, 1u << (32 - __clz(GLP_W_LOAD * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
       const Table tab{tabs[wid], tsz};
       tab.clear(lane, 32);
       if (lane == 0) s_over[wid] = 0;
@@ -605,7 +636,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       Best<VAR> b;
       unsigned fresh = 0;
       bool over = false;
-      bool mono = VAR != V_SEEDED && !(pred & kMonoTried) && pred >= (unsigned)d;  // sorted-row candidate
+      bool mono = (pred & kMonoTried) != 0;  // sorted-row candidate
       const bool tried = mono;
       int prev = -1;
       bool next_loaded = false;  // x0/x1 hold the next row's first round
@@ -709,7 +740,8 @@ __device__ __forceinline__ void block_load_round(const int32_t* col, int64_t sta
 
 // `u` holds round 0 of the row (loaded ahead by the caller); each round loads
 // the next one before gathering its own labels.
-template <int VAR, int BLOCK, int UNROLL>
+// IPF = false: rounds after the first are loaded in place (register-capped L).
+template <int VAR, int BLOCK, int UNROLL, bool IPF>
 __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int d, const Table& tab,
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
                                             volatile int* overflow, int* distinct, Best<VAR>& b) {
@@ -717,7 +749,8 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
   unsigned fresh = 0;
   for (int base = 0; base < d; base += STEP) {
     int4 un[UNROLL];
-    block_load_round<BLOCK, UNROLL>(a.col, start, d, base + STEP, un);
+    if (!IPF && base > 0) block_load_round<BLOCK, UNROLL>(a.col, start, d, base, u);
+    if (IPF) block_load_round<BLOCK, UNROLL>(a.col, start, d, base + STEP, un);
     int lab[4 * UNROLL];
 #pragma unroll
     for (int j = 0; j < UNROLL; ++j) {
@@ -729,8 +762,10 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
       if (stage_out != nullptr && idx < d)
         __stcg((int4*)(stage_out + idx), make_int4(lab[4 * j], lab[4 * j + 1], lab[4 * j + 2], lab[4 * j + 3]));
     }
+    if (IPF) {
 #pragma unroll
-    for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
+      for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
+    }
     fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow);
     if (__any_sync(kFull, *overflow != 0)) break;  // warp-uniform exit
   }
@@ -852,9 +887,12 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
 // Both record the row's exact distinct-label count as the next `pred`.
 template <int VAR, int BLOCK, int SLOTS, bool PART, int UNROLL, int CLS>
 #ifndef GLP_M_MINB
-#define GLP_M_MINB 1
+#define GLP_M_MINB 5
 #endif
-__global__ void __launch_bounds__(BLOCK, PART ? 1 : GLP_M_MINB) mfl_block(MflArgs a) {
+#ifndef GLP_L_MINB
+#define GLP_L_MINB 2
+#endif
+__global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_block(MflArgs a) {
   extern __shared__ __align__(16) unsigned long long smem_tab[];  // SLOTS
   __shared__ int s_over, s_distinct;
   __shared__ int s_hist[PART ? 256 : 1], s_cur[PART ? 256 : 1];
@@ -886,8 +924,8 @@ __global__ void __launch_bounds__(BLOCK, PART ? 1 : GLP_M_MINB) mfl_block(MflArg
         if (!a.mode) {
           const BinItem itk = a.items[ik];
           const unsigned raw = a.pred[ik];
-          const unsigned pk = a.pred_cap ? min(raw & kPredMask, a.pred_cap) : (raw & kPredMask);
-          ok = row_class(pk, itk.d) == CLS;
+          ok = row_class(pred_est(raw, a.pred_prev[ik], a.pred_cap), itk.d, mono_cand<VAR>(raw, a.pred_cap, itk.d)) ==
+               CLS;
           if (ok && !a.dense && !a.flag[a.vb + itk.v]) {
             ok = false;
             a.pred_next[ik] = raw;  // inactive: carry the prediction forward
@@ -921,13 +959,13 @@ __global__ void __launch_bounds__(BLOCK, PART ? 1 : GLP_M_MINB) mfl_block(MflArg
       block_load_round<BLOCK, UNROLL>(a.col, it.start, it.d, 0, cur);
     }
     const unsigned praw = a.pred[i];
-    const bool tried_before = (praw & kMonoTried) != 0;
-    const unsigned pred = a.pred_cap ? min(praw & kPredMask, a.pred_cap) : (praw & kPredMask);
+    const bool cand = mono_cand<VAR>(praw, a.pred_cap, it.d);
+    const unsigned pred = pred_est(praw, a.pred_prev[i], a.pred_cap);
     const int d = it.d;
     Best<VAR> b;
     if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; }
     bool mono_done = false;
-    if (!a.mode && VAR != V_SEEDED && !tried_before && pred >= (unsigned)d) {
+    if (!a.mode && cand) {
       __syncthreads();
       unsigned fr = 0;
       mono_done = block_mono<VAR, BLOCK, UNROLL>(a, it.start, d, cur, b, &fr);
@@ -944,8 +982,14 @@ __global__ void __launch_bounds__(BLOCK, PART ? 1 : GLP_M_MINB) mfl_block(MflArg
     // a re-queued row overflowed a smaller table: its pred is stale.  A row
     // whose last count took the sorted fast path (all labels distinct then)
     // tries one table-sized pass first: labels collapse after t = 1 [P:130]
-    const unsigned est = a.mode ? (unsigned)d : (GLP_L_OPT && tried_before && PART) ? min(max(pred, 1u), (unsigned)SLOTS / 2)
-                                                                         : max(pred, 1u);
+    // L: a row whose last count took the sorted fast path (all labels distinct
+    // at t = 1) is sized at GLP_L_EST % of that count -- labels collapse
+    // [P:130] (RMAT probe at t = 2: 26-36 % distinct for deg > 2048); the
+    // labels are staged, so an overflow recounts them in partitions
+    const unsigned est = a.mode ? (unsigned)d
+                                : (PART && (praw & kMonoTried))
+                                      ? max(1u, (unsigned)(((unsigned long long)pred * GLP_L_EST) / 100ull))
+                                      : pred;
     unsigned nparts = PART ? max(1u, (min(est, (unsigned)d) + SLOTS / 2 - 1) / (SLOTS / 2)) : 1u;
     bool staged = false;  // stageA holds the row's gathered labels
     bool over = false;
@@ -957,7 +1001,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? 1 : GLP_M_MINB) mfl_block(MflArg
       tab.clear(threadIdx.x, BLOCK);
       __syncthreads();
       const bool may_over = PART && 2u * (unsigned)d > (unsigned)SLOTS;
-      block_count<VAR, BLOCK, UNROLL>(a, it.start, d, tab, may_over ? kLProbe : tsz, cur,
+      block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : tsz, cur,
                                       may_over ? stageA : nullptr, &s_over, &s_distinct, b);
       __syncthreads();
       over = s_over != 0;

@@ -4,5 +4,5 @@
 scale=$1; iters=$2; shift 2
 for v in "$@"; do
   echo "=== $v"
-  GLP_LIB=build/$v.so python tools/quick_perf.py $scale $iters 2>&1 | grep -E "^(RunInfo|iter|mfl|push|gen)" | tail -12
+  GLP_LIB=build/$v.so python tools/quick_perf.py $scale $iters 2>&1 | grep -E "^(RunInfo|iter|arcs|mfl|push|gen)" | tail -12
 done

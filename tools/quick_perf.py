@@ -20,9 +20,11 @@ for k in g.kernel_stats():
         print(k['name'], k['launches'], round(k['ms'], 3), 'ms', round(k['bytes'] / max(k['ms'], 1e-9) / 1e6, 1), 'GB/s alg',
               round(k['arcs'] / max(k['ms'], 1e-9) / 1e6, 2), 'Garcs/s')
 # per-iteration kernel breakdown (profiled runs of 1..4 iterations, differences)
-prev = {}
+prev, preva = {}, {}
 for t in range(1, int(sys.argv[2]) + 1 if len(sys.argv) > 2 else 5):
     g.run('classic', t, profile=True)
     cur = {k['name']: k['ms'] for k in g.kernel_stats()}
+    cura = {k['name']: k['arcs'] for k in g.kernel_stats()}
     print('iter', t, {k: round(cur[k] - prev.get(k, 0), 3) for k in cur if cur[k] - prev.get(k, 0) > 0})
-    prev = cur
+    print('arcs', t, {k: round((cura[k] - preva.get(k, 0)) / 1e6, 1) for k in cura if cura[k] - preva.get(k, 0) > 0})
+    prev, preva = cur, cura
