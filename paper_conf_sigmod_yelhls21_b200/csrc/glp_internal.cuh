@@ -45,7 +45,10 @@ constexpr int kWBlock = 256;
 constexpr int kWSlots = 512;
 constexpr int kMBlock = 128;
 constexpr int kMSlots = 4096;
-constexpr int kMUnroll = 2;
+#ifndef GLP_MUNROLL
+#define GLP_MUNROLL 2
+#endif
+constexpr int kMUnroll = GLP_MUNROLL;
 #ifndef GLP_LBLOCK
 #define GLP_LBLOCK 512
 #endif
@@ -54,7 +57,10 @@ constexpr int kMUnroll = 2;
 #endif
 constexpr int kLBlock = GLP_LBLOCK;
 constexpr int kLSlots = GLP_LSLOTS;
-constexpr int kLUnroll = 2;
+#ifndef GLP_LUNROLL
+#define GLP_LUNROLL 1
+#endif
+constexpr int kLUnroll = GLP_LUNROLL;
 constexpr int kLProbe = 32;  // probe limit before declaring a partition overflowed
 // Giant rows (deg > kGiantMin) are split into segments of kGiantSeg arcs that
 // many blocks count concurrently into one global-memory table per row

@@ -51,7 +51,7 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 // loads carry an L2 evict_first hint.  GLP_GATHER_POLICY selects the gathers'
 // hint: 0 none, 1 evict_last.
 #ifndef GLP_STREAM_POLICY
-#define GLP_STREAM_POLICY 1
+#define GLP_STREAM_POLICY 0
 #endif
 #ifndef GLP_GATHER_POLICY
 #define GLP_GATHER_POLICY 0
@@ -73,7 +73,7 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #define GLP_L_EST 40
 #endif
 #ifndef GLP_W_LOAD
-#define GLP_W_LOAD 2
+#define GLP_W_LOAD 4
 #endif
 __device__ __forceinline__ int ld_stream(const int32_t* p) {
   int r;
@@ -162,44 +162,63 @@ __device__ __forceinline__ unsigned slot_hash(unsigned lab, unsigned tsz) {
   return __umulhi(lab * 0x9E3779B1u, tsz);
 }
 
-// Open-addressing count table in shared memory: tsz (a power of two) u64
-// slots holding (label << 32) | count, kEmpty when free; linear probing.
-constexpr unsigned long long kEmpty = ~0ull;
+// Open-addressing count table in shared memory: tsz (a power of two) slots
+// in the storage of tsz u64 words -- key[tsz] (u32 label, kFree when free)
+// then cnt[tsz] (u32) -- with linear probing.  A new label claims its key with
+// a 32-bit CAS; every occurrence (the claimer's included) then adds to the
+// count with a native 32-bit shared atomic, so counts start from the cleared 0.
+constexpr unsigned kFree = 0xffffffffu;
 struct Table {
-  unsigned long long* slots;
+  unsigned* key;
+  unsigned* cnt;
   unsigned tsz;
+  __device__ __forceinline__ Table(unsigned long long* storage, unsigned tsz_)
+      : key((unsigned*)storage), cnt((unsigned*)storage + tsz_), tsz(tsz_) {}
   // cooperative clear by `nthr` threads starting at thread `tid` (16-B stores)
   __device__ __forceinline__ void clear(unsigned tid, unsigned nthr) const {
-    uint4* s4 = (uint4*)slots;
-    for (unsigned j = tid; j < tsz / 2; j += nthr) s4[j] = make_uint4(kFree32, kFree32, kFree32, kFree32);
+    uint4* k4 = (uint4*)key;
+    uint4* c4 = (uint4*)cnt;
+    for (unsigned j = tid; j < tsz / 4; j += nthr) {
+      k4[j] = make_uint4(kFree, kFree, kFree, kFree);
+      c4[j] = make_uint4(0u, 0u, 0u, 0u);
+    }
   }
-  static constexpr unsigned kFree32 = 0xffffffffu;
 };
 
-// Insert `c` occurrences of `lab`.  Returns the post-increment count, or 0
-// when no slot was found within `max_probe` probes (overflow).  *fresh is set
-// when this call claimed a new slot (distinct-label accounting).  A new label
-// costs one CAS that claims the slot and sets its count.
-__device__ __forceinline__ unsigned ht_add(const Table& t, unsigned lab, unsigned c, unsigned max_probe,
-                                           bool* fresh) {
-  unsigned h = slot_hash(lab, t.tsz);
-  for (unsigned p = 0;; ++p) {
-    unsigned long long e = *((volatile unsigned long long*)(t.slots + h));
-    if (e == kEmpty) {
-      const unsigned long long prev = atomicCAS(t.slots + h, kEmpty, ((unsigned long long)lab << 32) | c);
-      if (prev == kEmpty) {
-        *fresh = true;
-        return c;
-      }
-      e = prev;
-    }
-    // increments go to the count half with a native 32-bit shared atomic (a
-    // 64-bit add would be a CAS loop under hot-key contention); a CAS.64 can no
-    // longer succeed on a claimed slot, so the two never race.
-    if ((unsigned)(e >> 32) == lab) return atomicAdd((unsigned*)(t.slots + h), c) + c;
-    if (p + 1 >= max_probe) return 0u;
-    h = (h + 1) & (t.tsz - 1);
+__device__ __forceinline__ unsigned ld_key(const Table& t, unsigned h) { return *((volatile unsigned*)(t.key + h)); }
+
+// One probe of slot h (whose key was read as k) for `c` occurrences of label
+// l: returns the post-add count, or 0 when the slot holds another label.
+// *fresh counts a slot claimed by this call.
+__device__ __forceinline__ unsigned slot_try(const Table& t, unsigned h, unsigned l, unsigned c, unsigned k,
+                                             unsigned* fresh) {
+  if (k == kFree) {
+    const unsigned p = atomicCAS(t.key + h, kFree, l);
+    *fresh += p == kFree ? 1u : 0u;
+    k = p == kFree ? l : p;
   }
+  return k == l ? atomicAdd(t.cnt + h, c) + c : 0u;
+}
+
+// Probe from slot h + 1 on (the home slot h held another label).  Returns the
+// post-add count, or 0 when no slot was found within `max_probe` probes in
+// total (overflow).
+__device__ __forceinline__ unsigned ht_probe_from(const Table& t, unsigned lab, unsigned c, unsigned h,
+                                                  unsigned max_probe, unsigned* fresh) {
+  for (unsigned p = 1; p < max_probe; ++p) {
+    h = (h + 1) & (t.tsz - 1);
+    const unsigned r = slot_try(t, h, lab, c, ld_key(t, h), fresh);
+    if (r) return r;
+  }
+  return 0u;
+}
+
+// Insert `c` occurrences of `lab` (home slot first).
+__device__ __forceinline__ unsigned ht_add(const Table& t, unsigned lab, unsigned c, unsigned max_probe,
+                                           unsigned* fresh) {
+  const unsigned h = slot_hash(lab, t.tsz);
+  const unsigned r = slot_try(t, h, lab, c, ld_key(t, h), fresh);
+  return r ? r : ht_probe_from(t, lab, c, h, max_probe, fresh);
 }
 
 // Batched insert of N labels per lane (-1 = no vote).  First the warp's
@@ -208,28 +227,11 @@ __device__ __forceinline__ unsigned ht_add(const Table& t, unsigned lab, unsigne
 // reduction sums them and lane 0 adds the sum with a single shared atomic, so a
 // collapsed neighbourhood (most neighbours share a community label [P:130])
 // costs a few ALU ops per arc instead of same-address atomics.  The remaining
-// labels are inserted one by one: the N home-slot probes are issued as
-// independent shared loads, then the N atomics, so their latencies overlap;
-// only labels whose home slot holds another label fall back to the probing
-// loop.  Returns this lane's count of newly claimed slots.
-__device__ __forceinline__ unsigned ht_probe_from(const Table& t, unsigned lab, unsigned c, unsigned h,
-                                                  unsigned max_probe, bool* fresh) {
-  for (unsigned p = 1; p < max_probe; ++p) {
-    h = (h + 1) & (t.tsz - 1);
-    unsigned long long e = *((volatile unsigned long long*)(t.slots + h));
-    if (e == kEmpty) {
-      const unsigned long long prev = atomicCAS(t.slots + h, kEmpty, ((unsigned long long)lab << 32) | c);
-      if (prev == kEmpty) {
-        *fresh = true;
-        return c;
-      }
-      e = prev;
-    }
-    if ((unsigned)(e >> 32) == lab) return atomicAdd((unsigned*)(t.slots + h), c) + c;
-  }
-  return 0u;
-}
-
+// labels are inserted one by one: the N home-slot keys are read as
+// independent shared loads, then each label takes its home slot (claim or
+// match) with predicated atomics; only labels whose home slot holds another
+// label fall back to the probing loop.  Returns this lane's count of newly
+// claimed slots.
 template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
                                                   const int (&labin)[N], Best<VAR>& b, volatile int* overflow) {
@@ -240,58 +242,35 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
   unsigned nfresh = 0;
   int cand = b.have() ? (int)b.label() : -1;
 #pragma unroll
-  for (int j = N - 1; j >= 0; --j)
-    if (cand < 0 && lab[j] >= 0) cand = lab[j];
+  for (int j = N - 1; j >= 0; --j) cand = (cand < 0 && lab[j] >= 0) ? lab[j] : cand;
   const int hot = __shfl_sync(kFull, cand, 0);
   if (hot >= 0) {  // warp-uniform
     unsigned hc = 0;
 #pragma unroll
-    for (int j = 0; j < N; ++j)
-      if (lab[j] == hot) {
-        ++hc;
-        lab[j] = -1;
-      }
+    for (int j = 0; j < N; ++j) {
+      hc += lab[j] == hot ? 1u : 0u;
+      lab[j] = lab[j] == hot ? -1 : lab[j];
+    }
     const unsigned tot = __reduce_add_sync(kFull, hc);
     if (lane == 0 && tot) {
-      bool fr = false;
-      const unsigned cnt = ht_add(t, (unsigned)hot, tot, max_probe, &fr);
-      nfresh += fr ? 1u : 0u;
+      const unsigned cnt = ht_add(t, (unsigned)hot, tot, max_probe, &nfresh);
       if (cnt == 0u) *overflow = 1;
       else b.observe(cnt, (unsigned)hot, a);
     }
   }
-  unsigned h[N];
-  unsigned long long e[N];
+  unsigned h[N], k[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     h[j] = slot_hash((unsigned)lab[j], t.tsz);
-    e[j] = lab[j] >= 0 ? *((volatile unsigned long long*)(t.slots + h[j])) : 0ull;
+    k[j] = lab[j] >= 0 ? ld_key(t, h[j]) : 0u;
   }
   unsigned cnt[N];
 #pragma unroll
-  for (int j = 0; j < N; ++j) {
-    cnt[j] = 0u;
-    if (lab[j] >= 0) {
-      const unsigned l = (unsigned)lab[j];
-      if ((unsigned)(e[j] >> 32) == l) {
-        cnt[j] = atomicAdd((unsigned*)(t.slots + h[j]), 1u) + 1u;
-      } else if (e[j] == kEmpty) {
-        const unsigned long long prev = atomicCAS(t.slots + h[j], kEmpty, ((unsigned long long)l << 32) | 1u);
-        if (prev == kEmpty) {
-          cnt[j] = 1u;
-          ++nfresh;
-        } else if ((unsigned)(prev >> 32) == l) {
-          cnt[j] = atomicAdd((unsigned*)(t.slots + h[j]), 1u) + 1u;
-        }
-      }
-    }
-  }
+  for (int j = 0; j < N; ++j) cnt[j] = lab[j] >= 0 ? slot_try(t, h[j], (unsigned)lab[j], 1u, k[j], &nfresh) : 0u;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     if (lab[j] >= 0 && cnt[j] == 0u) {
-      bool fr = false;
-      cnt[j] = ht_probe_from(t, (unsigned)lab[j], 1u, h[j], max_probe, &fr);
-      nfresh += fr ? 1u : 0u;
+      cnt[j] = ht_probe_from(t, (unsigned)lab[j], 1u, h[j], max_probe, &nfresh);
       if (cnt[j] == 0u) *overflow = 1;
     }
   }
