@@ -444,7 +444,11 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, ls_));
     CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, ls_));
     g->grid_low = grid_for(sms, (const void*)mfl_low<V_LLP>, kLowBlock, 0);
-    g->grid_w = grid_for(sms, (const void*)mfl_warp<V_LLP>, kWBlock, 0);
+    const int ws_ = (kWBlock / 32) * kWSlots * 8;
+    CK(cudaFuncSetAttribute(mfl_warp<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
+    CK(cudaFuncSetAttribute(mfl_warp<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
+    CK(cudaFuncSetAttribute(mfl_warp<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
+    g->grid_w = grid_for(sms, (const void*)mfl_warp<V_LLP>, kWBlock, ws_);
     g->grid_m = grid_for(sms, (const void*)GLP_M_KERNEL(V_LLP), kMBlock, ms_);
     g->grid_l = grid_for(sms, (const void*)GLP_L_KERNEL(V_LLP), kLBlock, ls_);
     g->grid_g = grid_for(sms, (const void*)mfl_giant_count<V_LLP>, kGBlock, 0);
@@ -539,7 +543,8 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     MflArgs b = r;
     b.n_items = g->n_rows; b.cnt = c + 1; b.redo_out = g->redo_m; b.redo_out_n = &sc->n_redo_m;
     const int grid = std::min<int>(g->grid_w, (g->n_rows + kWBlock - 1) / kWBlock);
-    timed(g, prof, 1, pend, used, [&] { mfl_warp<VAR><<<grid, kWBlock, 0, g->stream>>>(b); });
+    timed(g, prof, 1, pend, used,
+          [&] { mfl_warp<VAR><<<grid, kWBlock, (kWBlock / 32) * kWSlots * 8, g->stream>>>(b); });
     ++n;
   }
   if (g->n_chunks) {

@@ -39,10 +39,16 @@ constexpr int kLowBlock = 256;
 // Sorted-row candidates (row_class `mono`) go to W whatever their size.
 // A row whose labels overflow its table is re-queued to the next class in the
 // same iteration (exact recount), so `pred` only steers performance.
-constexpr unsigned kWPred = 256, kMPred = 2048;
+#ifndef GLP_WPRED
+#define GLP_WPRED 256
+#endif
+#ifndef GLP_WSLOTS
+#define GLP_WSLOTS 512
+#endif
+constexpr unsigned kWPred = GLP_WPRED, kMPred = 2048;
 constexpr int kWMaxDeg = 4096, kMMaxDeg = 16384;
 constexpr int kWBlock = 256;
-constexpr int kWSlots = 512;
+constexpr int kWSlots = GLP_WSLOTS;
 constexpr int kMBlock = 128;
 constexpr int kMSlots = 4096;
 #ifndef GLP_MUNROLL

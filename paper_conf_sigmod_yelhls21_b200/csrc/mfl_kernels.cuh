@@ -63,14 +63,14 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_L_OPT
 #define GLP_L_OPT 0
 #endif
-#ifndef GLP_XROW
-#define GLP_XROW 0
-#endif
 #ifndef GLP_L_IPF
 #define GLP_L_IPF 0
 #endif
 #ifndef GLP_L_EST
 #define GLP_L_EST 40
+#endif
+#ifndef GLP_M_LOAD
+#define GLP_M_LOAD 4
 #endif
 #ifndef GLP_W_LOAD
 #define GLP_W_LOAD 4
@@ -557,7 +557,7 @@ template <int VAR>
 #define GLP_W_MINB 3
 #endif
 __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
-  __shared__ __align__(16) unsigned long long tabs[kWBlock / 32][kWSlots];
+  extern __shared__ __align__(16) unsigned long long wtabs[];  // [kWBlock / 32][kWSlots] (dynamic)
   __shared__ int s_over[kWBlock / 32];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -608,7 +608,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       }
       const unsigned tsz =
           min(max(64u, 1u << (32 - __clz(GLP_W_LOAD * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
-      const Table tab{tabs[wid], tsz};
+      const Table tab{wtabs + (size_t)wid * kWSlots, tsz};
       tab.clear(lane, 32);
       if (lane == 0) s_over[wid] = 0;
       __syncwarp();
@@ -878,7 +878,9 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
   Tally ty;
   int32_t* stageA = PART ? a.stage + (int64_t)blockIdx.x * 2 * a.stage_stride : nullptr;
   int32_t* stageB = PART ? stageA + a.stage_stride : nullptr;
-  __shared__ int s_k0, s_nsel, s_sel[32];
+  __shared__ int s_k0, s_nsel, s_sel[32], s_cand[32];
+  __shared__ BinItem s_item[32];
+  __shared__ unsigned s_pe[32], s_raw[32];
   const int n_redo = a.mode ? (int)*a.redo_in_n : 0;
   const int lim = a.mode ? n_redo : a.n_items;
   for (;;) {
@@ -895,16 +897,24 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     const int kn = tk < big ? 1 : 32;
     if (k0 >= lim) break;
     if (threadIdx.x < 32) {
+      // lane-parallel selection; the selected rows' descriptors and
+      // predictions are staged in shared memory (no dependent global loads
+      // in the per-row loop)
       const int k = k0 + (int)threadIdx.x;
       bool ok = (int)threadIdx.x < kn && k < lim;
       int ik = -1;
+      BinItem itk;
+      itk.start = 0; itk.v = 0; itk.d = 0;
+      unsigned raw = 0u, pe = 1u;
+      bool cnd = false;
       if (ok) {
         ik = a.mode ? a.redo_in[k] : k;
+        itk = a.items[ik];
+        raw = a.pred[ik];
+        pe = pred_est(raw, a.pred_prev[ik], a.pred_cap);
+        cnd = mono_cand<VAR>(raw, a.pred_cap, itk.d);
         if (!a.mode) {
-          const BinItem itk = a.items[ik];
-          const unsigned raw = a.pred[ik];
-          ok = row_class(pred_est(raw, a.pred_prev[ik], a.pred_cap), itk.d, mono_cand<VAR>(raw, a.pred_cap, itk.d)) ==
-               CLS;
+          ok = row_class(pe, itk.d, cnd) == CLS;
           if (ok && !a.dense && !a.flag[a.vb + itk.v]) {
             ok = false;
             a.pred_next[ik] = raw;  // inactive: carry the prediction forward
@@ -912,34 +922,26 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
         }
       }
       const unsigned m = __ballot_sync(kFull, ok);
-      if (ok) s_sel[__popc(m & ((1u << threadIdx.x) - 1u))] = ik;
+      if (ok) {
+        const int pos = __popc(m & ((1u << threadIdx.x) - 1u));
+        s_sel[pos] = ik;
+        s_item[pos] = itk;
+        s_pe[pos] = pe;
+        s_raw[pos] = raw;
+        s_cand[pos] = cnd ? 1 : 0;
+      }
       if (threadIdx.x == 0) s_nsel = __popc(m);
     }
     __syncthreads();
     const int nsel = s_nsel;
-    // round 0 of the next selected row is loaded while the current row is
-    // counted (cross-row software pipeline)
-    BinItem nit;
-    nit.start = 0; nit.v = 0; nit.d = 0;
-    int4 pre[UNROLL];
-    if (nsel > 0) nit = a.items[s_sel[0]];
-    if (GLP_XROW) block_load_round<BLOCK, UNROLL>(a.col, nit.start, nit.d, 0, pre);
     for (int q = 0; q < nsel; ++q) {
     const int i = s_sel[q];
-    const BinItem it = nit;
+    const BinItem it = s_item[q];
     int4 cur[UNROLL];
-#pragma unroll
-    for (int j = 0; j < UNROLL; ++j) cur[j] = pre[j];
-    nit.d = 0;
-    if (q + 1 < nsel) nit = a.items[s_sel[q + 1]];
-    if (GLP_XROW) {
-      block_load_round<BLOCK, UNROLL>(a.col, nit.start, nit.d, 0, pre);
-    } else {
-      block_load_round<BLOCK, UNROLL>(a.col, it.start, it.d, 0, cur);
-    }
-    const unsigned praw = a.pred[i];
-    const bool cand = mono_cand<VAR>(praw, a.pred_cap, it.d);
-    const unsigned pred = pred_est(praw, a.pred_prev[i], a.pred_cap);
+    block_load_round<BLOCK, UNROLL>(a.col, it.start, it.d, 0, cur);
+    const unsigned praw = s_raw[q];
+    const bool cand = s_cand[q] != 0;
+    const unsigned pred = s_pe[q];
     const int d = it.d;
     Best<VAR> b;
     if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; }
@@ -958,9 +960,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       }
     }
     if (!mono_done) {
-    // a re-queued row overflowed a smaller table: its pred is stale.  A row
-    // whose last count took the sorted fast path (all labels distinct then)
-    // tries one table-sized pass first: labels collapse after t = 1 [P:130]
+    // a re-queued row overflowed a smaller table: its pred is stale.
     // L: a row whose last count took the sorted fast path (all labels distinct
     // at t = 1) is sized at GLP_L_EST % of that count -- labels collapse
     // [P:130] (RMAT probe at t = 2: 26-36 % distinct for deg > 2048); the
@@ -974,7 +974,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     bool over = false;
     if (nparts == 1u) {
       // single pass: gather + count (L: stage the labels if an overflow is possible)
-      const unsigned want = PART ? 2u * (unsigned)d : 4u * est;
+      const unsigned want = PART ? 2u * (unsigned)d : GLP_M_LOAD * est;
       const unsigned tsz = min(max(64u, 1u << (32 - __clz(want - 1u))), (unsigned)SLOTS);
       const Table tab{smem_tab, tsz};
       tab.clear(threadIdx.x, BLOCK);

@@ -103,3 +103,27 @@ extern "C" float ub_match(const int* L, unsigned long long* out, int sms) {
   Args a{nullptr, 0, L, out, sms, 0};
   return time_it([](void* p) { Args* a = (Args*)p; k_match<<<a->sms * 4, 512>>>(1024, a->L, a->out); }, &a, 5);
 }
+
+// Realistic table traffic: every lane hits a hashed slot of a 4096-entry
+// shared table (bank conflicts as in the MFL tables).  mode 0: LDS, 1: atomicAdd
+// with the return value used, 2: atomicCAS (32-bit), 3: atomicAdd without return.
+__global__ void k_atoms2(int iters, int mode, unsigned long long* out) {
+  __shared__ unsigned tab[4096];
+  for (int i = threadIdx.x; i < 4096; i += blockDim.x) tab[i] = 0;
+  __syncthreads();
+  unsigned x = threadIdx.x * 2654435761u + blockIdx.x, s = 0;
+  for (int i = 0; i < iters; ++i) {
+    const unsigned h = __umulhi(x * 0x9E3779B1u, 4096u);
+    if (mode == 0) s += ((volatile unsigned*)tab)[h];
+    else if (mode == 1) s += atomicAdd(&tab[h], 1u);
+    else if (mode == 2) s += atomicCAS(&tab[h], s, x);
+    else atomicAdd(&tab[h], 1u);
+    x = x * 1664525u + 1013904223u + (s & 1u);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && (tab[5] + s) == 0x1234567) atomicAdd(out, 1ull);
+}
+extern "C" float ub_atoms2(int mode, unsigned long long* out, int sms) {
+  Args a{nullptr, 0, nullptr, out, sms, mode};
+  return time_it([](void* p) { Args* a = (Args*)p; k_atoms2<<<a->sms * 4, 512>>>(1024, a->mode, a->out); }, &a, 5);
+}

@@ -6,11 +6,11 @@ here = os.path.dirname(os.path.abspath(__file__))
 so = os.path.join(here, 'libubench.so')
 subprocess.check_call(['nvcc', '-gencode', 'arch=compute_100a,code=sm_100a', '-O3', '-Xcompiler', '-fPIC', '-shared', '-o', so, os.path.join(here, 'ubench.cu')])
 lib = ctypes.CDLL(so)
-for f in ['ub_stream', 'ub_gather', 'ub_atoms', 'ub_match']:
+for f in ['ub_stream', 'ub_gather', 'ub_atoms', 'ub_match', 'ub_atoms2']:
     getattr(lib, f).restype = ctypes.c_float
 P, I64, I32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
 lib.ub_stream.argtypes = [P, I64, P, I32]; lib.ub_gather.argtypes = [P, I64, P, P, I32, I32]
-lib.ub_atoms.argtypes = [I32, P, I32]; lib.ub_match.argtypes = [P, P, I32]
+lib.ub_atoms.argtypes = [I32, P, I32]; lib.ub_atoms2.argtypes = [I32, P, I32]; lib.ub_match.argtypes = [P, P, I32]
 scale = int(sys.argv[1]) if len(sys.argv) > 1 else 24
 csr = graphs.rmat(scale, seed=1, device='cuda')
 sms = torch.cuda.get_device_properties(0).multi_processor_count
@@ -34,3 +34,7 @@ for d in (1, 0):
 ms = lib.ub_match(L.data_ptr(), out.data_ptr(), sms)
 ops = sms * 4 * 16 * 1024
 print(f'match_any: {ms:.3f} ms  {ops/ms/1e6/sms/1.9:.3f} warp-ops/clk/SM')
+for mode, name in [(0, 'LDS hashed'), (1, 'atomicAdd hashed, return used'), (2, 'atomicCAS hashed'), (3, 'atomicAdd hashed, no return')]:
+    ms = lib.ub_atoms2(mode, out.data_ptr(), sms)
+    ops = sms * 4 * 512 * 1024
+    print(f'smem {name}: {ms:.3f} ms  {ops/ms/1e6/sms/1.965:.2f} lane-ops/clk/SM')
