@@ -17,6 +17,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <string>
 #include <vector>
 
@@ -120,6 +121,8 @@ void free_graph(glp_graph* g) {
   if (g->ev_a) cudaEventDestroy(g->ev_a);
   if (g->ev_b) cudaEventDestroy(g->ev_b);
   for (auto& e : g->ev_pool) cudaEventDestroy(e);
+  for (auto& e : g->xev) if (e) cudaEventDestroy(e);
+  for (auto& x : g->xs) if (x) cudaStreamDestroy(x);
   nccl_destroy(g);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   delete g;
@@ -434,6 +437,12 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaMallocHost(&g->h_cnt, 5 * sizeof(Counters)));
     CK(cudaEventCreate(&g->ev_a));
     CK(cudaEventCreate(&g->ev_b));
+    {
+      const char* ser = getenv("GLP_SERIAL");
+      g->concurrent = !(ser && ser[0] == '1');
+    }
+    for (auto& x : g->xs) CK(cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking));
+    for (auto& e : g->xev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
 
     const int sms = g->sms;
     const int ms_ = kMSlots * 8, ls_ = kLSlots * 8;
@@ -513,14 +522,30 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   r.items = g->rows; r.big_prefix = g->n_ge8k; r.pred = g->pred[g->pb]; r.pred_prev = g->pred[(g->pb + 2) % 3];
   r.pred_next = g->pred[(g->pb + 1) % 3];
   r.stage = g->stage; r.stage_stride = g->stage_stride;
+  // The class kernels of one iteration touch disjoint rows, so they run
+  // concurrently (filling each other's tails) unless profiling or GLP_SERIAL:
+  // giant | L | M | low on their own streams, W -> redo M -> redo L on the
+  // main stream (redo L also waits for the static M, which feeds its queue).
+  const bool cc = g->concurrent && !prof;
+  cudaStream_t s0 = g->stream;
+  bool used_x[4] = {false, false, false, false};
+  auto S = [&](int i) -> cudaStream_t {
+    if (!cc) return s0;
+    used_x[i] = true;
+    return g->xs[i];
+  };
+  if (cc) {
+    CK(cudaEventRecord(g->xev[0], s0));
+    for (auto x : g->xs) CK(cudaStreamWaitEvent(x, g->xev[0], 0));
+  }
   if (g->n_giant) {  // giant rows: all blocks count segments into per-row global tables
     MflArgs b = r;
     b.cnt = c + 4; b.work = &sc->work_g;
     b.gsegs = g->gsegs; b.n_gsegs = g->n_gsegs; b.gtab = g->gtab; b.gtab_off = g->gtab_off;
     b.gcand_key = g->gcand_key; b.gcand_lab = g->gcand_lab; b.gdistinct = g->gdistinct; b.epoch = g->gepoch;
     timed(g, prof, 7, pend, used, [&] {
-      mfl_giant_count<VAR><<<std::min(g->grid_g, g->n_gsegs), kGBlock, 0, g->stream>>>(b);
-      mfl_giant_finish<VAR><<<g->n_giant, 256, 0, g->stream>>>(b, g->gseg_first);
+      mfl_giant_count<VAR><<<std::min(g->grid_g, g->n_gsegs), kGBlock, 0, S(0)>>>(b);
+      mfl_giant_finish<VAR><<<g->n_giant, 256, 0, S(0)>>>(b, g->gseg_first);
     });
     n += 2;
   }
@@ -528,7 +553,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     MflArgs b = r;
     b.n_items = g->n_gt2048; b.cnt = c + 3; b.work = &sc->work_l;
     const int grid = std::min<int>(g->grid_l, g->n_ge8k + (g->n_gt2048 - g->n_ge8k + 31) / 32);
-    timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<grid, kLBlock, ls_, g->stream>>>(b); });
+    timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<grid, kLBlock, ls_, S(1)>>>(b); });
     ++n;
   }
   if (g->n_gt256) {  // M, static; overflowing rows -> L redo list
@@ -536,7 +561,8 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     b.n_items = g->n_gt256; b.cnt = c + 2; b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
     b.work = &sc->work_m;
     const int grid = std::min<int>(g->grid_m, g->n_ge8k + (g->n_gt256 - g->n_ge8k + 31) / 32);
-    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<grid, kMBlock, ms_, g->stream>>>(b); });
+    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<grid, kMBlock, ms_, S(2)>>>(b); });
+    if (cc) CK(cudaEventRecord(g->xev[1], g->xs[2]));
     ++n;
   }
   if (g->n_rows) {  // W: every row of class W; overflowing rows -> M redo list
@@ -544,14 +570,14 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     b.n_items = g->n_rows; b.cnt = c + 1; b.redo_out = g->redo_m; b.redo_out_n = &sc->n_redo_m;
     const int grid = std::min<int>(g->grid_w, (g->n_rows + kWBlock - 1) / kWBlock);
     timed(g, prof, 1, pend, used,
-          [&] { mfl_warp<VAR><<<grid, kWBlock, (kWBlock / 32) * kWSlots * 8, g->stream>>>(b); });
+          [&] { mfl_warp<VAR><<<grid, kWBlock, (kWBlock / 32) * kWSlots * 8, s0>>>(b); });
     ++n;
   }
   if (g->n_chunks) {
     MflArgs b = a;
     b.low_base = g->low_base; b.chunks = g->chunks; b.cflag = g->cflag; b.n_chunks = g->n_chunks; b.cnt = c + 0;
     const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock - 1) / kLowBlock);
-    timed(g, prof, 0, pend, used, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, g->stream>>>(b); });
+    timed(g, prof, 0, pend, used, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, S(3)>>>(b); });
     ++n;
   }
   if (g->n_rows) {
@@ -561,11 +587,22 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     MflArgs b = r;
     b.mode = 1; b.cnt = c + 2; b.redo_in = g->redo_m; b.redo_in_n = &sc->n_redo_m; b.work = &sc->work_mr;
     b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
-    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<g->grid_m, kMBlock, ms_, g->stream>>>(b); });
+    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<g->grid_m, kMBlock, ms_, s0>>>(b); });
+    if (used_x[2]) CK(cudaStreamWaitEvent(s0, g->xev[1], 0));
     MflArgs q = r;
     q.mode = 1; q.cnt = c + 3; q.redo_in = g->redo_l; q.redo_in_n = &sc->n_redo_l; q.work = &sc->work_lr;
-    timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<g->grid_l, kLBlock, ls_, g->stream>>>(q); });
+    timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<g->grid_l, kLBlock, ls_, s0>>>(q); });
     n += 2;
+  }
+  if (cc) {
+    // join: the main stream waits for every side stream used
+    const int xe[4] = {2, 3, 1, 4};
+    for (int i = 0; i < 4; ++i)
+      if (used_x[i] && i != 2) {
+        CK(cudaEventRecord(g->xev[xe[i]], g->xs[i]));
+        CK(cudaStreamWaitEvent(s0, g->xev[xe[i]], 0));
+      }
+    if (used_x[2] && !g->n_rows) CK(cudaStreamWaitEvent(s0, g->xev[1], 0));
   }
   return n;
 }

@@ -268,6 +268,11 @@ struct glp_graph {
   std::vector<glp_iter_stat> iter_stats;
   std::vector<glp::KStat> kstats;
   cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+  // concurrent class kernels within an iteration (GLP_SERIAL=1 disables):
+  // xs[0] giant, xs[1] L, xs[2] M, xs[3] low; W and the redo chain on `stream`
+  bool concurrent = true;
+  cudaStream_t xs[4] = {nullptr, nullptr, nullptr, nullptr};
+  cudaEvent_t xev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
   std::vector<cudaEvent_t> ev_pool;
 
   // pooled device allocations (freed in destroy)
