@@ -497,17 +497,19 @@ const char* kKernelNames[] = {"mfl_low", "mfl_warp", "mfl_block_m", "mfl_block_l
 constexpr int kNumKernelNames = 8;
 
 template <class F>
-void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t& used, F f) {
+void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t& used, cudaStream_t st, F f) {
   if (!prof) {
     f();
     CK(cudaGetLastError());
     return;
   }
+  // events on the launching stream: with concurrent class kernels the time is
+  // the launch's duration while it shares the GPU with the others
   cudaEvent_t a = pool_event(g, used), b = pool_event(g, used);
-  CK(cudaEventRecord(a, g->stream));
+  CK(cudaEventRecord(a, st));
   f();
   CK(cudaGetLastError());
-  CK(cudaEventRecord(b, g->stream));
+  CK(cudaEventRecord(b, st));
   pend.push_back({kid, a, b, g->cur_t});
 }
 
@@ -526,7 +528,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   // concurrently (filling each other's tails) unless profiling or GLP_SERIAL:
   // giant | L | M | low on their own streams, W -> redo M -> redo L on the
   // main stream (redo L also waits for the static M, which feeds its queue).
-  const bool cc = g->concurrent && !prof;
+  const bool cc = g->concurrent;
   cudaStream_t s0 = g->stream;
   bool used_x[4] = {false, false, false, false};
   auto S = [&](int i) -> cudaStream_t {
@@ -543,7 +545,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     b.cnt = c + 4; b.work = &sc->work_g;
     b.gsegs = g->gsegs; b.n_gsegs = g->n_gsegs; b.gtab = g->gtab; b.gtab_off = g->gtab_off;
     b.gcand_key = g->gcand_key; b.gcand_lab = g->gcand_lab; b.gdistinct = g->gdistinct; b.epoch = g->gepoch;
-    timed(g, prof, 7, pend, used, [&] {
+    timed(g, prof, 7, pend, used, cc ? g->xs[0] : s0, [&] {
       mfl_giant_count<VAR><<<std::min(g->grid_g, g->n_gsegs), kGBlock, 0, S(0)>>>(b);
       mfl_giant_finish<VAR><<<g->n_giant, 256, 0, S(0)>>>(b, g->gseg_first);
     });
@@ -553,7 +555,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     MflArgs b = r;
     b.n_items = g->n_gt2048; b.cnt = c + 3; b.work = &sc->work_l;
     const int grid = std::min<int>(g->grid_l, g->n_ge8k + (g->n_gt2048 - g->n_ge8k + 31) / 32);
-    timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<grid, kLBlock, ls_, S(1)>>>(b); });
+    timed(g, prof, 3, pend, used, cc ? g->xs[1] : s0, [&] { GLP_L_KERNEL(VAR)<<<grid, kLBlock, ls_, S(1)>>>(b); });
     ++n;
   }
   if (g->n_gt256) {  // M, static; overflowing rows -> L redo list
@@ -561,7 +563,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     b.n_items = g->n_gt256; b.cnt = c + 2; b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
     b.work = &sc->work_m;
     const int grid = std::min<int>(g->grid_m, g->n_ge8k + (g->n_gt256 - g->n_ge8k + 31) / 32);
-    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<grid, kMBlock, ms_, S(2)>>>(b); });
+    timed(g, prof, 2, pend, used, cc ? g->xs[2] : s0, [&] { GLP_M_KERNEL(VAR)<<<grid, kMBlock, ms_, S(2)>>>(b); });
     if (cc) CK(cudaEventRecord(g->xev[1], g->xs[2]));
     ++n;
   }
@@ -569,7 +571,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     MflArgs b = r;
     b.n_items = g->n_rows; b.cnt = c + 1; b.redo_out = g->redo_m; b.redo_out_n = &sc->n_redo_m;
     const int grid = std::min<int>(g->grid_w, (g->n_rows + kWBlock - 1) / kWBlock);
-    timed(g, prof, 1, pend, used,
+    timed(g, prof, 1, pend, used, s0,
           [&] { mfl_warp<VAR><<<grid, kWBlock, (kWBlock / 32) * kWSlots * 8, s0>>>(b); });
     ++n;
   }
@@ -577,7 +579,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     MflArgs b = a;
     b.low_base = g->low_base; b.chunks = g->chunks; b.cflag = g->cflag; b.n_chunks = g->n_chunks; b.cnt = c + 0;
     const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock - 1) / kLowBlock);
-    timed(g, prof, 0, pend, used, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, S(3)>>>(b); });
+    timed(g, prof, 0, pend, used, cc ? g->xs[3] : s0, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, S(3)>>>(b); });
     ++n;
   }
   if (g->n_rows) {
@@ -587,11 +589,11 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     MflArgs b = r;
     b.mode = 1; b.cnt = c + 2; b.redo_in = g->redo_m; b.redo_in_n = &sc->n_redo_m; b.work = &sc->work_mr;
     b.redo_out = g->redo_l; b.redo_out_n = &sc->n_redo_l;
-    timed(g, prof, 2, pend, used, [&] { GLP_M_KERNEL(VAR)<<<g->grid_m, kMBlock, ms_, s0>>>(b); });
+    timed(g, prof, 2, pend, used, s0, [&] { GLP_M_KERNEL(VAR)<<<g->grid_m, kMBlock, ms_, s0>>>(b); });
     if (used_x[2]) CK(cudaStreamWaitEvent(s0, g->xev[1], 0));
     MflArgs q = r;
     q.mode = 1; q.cnt = c + 3; q.redo_in = g->redo_l; q.redo_in_n = &sc->n_redo_l; q.work = &sc->work_lr;
-    timed(g, prof, 3, pend, used, [&] { GLP_L_KERNEL(VAR)<<<g->grid_l, kLBlock, ls_, s0>>>(q); });
+    timed(g, prof, 3, pend, used, s0, [&] { GLP_L_KERNEL(VAR)<<<g->grid_l, kLBlock, ls_, s0>>>(q); });
     n += 2;
   }
   if (cc) {
@@ -745,7 +747,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       default: launches += launch_mfl<V_LLP>(g, a, prof, pend, used); break;
     }
     if (g->nccl) {
-      timed(g, prof, 6, pend, used, [&] { nccl_exchange(g, g->L[1 - rb]); });
+      timed(g, prof, 6, pend, used, s, [&] { nccl_exchange(g, g->L[1 - rb]); });
       nccl_sum_counters(g, g->d_cnt, 5 * sizeof(Counters) / sizeof(unsigned long long));
     }
     CK(cudaMemcpyAsync(g->h_cnt, g->d_cnt, 5 * sizeof(Counters), cudaMemcpyDeviceToHost, s));
@@ -785,7 +787,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       next_dense = (double)tot.chdeg * (double)p.dense_divisor > (double)g->nnz_global;
     if (!stop && !next_dense) {
       launches += 1;
-      timed(g, prof, 4, pend, used, [&] {
+      timed(g, prof, 4, pend, used, s, [&] {
         k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, g->flag[nf]);
         if (g->nccl) nccl_merge_flags(g, g->flag[nf]);
         if (g->n_chunks)
@@ -800,7 +802,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     }
     if (!stop && variant == GLP_VARIANT_LLP) {
       launches += 1;
-      timed(g, prof, 5, pend, used, [&] {
+      timed(g, prof, 5, pend, used, s, [&] {
         CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
         k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb], g->n, g->V);
       });
