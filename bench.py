@@ -46,6 +46,7 @@ WORKLOADS = {
     "taobao100m": (dict(kind="taobao", users=80_000_000, items=20_000_000, pairs=1_000_000_000, seed=7),
                    "seeded", 20, 0.0),
     "rmat24_llp": (dict(kind="rmat", scale=24, edge_factor=16, seed=1), "llp", 20, 1.0),
+    "rmat28_llp": (dict(kind="rmat", scale=28, edge_factor=16, seed=1, buckets=16), "llp", 20, 1.0),
     "karate": (dict(kind="karate"), "classic", 20, 0.0),
 }
 
@@ -256,7 +257,8 @@ def bench_gpu(args):
             "data": "synthetic",
             "config": {"workload": args.workload, "generator": spec, "variant": variant, "gamma": gamma,
                        "max_iters": max_iters, "n": n, "arcs": nnz, "parallelism": f"vertex-range x{world}",
-                       "l2": "inputs larger than L2 (2.1 GB arcs for rmat24) and a 256 MB L2 flush before every step",
+                       "l2": f"inputs larger than L2 ({4 * nnz / 1e9:.2f} GB of arcs) and a 256 MB L2 flush "
+                             "before every step",
                        "graph_gen_s": round(t_gen, 2), "bins": info["bins"], "max_degree": info["max_degree"]},
             "iterations": iters, "stop_reason": glp.STOP_NAMES[infos[-1].stop_reason],
             "time_to_converge_ms": round(ms_per_step, 4),

@@ -161,9 +161,75 @@ def rmat_pairs(scale: int, edge_factor: int = 16, seed: int = 1, a=0.57, b=0.19,
     return n, src, dst
 
 
-def rmat(scale: int, edge_factor: int = 16, seed: int = 1, device="cpu", scramble=True) -> CSR:
-    n, src, dst = rmat_pairs(scale, edge_factor, seed, device=device, scramble=scramble)
-    return from_edges(n, src, dst, f"rmat{scale}ef{edge_factor}")
+def _rmat_chunk(scale, lo, hi, seed, a, ab, abc, device):
+    """(row, col) of Kronecker pairs [lo, hi) before the scramble (rmat_pairs' draws)."""
+    idx = torch.arange(lo, hi, dtype=torch.int64, device=device)
+    r = torch.zeros_like(idx)
+    cc = torch.zeros_like(idx)
+    for lvl in range(0, scale, 2):
+        u0, u1 = rng.uniform_pair(seed, 100 + lvl // 2, idx)
+        for j, u in enumerate((u0, u1)):
+            if lvl + j >= scale:
+                break
+            bit = 1 << (lvl + j)
+            r |= (u >= ab).to(torch.int64) * bit
+            cc |= (((u >= a) & (u < ab)) | (u >= abc)).to(torch.int64) * bit
+    return r, cc
+
+
+def rmat(scale: int, edge_factor: int = 16, seed: int = 1, device="cpu", scramble=True,
+         buckets: int = 0) -> CSR:
+    """RMAT CSR = from_edges(rmat_pairs(...)).  buckets > 1 builds the same CSR
+    in row buckets (pairs generated chunk by chunk, each directed arc kept as a
+    bucket-local int64 key) so that scale 28 (2^32 pairs, ~8.5e9 arcs) fits in
+    one GPU's memory; the result is identical to the unbucketed build."""
+    if buckets <= 1:
+        n, src, dst = rmat_pairs(scale, edge_factor, seed, device=device, scramble=scramble)
+        return from_edges(n, src, dst, f"rmat{scale}ef{edge_factor}")
+    n = 1 << scale
+    m = edge_factor * n
+    a, b, c = 0.57, 0.19, 0.19
+    perm = rng.permutation(seed, 99, n, device) if scramble else None
+    width = (n + buckets - 1) // buckets
+    keys = [[] for _ in range(buckets)]
+    chunk = 1 << 26
+    for s0 in range(0, m, chunk):
+        r, cc = _rmat_chunk(scale, s0, min(m, s0 + chunk), seed, a, a + b, a + b + c, device)
+        if perm is not None:
+            r, cc = perm[r], perm[cc]
+        keep = r != cc
+        r, cc = r[keep], cc[keep]
+        src, dst = torch.cat([r, cc]), torch.cat([cc, r])  # symmetrise (R1)
+        del r, cc, keep
+        bk = torch.div(src, width, rounding_mode="floor")
+        order = torch.argsort(bk, stable=True)
+        src, dst, bk = src[order], dst[order], bk[order]
+        cnt = torch.bincount(bk, minlength=buckets).tolist()
+        pos = 0
+        for i, k in enumerate(cnt):
+            if k:
+                keys[i].append((src[pos:pos + k] - i * width) * n + dst[pos:pos + k])
+            pos += k
+        del src, dst, bk, order
+    off = torch.zeros(n + 1, dtype=torch.int64, device=device)
+    cols = []
+    base = 0
+    for i in range(buckets):
+        r0, r1 = i * width, min(n, (i + 1) * width)
+        if keys[i]:
+            key = torch.unique(torch.cat(keys[i]))  # sorted, deduplicated
+        else:
+            key = torch.zeros(0, dtype=torch.int64, device=device)
+        keys[i] = None
+        rows = torch.div(key, n, rounding_mode="floor")
+        cols.append((key - rows * n).to(torch.int32))
+        counts = torch.bincount(rows, minlength=r1 - r0)
+        off[r0 + 1:r1 + 1] = base + torch.cumsum(counts, 0)
+        base += int(key.numel())
+        del key, rows, counts
+    col = torch.cat(cols) if len(cols) > 1 else cols[0]
+    del cols
+    return CSR(n, off, col.contiguous(), f"rmat{scale}ef{edge_factor}")
 
 
 def _trunc_powerlaw_quantiles(count: int, alpha: float, lo: float, hi: float, device):
@@ -244,7 +310,7 @@ CONFIGS = {
     "sbm1m": dict(kind="sbm", n=1_000_000, k=1000, m=20_000_000, mu=0.1, seed=42),
     "rmat24": dict(kind="rmat", scale=24, edge_factor=16, seed=1),
     "taobao100m": dict(kind="taobao", users=80_000_000, items=20_000_000, pairs=1_000_000_000, seed=7),
-    "rmat28": dict(kind="rmat", scale=28, edge_factor=16, seed=1),
+    "rmat28": dict(kind="rmat", scale=28, edge_factor=16, seed=1, buckets=16),
 }
 
 

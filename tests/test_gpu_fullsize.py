@@ -84,3 +84,64 @@ def test_taobao100m_seeded_first_iterations():
     assert [x["changed"] for x in st] == list(ref.changed)
     assert (lab == ref.labels).all()
     assert (lab[s] == s).all()
+
+
+# ---- RMAT-28 (configs[4]: ~8.5e9 arcs, LLP gamma = 1) on one B200 ----------
+# The whole-run oracle would take hours here, so parity is checked on what the
+# oracle can compute at this size: iteration 1 everywhere (closed form), and
+# iteration 2 on sampled vertices recomputed by oracle.step from the GPU's L_1
+# (which iteration 1 pins) and its histogram V.
+
+@pytest.fixture(scope="module")
+def rmat28():
+    if os.environ.get("GLP_SKIP_R28") == "1":
+        pytest.skip("GLP_SKIP_R28=1")
+    free, _ = torch.cuda.mem_get_info()
+    if free < 150e9:
+        pytest.skip("RMAT-28 needs ~120 GB of device memory")
+    csr = graphs.rmat(28, seed=1, device="cuda", buckets=16)
+    g = glp.Graph(csr)
+    yield csr, g
+    g.close()
+
+
+def test_rmat28_llp_iteration1_closed_form(rmat28):
+    csr, g = rmat28
+    info = g.run("llp", 1, gamma=1.0)
+    assert info.iterations == 1
+    lab = g.labels("cuda")
+    off = csr.row_offsets
+    deg = off[1:] - off[:-1]
+    first = csr.col_idx[off[:-1].clamp(max=max(csr.nnz - 1, 0))].to(torch.int64)  # rows are sorted: min N(v)
+    exp = torch.where(deg > 0, first, torch.arange(csr.n, device="cuda"))
+    assert torch.equal(lab.to(torch.int64), exp)
+
+
+def test_rmat28_llp_iteration2_sampled_oracle(rmat28):
+    csr, g = rmat28
+    g.run("llp", 1, gamma=1.0)
+    L1 = g.labels("cuda").clone()
+    g.run("llp", 2, gamma=1.0)
+    L2 = g.labels("cuda")
+    n = csr.n
+    off = csr.row_offsets
+    deg = off[1:] - off[:-1]
+    gen = torch.Generator(device="cpu").manual_seed(28)
+    samp = torch.randint(0, n, (3000,), generator=gen).to("cuda")
+    top = torch.topk(deg, 24).indices  # the longest rows (giant / L paths)
+    samp = torch.unique(torch.cat([samp, top, (deg > 32).nonzero().flatten()[:500]]))
+    # compact problem for oracle.step: rows = samples, their arcs point at a
+    # copy of the neighbours' L_1 values placed after the sample rows
+    d = deg[samp]
+    S, A = samp.numel(), int(d.sum())
+    offc = torch.zeros(S + A + 1, dtype=torch.int64, device="cuda")
+    offc[1:S + 1] = torch.cumsum(d, 0)
+    offc[S + 1:] = A
+    starts = off[samp]
+    rel = torch.arange(A, device="cuda") - torch.repeat_interleave(offc[:S], d)
+    nbr = csr.col_idx[torch.repeat_interleave(starts, d) + rel].to(torch.int64)
+    colc = (S + torch.arange(A, device="cuda")).to(torch.int32)
+    Lp = torch.cat([L1[samp], L1[nbr]]).cpu().numpy()
+    V = torch.bincount(L1.to(torch.int64), minlength=n).to(torch.int32).cpu().numpy()
+    out = oracle.step((S + A, offc.cpu().numpy(), colc.cpu().numpy()), oracle.LLP, Lp, 0, S, V=V, gamma=1.0)
+    assert (out[:S] == L2[samp].cpu().numpy()).all()
