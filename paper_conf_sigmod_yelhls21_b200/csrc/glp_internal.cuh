@@ -68,6 +68,12 @@ constexpr int kLSlots = GLP_LSLOTS;
 #endif
 constexpr int kLUnroll = GLP_LUNROLL;
 constexpr int kLProbe = 32;  // probe limit before declaring a partition overflowed
+// Probe limit of the W and M tables (sized >= 4x the predicted distinct
+// labels, so a legitimate insert rarely probes far).  A row whose prediction
+// was far too low (LLP's oscillating regime) fills its table; without a limit
+// every further new label would probe the whole table before the overflow is
+// noticed.  Hitting the limit re-queues the row to the next class (exact).
+constexpr unsigned kTabProbe = 32;
 // Giant rows (deg > kGiantMin) are split into segments of kGiantSeg arcs that
 // many blocks count concurrently into one global-memory table per row
 // (epoch-tagged slots, never cleared between iterations); a second kernel

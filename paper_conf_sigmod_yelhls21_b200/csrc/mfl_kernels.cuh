@@ -187,6 +187,22 @@ struct Table {
 
 __device__ __forceinline__ unsigned ld_key(const Table& t, unsigned h) { return *((volatile unsigned*)(t.key + h)); }
 
+// LLP scores each distinct label once, from the final table (one V[l] gather
+// per distinct label), instead of at every insert: the table
+// inserts skip `observe` for LLP, and the counting threads scan the table after
+// the barrier that ends the count.  (CLASSIC/SEEDED keep the running arg-max
+// of the insert observations, which needs no scan.)
+template <int VAR>
+__device__ __forceinline__ void table_scan(const Table& t, unsigned tid, unsigned nthr, const MflArgs& a,
+                                           Best<VAR>& b) {
+  if constexpr (VAR == V_LLP) {
+    for (unsigned j = tid; j < t.tsz; j += nthr) {
+      const unsigned k = t.key[j];
+      if (k != kFree) b.observe(t.cnt[j], k, a);
+    }
+  }
+}
+
 // One probe of slot h (whose key was read as k) for `c` occurrences of label
 // l: returns the post-add count, or 0 when the slot holds another label.
 // *fresh counts a slot claimed by this call.
@@ -255,7 +271,7 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
     if (lane == 0 && tot) {
       const unsigned cnt = ht_add(t, (unsigned)hot, tot, max_probe, &nfresh);
       if (cnt == 0u) *overflow = 1;
-      else b.observe(cnt, (unsigned)hot, a);
+      else if (VAR != V_LLP) b.observe(cnt, (unsigned)hot, a);
     }
   }
   unsigned h[N], k[N];
@@ -274,9 +290,11 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
       if (cnt[j] == 0u) *overflow = 1;
     }
   }
+  if (VAR != V_LLP) {
 #pragma unroll
-  for (int j = 0; j < N; ++j)
-    if (cnt[j]) b.observe(cnt[j], (unsigned)lab[j], a);
+    for (int j = 0; j < N; ++j)
+      if (cnt[j]) b.observe(cnt[j], (unsigned)lab[j], a);
+  }
   return nfresh;
 }
 
@@ -449,13 +467,18 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       const int sstart = 31 - __clz(segs & ((2u << lane) - 1u));
       // label frequency inside the vertex's lanes [P:231-232]
       unsigned k = 0;
+      bool first = true;  // LLP: only a label's first lane scores it (one V[l] gather per distinct label)
 #pragma unroll 4
-      for (int i = 0; i < d; ++i) k += __shfl_sync(kFull, lab, sstart + i) == lab ? 1u : 0u;
+      for (int i = 0; i < d; ++i) {
+        const bool eq = __shfl_sync(kFull, lab, sstart + i) == lab;
+        k += eq ? 1u : 0u;
+        if (VAR == V_LLP) first = first && !(eq && sstart + i < lane);
+      }
       const int head = (lane < nv ? lane * d : 0) & 31;  // lane jv takes segment jv
       Best<VAR> h;
       if (VAR == V_LLP || !GLP_LOW_REDUX) {
         Best<VAR> b;
-        if (vote) b.observe(k, (unsigned)lab, a);
+        if (vote && first) b.observe(k, (unsigned)lab, a);
         // segmented arg-max toward the segment head: ceil(log2 d) steps (d is
         // warp-uniform)
         const int send = sstart + d;
@@ -653,14 +676,14 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
             load_round(a.col, start, b2, d, v0, v1);
             const int m8[8] = {gather(a, v0.x), gather(a, v0.y), gather(a, v0.z), gather(a, v0.w),
                                gather(a, v1.x), gather(a, v1.y), gather(a, v1.z), gather(a, v1.w)};
-            fresh += warp_insert_n<VAR, 8>(a, tab, tsz, m8, b, &s_over[wid]);
+            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid]);
           }
         }
         if (d - off > 128) {  // warp-uniform
-          fresh += warp_insert_n<VAR, 8>(a, tab, tsz, l, b, &s_over[wid]);
+          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid]);
         } else {
           const int l4[4] = {l[0], l[1], l[2], l[3]};
-          fresh += warp_insert_n<VAR, 4>(a, tab, tsz, l4, b, &s_over[wid]);
+          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid]);
         }
         __syncwarp();
         over = s_over[wid] != 0;
@@ -669,6 +692,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
         if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = base + jl * nwarps + gw;
         if (!next_loaded) load_round(a.col, nstart, 0, nd, x0, x1);
       } else {
+        table_scan<VAR>(tab, lane, 32, a, b);  // LLP (s_over's __syncwarp ended the count)
         b.warp_reduce();
         fresh = __reduce_add_sync(kFull, fresh);
         if (lane == jl) {
@@ -980,10 +1004,11 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       tab.clear(threadIdx.x, BLOCK);
       __syncthreads();
       const bool may_over = PART && 2u * (unsigned)d > (unsigned)SLOTS;
-      block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : tsz, cur,
+      block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : (PART ? tsz : kTabProbe), cur,
                                       may_over ? stageA : nullptr, &s_over, &s_distinct, b);
       __syncthreads();
       over = s_over != 0;
+      if (!over) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
       __syncthreads();
       if (over && PART) {
         nparts = min(max(2u, ((unsigned)d + SLOTS / 2 - 1) / (SLOTS / 2)), 255u);
@@ -1064,6 +1089,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
           count_staged<VAR, BLOCK>(a, stageB + (end - cnt), cnt, tab, probe, &s_over, &s_distinct, b);
           __syncthreads();
           pover = s_over != 0;
+          if (!pover) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
           __syncthreads();
         }
         if (!pover) break;

@@ -96,8 +96,11 @@ def test_taobao100m_seeded_first_iterations():
 def rmat28():
     if os.environ.get("GLP_SKIP_R28") == "1":
         pytest.skip("GLP_SKIP_R28=1")
+    import gc
+    gc.collect()
+    torch.cuda.empty_cache()
     free, _ = torch.cuda.mem_get_info()
-    if free < 150e9:
+    if free < 130e9:
         pytest.skip("RMAT-28 needs ~120 GB of device memory")
     csr = graphs.rmat(28, seed=1, device="cuda", buckets=16)
     g = glp.Graph(csr)
