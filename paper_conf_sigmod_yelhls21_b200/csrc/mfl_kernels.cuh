@@ -158,6 +158,21 @@ struct Best {
   }
 };
 
+// Majority early exit (CLASSIC/SEEDED): a label observed with a count above
+// d/2 is the strict maximum of the row's final counts (any other label has at
+// most d - count < count votes), so it is the MFL whatever the unread arcs
+// hold, and min-label ties cannot arise.  Counts in the shared table are
+// row totals, so one lane's observation suffices.  Exact; saves reading the
+// rest of collapsed rows (labels concentrate as communities form [P:130]).
+#ifndef GLP_MAJORITY
+#define GLP_MAJORITY 1
+#endif
+template <int VAR>
+__device__ __forceinline__ bool strict_majority(const Best<VAR>& b, int d) {
+  const unsigned k = (unsigned)(b.key >> 32);
+  return __any_sync(kFull, 2ull * k > (unsigned long long)d);
+}
+
 __device__ __forceinline__ unsigned slot_hash(unsigned lab, unsigned tsz) {
   return __umulhi(lab * 0x9E3779B1u, tsz);
 }
@@ -642,7 +657,8 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       const bool tried = mono;
       int prev = -1;
       bool next_loaded = false;  // x0/x1 hold the next row's first round
-      for (int off = 0; off < d && !over; off += 256) {
+      bool major = false;        // a strict-majority label was observed: the rest of the row cannot change the MFL
+      for (int off = 0; off < d && !over && !major; off += 256) {
         int4 p0, p1;
         if (off + 256 < d) {
           load_round(a.col, start, off + 256, d, p0, p1);
@@ -687,10 +703,11 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
         }
         __syncwarp();
         over = s_over[wid] != 0;
+        if (GLP_MAJORITY && VAR != V_LLP && !over && off + 256 < d) major = strict_majority(b, d);
       }
+      if ((over || major) && !next_loaded) load_round(a.col, nstart, 0, nd, x0, x1);
       if (over) {
         if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = base + jl * nwarps + gw;
-        if (!next_loaded) load_round(a.col, nstart, 0, nd, x0, x1);
       } else {
         table_scan<VAR>(tab, lane, 32, a, b);  // LLP (s_over's __syncwarp ended the count)
         b.warp_reduce();
@@ -700,7 +717,8 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           rkey = b.key;
           rlab = b.lab;
           // a row that just took the sorted fast path is not retried next time
-          rpred = max(fresh, 1u) | (tried && mono ? kMonoTried : 0u);
+          // (a majority exit saw part of the row: keep the old prediction if larger)
+          rpred = max(major ? max(fresh, pred & kPredMask) : fresh, 1u) | (tried && mono ? kMonoTried : 0u);
         }
       }
       __syncwarp();
@@ -747,7 +765,8 @@ __device__ __forceinline__ void block_load_round(const int32_t* col, int64_t sta
 template <int VAR, int BLOCK, int UNROLL, bool IPF>
 __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int d, const Table& tab,
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
-                                            volatile int* overflow, int* distinct, Best<VAR>& b) {
+                                            volatile int* overflow, int* distinct, Best<VAR>& b,
+                                            volatile int* major) {
   constexpr int STEP = BLOCK * 4 * UNROLL;
   unsigned fresh = 0;
   for (int base = 0; base < d; base += STEP) {
@@ -770,6 +789,12 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
       for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
     }
     fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow);
+    if (GLP_MAJORITY && VAR != V_LLP && major != nullptr && base + STEP < d) {
+      // a strict-majority observation ends the row for every warp (they poll the flag)
+      const bool m = strict_majority(b, d);
+      if (m && (threadIdx.x & 31) == 0) *major = 1;
+      if (m || __any_sync(kFull, *major != 0)) break;
+    }
     if (__any_sync(kFull, *overflow != 0)) break;  // warp-uniform exit
   }
   fresh = __reduce_add_sync(kFull, fresh);
@@ -897,7 +922,7 @@ template <int VAR, int BLOCK, int SLOTS, bool PART, int UNROLL, int CLS>
 #endif
 __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_block(MflArgs a) {
   extern __shared__ __align__(16) unsigned long long smem_tab[];  // SLOTS
-  __shared__ int s_over, s_distinct;
+  __shared__ int s_over, s_distinct, s_major;
   __shared__ int s_hist[PART ? 256 : 1], s_cur[PART ? 256 : 1];
   Tally ty;
   int32_t* stageA = PART ? a.stage + (int64_t)blockIdx.x * 2 * a.stage_stride : nullptr;
@@ -968,7 +993,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     const unsigned pred = s_pe[q];
     const int d = it.d;
     Best<VAR> b;
-    if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; }
+    if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; s_major = 0; }
     bool mono_done = false;
     if (!a.mode && cand) {
       __syncthreads();
@@ -1005,7 +1030,8 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       __syncthreads();
       const bool may_over = PART && 2u * (unsigned)d > (unsigned)SLOTS;
       block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : (PART ? tsz : kTabProbe), cur,
-                                      may_over ? stageA : nullptr, &s_over, &s_distinct, b);
+                                      may_over ? stageA : nullptr, &s_over, &s_distinct, b,
+                                      may_over ? nullptr : &s_major);
       __syncthreads();
       over = s_over != 0;
       if (!over) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
@@ -1099,7 +1125,8 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     }  // !mono_done
     b = block_best<VAR, BLOCK>(b);
     if (threadIdx.x == 0) {
-      a.pred_next[i] = max((unsigned)s_distinct, 1u) | (mono_done ? kMonoTried : 0u);
+      const unsigned dist = s_major ? max((unsigned)s_distinct, pred) : (unsigned)s_distinct;  // partial on a majority exit
+      a.pred_next[i] = max(dist, 1u) | (mono_done ? kMonoTried : 0u);
       update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty);
     }
     __syncthreads();
