@@ -15,6 +15,8 @@
 #include <string.h>
 
 #include <algorithm>
+#include <array>
+#include <mutex>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -45,11 +47,53 @@ thread_local std::string g_last_error = "";
     }                                                                                      \
   } while (0)
 
+// Device memory comes from the device's stream-ordered memory pool
+// (cudaMallocAsync), which keeps up to kPoolKeep bytes of freed memory mapped
+// between graphs: create/destroy of a multi-GB graph then costs no driver
+// map/unmap (plain cudaMalloc/cudaFree made end-to-end create times vary from
+// 0.1 to 2 s on the B200 box).
+constexpr uint64_t kPoolKeep = 16ull << 30;
+cudaError_t pool_malloc(void** p, size_t bytes, cudaStream_t s) {
+  static std::mutex mu;
+  static std::vector<int> ready;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  {
+    std::lock_guard<std::mutex> lock(mu);
+    if (std::find(ready.begin(), ready.end(), dev) == ready.end()) {
+      cudaMemPool_t pool;
+      if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t keep = kPoolKeep;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+      }
+      ready.push_back(dev);
+    }
+  }
+  return cudaMallocAsync(p, bytes, s);
+}
+void pool_free(void* p, cudaStream_t s) {
+  if (p) cudaFreeAsync(p, s);
+}
+// thrust temporaries from the same pool
+struct PoolAlloc {
+  typedef char value_type;
+  cudaStream_t s;
+  char* allocate(std::ptrdiff_t n) {
+    void* p = nullptr;
+    if (pool_malloc(&p, std::max<std::ptrdiff_t>(n, 16), s) != cudaSuccess) {
+      cudaGetLastError();
+      throw std::bad_alloc();
+    }
+    return (char*)p;
+  }
+  void deallocate(char* p, size_t) { pool_free(p, s); }
+};
+
 template <class T>
 T* dalloc(glp_graph* g, size_t count) {
   void* p = nullptr;
   size_t bytes = std::max<size_t>(count * sizeof(T), 16);
-  cudaError_t e = cudaMalloc(&p, bytes);
+  cudaError_t e = pool_malloc(&p, bytes, g->stream);
   if (e != cudaSuccess) {
     cudaGetLastError();
     fail(GLP_ERR_OUT_OF_MEMORY, "cudaMalloc(" + std::to_string(bytes) + " B) failed: " + cudaGetErrorString(e));
@@ -115,17 +159,33 @@ void free_graph(glp_graph* g) {
   if (!g) return;
   if (g->device >= 0) cudaSetDevice(g->device);
   if (g->stream) cudaStreamSynchronize(g->stream);
-  for (void* p : g->allocs) cudaFree(p);
+  for (void* p : g->allocs) pool_free(p, g->stream);
+  if (g->stream) cudaStreamSynchronize(g->stream);
   g->allocs.clear();
   if (g->h_cnt) cudaFreeHost(g->h_cnt);
   if (g->ev_a) cudaEventDestroy(g->ev_a);
   if (g->ev_b) cudaEventDestroy(g->ev_b);
   for (auto& e : g->ev_pool) cudaEventDestroy(e);
   for (auto& e : g->xev) if (e) cudaEventDestroy(e);
-  for (auto& x : g->xs) if (x) cudaStreamDestroy(x);
   nccl_destroy(g);
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   delete g;
+}
+
+// Side streams of the concurrent class kernels: one set per device for the
+// process lifetime (stream creation/destruction per graph made graph create
+// and destroy times erratic).  Graphs on different threads may share them:
+// every graph forks and joins through its own events, so sharing only orders
+// their side-stream kernels, never breaks a dependency.
+void side_streams(int dev, cudaStream_t (&xs)[4]) {
+  static std::mutex mu;
+  static std::vector<std::array<cudaStream_t, 4>> pool;
+  std::lock_guard<std::mutex> lock(mu);
+  if ((int)pool.size() <= dev) pool.resize(dev + 1, std::array<cudaStream_t, 4>{nullptr, nullptr, nullptr, nullptr});
+  for (int i = 0; i < 4; ++i) {
+    if (!pool[dev][i]) CK(cudaStreamCreateWithFlags(&pool[dev][i], cudaStreamNonBlocking));
+    xs[i] = pool[dev][i];
+  }
 }
 
 // ---------------------------------------------------------------- layout
@@ -137,14 +197,15 @@ void free_graph(glp_graph* g) {
 // caller's CSR on the device (borrowed or staged).
 void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
   cudaStream_t s = g->stream;
-  auto pol = thrust::cuda::par.on(s);
+  PoolAlloc palloc{s};
+  auto pol = thrust::cuda::par(palloc).on(s);
   const int64_t nl = g->nl;
   std::vector<void*> tmp;
   auto talloc = [&](size_t bytes) {
     void* p = nullptr;
-    if (cudaMalloc(&p, std::max<size_t>(bytes, 16)) != cudaSuccess) {
+    if (pool_malloc(&p, std::max<size_t>(bytes, 16), s) != cudaSuccess) {
       cudaGetLastError();
-      for (void* q : tmp) cudaFree(q);
+      for (void* q : tmp) pool_free(q, s);
       fail(GLP_ERR_OUT_OF_MEMORY, "layout scratch allocation failed");
     }
     tmp.push_back(p);
@@ -154,8 +215,7 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     std::vector<void*>& v;
     cudaStream_t s;
     ~Free() {
-      cudaStreamSynchronize(s);
-      for (void* p : v) cudaFree(p);
+      for (void* p : v) pool_free(p, s);
     }
   } fr{tmp, s};
   int32_t* deg = (int32_t*)talloc(nl * sizeof(int32_t));
@@ -375,11 +435,11 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       col_d = csr->col_idx;
     } else {
       void *po = nullptr, *pc = nullptr;
-      if (cudaMalloc(&po, (g->nl + 1) * sizeof(int64_t)) != cudaSuccess ||
-          cudaMalloc(&pc, std::max<int64_t>(g->nnz, 1) * sizeof(int32_t)) != cudaSuccess) {
+      if (pool_malloc(&po, (g->nl + 1) * sizeof(int64_t), g->stream) != cudaSuccess ||
+          pool_malloc(&pc, std::max<int64_t>(g->nnz, 1) * sizeof(int32_t), g->stream) != cudaSuccess) {
         cudaGetLastError();
-        if (po) cudaFree(po);
-        if (pc) cudaFree(pc);
+        if (po) pool_free(po, g->stream);
+        if (pc) pool_free(pc, g->stream);
         fail(GLP_ERR_OUT_OF_MEMORY, "staging the CSR on the device failed");
       }
       temps.push_back(po);
@@ -395,8 +455,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       std::vector<void*>& v;
       cudaStream_t s;
       ~TempGuard() {
-        if (!v.empty()) cudaStreamSynchronize(s);
-        for (void* p : v) cudaFree(p);
+        for (void* p : v) pool_free(p, s);
       }
     } tg{temps, g->stream};
     // structural checks on the device: off[0] == 0, off[nl] == nnz, monotone
@@ -441,7 +500,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       const char* ser = getenv("GLP_SERIAL");
       g->concurrent = !(ser && ser[0] == '1');
     }
-    for (auto& x : g->xs) CK(cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking));
+    side_streams(dev, g->xs);
     for (auto& e : g->xev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
 
     const int sms = g->sms;
@@ -528,7 +587,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   // concurrently (filling each other's tails) unless profiling or GLP_SERIAL:
   // giant | L | M | low on their own streams, W -> redo M -> redo L on the
   // main stream (redo L also waits for the static M, which feeds its queue).
-  const bool cc = g->concurrent;
+  const bool cc = g->concurrent && !prof;  // profiled runs serialise: clean per-kernel durations
   cudaStream_t s0 = g->stream;
   bool used_x[4] = {false, false, false, false};
   auto S = [&](int i) -> cudaStream_t {
