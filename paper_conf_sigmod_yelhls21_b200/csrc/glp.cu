@@ -360,7 +360,14 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     nccl_exchange(g, g->pos);
     nccl_exchange(g, g->orig);
   }
-  // ---- the arcs themselves
+  // ---- the arcs themselves (copied and checked on the side stream)
+  CK(cudaStreamWaitEvent(s, g->xev[1], 0));
+  {
+    int bad = 0;
+    CK(cudaMemcpyAsync(&bad, g->col_bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (bad & 8) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
+  }
   g->col2 = dalloc<int32_t>(g, g->nnz2);
   CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), s));  // padding = -1
   if (nl > 0 && g->nnz > 0) {
@@ -427,6 +434,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     if (g->nnz >= ((int64_t)1 << 40)) fail(GLP_ERR_INVALID_ARGUMENT, "nnz_local too large");
 
     g->sms = prop.multiProcessorCount;
+    side_streams(dev, g->xs);
+    for (auto& e : g->xev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     const int64_t* off_d = nullptr;
     const int32_t* col_d = nullptr;
     std::vector<void*> temps;  // caller-CSR staging freed after the relayout
@@ -445,34 +454,43 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       temps.push_back(po);
       temps.push_back(pc);
       CK(cudaMemcpyAsync(po, csr->row_offsets, (g->nl + 1) * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
-      if (g->nnz)
-        CK(cudaMemcpyAsync(pc, csr->col_idx, g->nnz * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
       off_d = (const int64_t*)po;
       col_d = (const int32_t*)pc;
       g->own_csr = true;
     }
+    // The arcs (the bulk of a host CSR) are copied, and checked, on a side
+    // stream while the layout is derived from the offsets alone; the arc
+    // relayout waits for them (col_ready).
+    int* dbad = dalloc<int>(g, 2);
+    CK(cudaMemsetAsync(dbad, 0, 2 * sizeof(int), g->stream));
+    CK(cudaEventRecord(g->xev[0], g->stream));
+    CK(cudaStreamWaitEvent(g->xs[0], g->xev[0], 0));
+    if (!csr->on_device && g->nnz)
+      CK(cudaMemcpyAsync((void*)col_d, csr->col_idx, g->nnz * sizeof(int32_t), cudaMemcpyHostToDevice, g->xs[0]));
+    if (p.validate && g->nnz) k_validate_col<<<g->sms * 4, 256, 0, g->xs[0]>>>(col_d, g->nnz, g->n, dbad + 1);
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(g->xev[1], g->xs[0]));
     struct TempGuard {
       std::vector<void*>& v;
       cudaStream_t s;
+      cudaEvent_t col_ready;
       ~TempGuard() {
+        cudaStreamWaitEvent(s, col_ready, 0);  // the side-stream copy may still read the staging
         for (void* p : v) pool_free(p, s);
       }
-    } tg{temps, g->stream};
+    } tg{temps, g->stream, g->xev[1]};
     // structural checks on the device: off[0] == 0, off[nl] == nnz, monotone
-    // offsets (always); col in [0, n) (validate = 1)
+    // offsets (always); col in [0, n) (validate = 1, checked before the relayout)
     {
-      int* dbad = dalloc<int>(g, 1);
-      CK(cudaMemsetAsync(dbad, 0, sizeof(int), g->stream));
       k_validate_off<<<g->sms * 4, 256, 0, g->stream>>>(off_d, g->nl, g->nnz, dbad);
-      if (p.validate && g->nnz) k_validate_col<<<g->sms * 4, 256, 0, g->stream>>>(col_d, g->nnz, g->n, dbad);
       CK(cudaGetLastError());
       int bad = 0;
       CK(cudaMemcpyAsync(&bad, dbad, sizeof(int), cudaMemcpyDeviceToHost, g->stream));
       CK(cudaStreamSynchronize(g->stream));
       if (bad & 3) fail(GLP_ERR_INVALID_GRAPH, "row_offsets[0] must be 0 and row_offsets[last] == nnz_local");
       if (bad & 4) fail(GLP_ERR_INVALID_GRAPH, "row_offsets not non-decreasing");
-      if (bad & 8) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
     }
+    g->col_bad = dbad + 1;
     // labels: replicated full arrays, padded to a multiple of nranks for the
     // in-place all-gather
     const int64_t npad = ((n + nranks - 1) / nranks) * nranks;
@@ -500,8 +518,6 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       const char* ser = getenv("GLP_SERIAL");
       g->concurrent = !(ser && ser[0] == '1');
     }
-    side_streams(dev, g->xs);
-    for (auto& e : g->xev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
 
     const int sms = g->sms;
     const int ms_ = kMSlots * 8, ls_ = kLSlots * 8;

@@ -277,6 +277,7 @@ struct glp_graph {
   // concurrent class kernels within an iteration (GLP_SERIAL=1 disables):
   // xs[0] giant, xs[1] L, xs[2] M, xs[3] low; W and the redo chain on `stream`
   bool concurrent = true;
+  int* col_bad = nullptr;  // create: col_idx range check flag (side stream)
   cudaStream_t xs[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaEvent_t xev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
   std::vector<cudaEvent_t> ev_pool;
