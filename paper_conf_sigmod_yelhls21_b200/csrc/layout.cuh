@@ -47,15 +47,41 @@ struct LayoutStats {
 
 __global__ void k_degree_stats(const int64_t* __restrict__ off, int64_t nl, int32_t* __restrict__ deg,
                                LayoutStats* st) {
+  // per-thread sums, then shared-memory totals, then one global atomic per
+  // counter per block (per-vertex global atomics on a handful of addresses
+  // serialised this kernel: 23 ms at RMAT-24)
+  __shared__ unsigned long long s_verts[NBINS], s_arcs[NBINS], s_max, s_hist[kLowMax + 1];
+  for (int i = threadIdx.x; i < NBINS; i += blockDim.x) { s_verts[i] = 0ull; s_arcs[i] = 0ull; }
+  for (int i = threadIdx.x; i <= kLowMax; i += blockDim.x) s_hist[i] = 0ull;
+  if (threadIdx.x == 0) s_max = 0ull;
+  __syncthreads();
+  unsigned long long verts[NBINS] = {0ull}, arcs[NBINS] = {0ull}, mx = 0ull;
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nl; v += (int64_t)gridDim.x * blockDim.x) {
     const int64_t d = off[v + 1] - off[v];
     deg[v] = (int32_t)min(d, (int64_t)0x7fffffff);
     const int b = d == 0 ? BIN_ISO : d <= kLowMax ? BIN_LOW : d <= 256 ? BIN_MID : d <= 2048 ? BIN_HIGH : BIN_HUGE;
-    atomicAdd(&st->verts[b], 1ull);
-    atomicAdd(&st->arcs[b], (unsigned long long)d);
-    atomicMax(&st->max_deg, (unsigned long long)d);
-    if (d >= 1 && d <= kLowMax) atomicAdd(&st->low_hist[d], 1ull);
+#pragma unroll
+    for (int i = 0; i < NBINS; ++i) {
+      verts[i] += (b == i) ? 1ull : 0ull;
+      arcs[i] += (b == i) ? (unsigned long long)d : 0ull;
+    }
+    mx = max(mx, (unsigned long long)d);
+    if (d >= 1 && d <= kLowMax) atomicAdd(&s_hist[d], 1ull);
   }
+#pragma unroll
+  for (int i = 0; i < NBINS; ++i) {
+    if (verts[i]) atomicAdd(&s_verts[i], verts[i]);
+    if (arcs[i]) atomicAdd(&s_arcs[i], arcs[i]);
+  }
+  if (mx) atomicMax(&s_max, mx);
+  __syncthreads();
+  for (int i = threadIdx.x; i < NBINS; i += blockDim.x) {
+    if (s_verts[i]) atomicAdd(&st->verts[i], s_verts[i]);
+    if (s_arcs[i]) atomicAdd(&st->arcs[i], s_arcs[i]);
+  }
+  for (int i = threadIdx.x; i <= kLowMax; i += blockDim.x)
+    if (s_hist[i]) atomicAdd(&st->low_hist[i], s_hist[i]);
+  if (threadIdx.x == 0 && s_max) atomicMax(&st->max_deg, s_max);
 }
 
 struct IsLow {
