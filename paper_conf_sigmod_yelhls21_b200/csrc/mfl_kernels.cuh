@@ -571,8 +571,10 @@ __device__ __forceinline__ bool warp_quads_increasing(const int (&x)[4], int bas
 
 // ---------------------------------------------------------------------------
 // mfl_warp: one warp per row of class W (few distinct labels): per-warp shared
-// table of pow2 >= 2*pred slots (<= 512), two 128-bit loads per lane per
-// round (256 arcs per warp), no block barriers.  Rows whose labels overflow the
+// table of pow2 >= 4*pred slots (<= 512), one 128-bit load per lane per
+// round (128 arcs per warp; 256-arc rounds measured 2 % slower: most W rows
+// have < 128 arcs, and the smaller round frees registers for a 4th block per
+// SM), no block barriers.  Rows whose labels overflow the
 // table are re-queued to the block kernel M.
 //   * 32 rows per warp at a time: the class / frontier test of the batch is
 //     lane-parallel; rows are degree-sorted, so a warp's batch is strided
@@ -582,17 +584,21 @@ __device__ __forceinline__ bool warp_quads_increasing(const int (&x)[4], int bas
 //     round is gathered and counted;
 //   * lane j keeps the result of batch row j, and the batch's vertices are
 //     updated lane-parallel at the end.
+#ifndef GLP_W_ROUND
+#define GLP_W_ROUND 128
+#endif
+constexpr int kWRound = GLP_W_ROUND;  // arcs per warp round: 256 (two 128-bit loads per lane) or 128
 __device__ __forceinline__ void load_round(const int32_t* col, int64_t start, int off, int d, int4& u0, int4& u1) {
   const int lane = threadIdx.x & 31;
   u0 = make_int4(-1, -1, -1, -1);
   u1 = u0;
   if (off + 4 * lane < d) u0 = ld_stream4(col + start + off + 4 * lane);
-  if (off + 128 + 4 * lane < d) u1 = ld_stream4(col + start + off + 128 + 4 * lane);
+  if (kWRound == 256 && off + 128 + 4 * lane < d) u1 = ld_stream4(col + start + off + 128 + 4 * lane);
 }
 
 template <int VAR>
 #ifndef GLP_W_MINB
-#define GLP_W_MINB 3
+#define GLP_W_MINB 4
 #endif
 __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
   extern __shared__ __align__(16) unsigned long long wtabs[];  // [kWBlock / 32][kWSlots] (dynamic)
@@ -658,24 +664,29 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       int prev = -1;
       bool next_loaded = false;  // x0/x1 hold the next row's first round
       bool major = false;        // a strict-majority label was observed: the rest of the row cannot change the MFL
-      for (int off = 0; off < d && !over && !major; off += 256) {
+      for (int off = 0; off < d && !over && !major; off += kWRound) {
         int4 p0, p1;
-        if (off + 256 < d) {
-          load_round(a.col, start, off + 256, d, p0, p1);
+        if (off + kWRound < d) {
+          load_round(a.col, start, off + kWRound, d, p0, p1);
         } else {
           load_round(a.col, nstart, 0, nd, p0, p1);  // nd == 0: no loads
           next_loaded = true;
         }
         int l[8];
         l[0] = gather(a, x0.x); l[1] = gather(a, x0.y); l[2] = gather(a, x0.z); l[3] = gather(a, x0.w);
-        l[4] = gather(a, x1.x); l[5] = gather(a, x1.y); l[6] = gather(a, x1.z); l[7] = gather(a, x1.w);
+        if (kWRound == 256) {
+          l[4] = gather(a, x1.x); l[5] = gather(a, x1.y); l[6] = gather(a, x1.z); l[7] = gather(a, x1.w);
+        } else {
+          l[4] = l[5] = l[6] = l[7] = -1;
+        }
         x0 = p0;
         x1 = p1;
         if (mono) {
           const int q0[4] = {l[0], l[1], l[2], l[3]}, q1[4] = {l[4], l[5], l[6], l[7]};
           int mid = -1, end = -1;
           bool okm = warp_quads_increasing(q0, off, d, prev, &mid);
-          okm = okm && warp_quads_increasing(q1, off + 128, d, mid, &end);
+          if (kWRound == 256) okm = okm && warp_quads_increasing(q1, off + 128, d, mid, &end);
+          else end = mid;
           if (okm) {  // every label of this round occurs once in the row so far
 #pragma unroll
             for (int j = 0; j < 8; ++j)
@@ -687,7 +698,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           // already observed (their count-1 observations stay valid lower bounds)
           mono = false;
           fresh = 0;
-          for (int b2 = 0; b2 < off; b2 += 256) {
+          for (int b2 = 0; b2 < off; b2 += kWRound) {
             int4 v0, v1;
             load_round(a.col, start, b2, d, v0, v1);
             const int m8[8] = {gather(a, v0.x), gather(a, v0.y), gather(a, v0.z), gather(a, v0.w),
@@ -695,7 +706,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
             fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid]);
           }
         }
-        if (d - off > 128) {  // warp-uniform
+        if (kWRound == 256 && d - off > 128) {  // warp-uniform
           fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid]);
         } else {
           const int l4[4] = {l[0], l[1], l[2], l[3]};
@@ -703,7 +714,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
         }
         __syncwarp();
         over = s_over[wid] != 0;
-        if (GLP_MAJORITY && VAR != V_LLP && !over && off + 256 < d) major = strict_majority(b, d);
+        if (GLP_MAJORITY && VAR != V_LLP && !over && off + kWRound < d) major = strict_majority(b, d);
       }
       if ((over || major) && !next_loaded) load_round(a.col, nstart, 0, nd, x0, x1);
       if (over) {
