@@ -72,6 +72,9 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_M_LOAD
 #define GLP_M_LOAD 4
 #endif
+#ifndef GLP_ADD_ALWAYS
+#define GLP_ADD_ALWAYS 1
+#endif
 #ifndef GLP_W_LOAD
 #define GLP_W_LOAD 4
 #endif
@@ -228,7 +231,15 @@ __device__ __forceinline__ unsigned slot_try(const Table& t, unsigned h, unsigne
     *fresh += p == kFree ? 1u : 0u;
     k = p == kFree ? l : p;
   }
+#if GLP_ADD_ALWAYS
+  // the add is issued by every lane (a lane whose slot holds another label
+  // adds 0): one divergent region less per label
+  const bool hit = k == l;
+  const unsigned old = atomicAdd(t.cnt + h, hit ? c : 0u);
+  return hit ? old + c : 0u;
+#else
   return k == l ? atomicAdd(t.cnt + h, c) + c : 0u;
+#endif
 }
 
 // Probe from slot h + 1 on (the home slot h held another label).  Returns the
