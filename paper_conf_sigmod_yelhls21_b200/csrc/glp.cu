@@ -816,6 +816,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     a.V = g->V; a.is_seed = g->is_seed; a.flag = g->flag[fb];
     a.vb = g->vb; a.gamma = p.gamma; a.t = t; a.dense = dense ? 1 : 0;
     a.pred_cap = p.debug_pred_cap > 0 ? (unsigned)p.debug_pred_cap : 0u;
+    // L_0 = PickLabel's identity labelling (a permutation): its histogram V is
+    // all ones (k_hist still writes it), so t = 1 needs no V gathers
+    a.v_ones = (variant == GLP_VARIANT_LLP && t == 1) ? 1 : 0;
     switch (variant) {
       case GLP_VARIANT_CLASSIC: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;

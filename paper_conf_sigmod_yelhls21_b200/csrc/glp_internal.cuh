@@ -184,6 +184,7 @@ struct MflArgs {
   double gamma;
   int32_t t;                            // iteration number (1-based)
   int32_t dense;                        // 1: process every listed vertex
+  int32_t v_ones;                       // LLP: V[l] == 1 for every l (L_{t-1} is PickLabel's permutation)
 };
 
 // Internal error: thrown inside the library, converted to glp_status at the ABI.

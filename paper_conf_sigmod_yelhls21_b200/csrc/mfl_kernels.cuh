@@ -135,7 +135,8 @@ struct Best {
   unsigned lab = kNoLabel;
   __device__ __forceinline__ void observe(unsigned cnt, unsigned l, const MflArgs& a) {
     if (VAR == V_LLP) {
-      const unsigned long long k = dkey(llp_score(cnt, ld_label(a.V + l), a.gamma));
+      const int vl = a.v_ones ? 1 : ld_label(a.V + l);  // V of a permutation labelling is all ones (t = 1)
+      const unsigned long long k = dkey(llp_score(cnt, vl, a.gamma));
       if (k > key || (k == key && l < lab)) { key = k; lab = l; }
     } else {
       const unsigned long long k = ((unsigned long long)cnt << 32) | (unsigned long long)(~l);

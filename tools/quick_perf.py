@@ -8,12 +8,12 @@ import os
 VAR = os.environ.get('GLP_VARIANT', 'classic')
 GAMMA = float(os.environ.get('GLP_GAMMA', '1.0' if VAR == 'llp' else '0'))
 t0 = time.time()
-csr = graphs.rmat(scale, seed=1, device='cuda')
+csr = graphs.rmat(scale, seed=1, device='cuda', buckets=16 if scale >= 27 else 0)
 torch.cuda.synchronize()
 print('gen', scale, csr.nnz, round(time.time() - t0, 2), 's', flush=True)
 g = glp.Graph(csr)
 print(json.dumps(g.info()), flush=True)
-for rep in range(3):
+for rep in range(int(os.environ.get('GLP_REPS', '3'))):
     info = g.run(VAR, 20, gamma=GAMMA, profile=(rep == 2))
     print(info, flush=True)
 for s in g.iter_stats():
