@@ -250,14 +250,28 @@ def bench_gpu(args):
                 traffic = json.load(open(tfile)).get(args.workload, {}).get(dom)
             except (OSError, ValueError):
                 traffic = None
+        gceil = None
+        gfile = os.path.join(ROOT, "profiles", "gather_ceilings.json")
+        if os.path.exists(gfile):
+            try:
+                gceil = json.load(open(gfile)).get(args.workload)
+            except (OSError, ValueError):
+                gceil = None
+        gath = s["arcs"] / (s["ms"] / 1e3) / 1e9  # one label gather per arc
         roof = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
                 "bytes_per_launch": s["bytes"] / s["launches"], "ms_per_launch": s["ms"] / s["launches"],
                 "share_of_step": round(s["ms"] / sum(prof_ms), 3) if world == 1 else None,
+                # the ceiling that actually binds: one random 4-B label gather per
+                # arc costs a 32-B sector, measured by tools/ubench.py
+                "gather_ceiling": {"achieved": round(gath, 1), "peak": gceil, "unit": "G label gathers/s",
+                                   "frac": round(gath / gceil, 4) if gceil else None,
+                                   "source": "profiles/gather_ceilings.json"},
                 "kernel_timing": f"{kprof_steps} profiled steps with the class kernels serialised (CUDA events per "
                                  f"launch; {sum(prof_ms) / kprof_steps:.3f} ms/step serialised vs the timed region's "
                                  f"concurrent steps)",
                 "kernels": {k: {"ms": round(v["ms"] / kprof_steps, 4), "launches": v["launches"] // kprof_steps,
+                                "Garcs_s": round(v["arcs"] / max(v["ms"], 1e-9) / 1e6, 1),
                                 "GBps_alg": round(v["bytes"] / max(v["ms"], 1e-9) / 1e6, 1)}
                             for k, v in kstats.items() if v["launches"]}}
 

@@ -46,7 +46,14 @@ constexpr int kLowBlock = 256;
 #define GLP_WSLOTS 512
 #endif
 constexpr unsigned kWPred = GLP_WPRED, kMPred = 2048;
-constexpr int kWMaxDeg = 4096, kMMaxDeg = 16384;
+#ifndef GLP_MMAXDEG
+#define GLP_MMAXDEG 16384
+#endif
+constexpr int kWMaxDeg = 4096, kMMaxDeg = GLP_MMAXDEG;
+#ifndef GLP_MONO_WMAX
+#define GLP_MONO_WMAX 65536
+#endif
+constexpr int kMonoWMax = GLP_MONO_WMAX;  // sorted-row candidates longer than this use the block path (L)
 constexpr int kWBlock = 256;
 constexpr int kWSlots = GLP_WSLOTS;
 constexpr int kMBlock = 128;
@@ -93,7 +100,7 @@ constexpr unsigned kPredMask = 0x7fffffffu, kMonoTried = 0x80000000u;
 // it goes to the barrier-free warp kernel whatever its size.
 __host__ __device__ __forceinline__ int row_class(unsigned pred, int d, bool mono) {
   if (d > kGiantMin) return CLS_G;
-  if (mono) return CLS_W;
+  if (mono) return d > kMonoWMax ? CLS_L : CLS_W;
   if (pred <= kWPred && d <= kWMaxDeg) return CLS_W;
   if (pred <= kMPred && d <= kMMaxDeg) return CLS_M;
   return CLS_L;
