@@ -71,3 +71,14 @@ def test_cuda_generation_matches_cpu():
                lambda d: graphs.sbm(n=5000, k=50, m=40000, device=d),
                lambda d: graphs.taobao(users=4000, items=1000, pairs=20000, rings=10, device=d)[0]]:
         assert mk("cpu").sha256() == mk("cuda").sha256()
+
+
+def test_rmat_bucketed_build_matches_plain():
+    """The memory-bounded RMAT-28 builder (row buckets) yields the same CSR."""
+    from glp_inputs import graphs
+    for scale in (9, 12):
+        a = graphs.rmat(scale, seed=1)
+        for buckets in (2, 5, 16):
+            b = graphs.rmat(scale, seed=1, buckets=buckets)
+            assert torch.equal(a.row_offsets, b.row_offsets)
+            assert torch.equal(a.col_idx, b.col_idx)
