@@ -48,7 +48,7 @@ thread_local std::string g_last_error = "";
   } while (0)
 
 // Device memory comes from the device's stream-ordered memory pool
-// (cudaMallocAsync), which keeps up to kPoolKeep bytes of freed memory mapped
+// (cudaMallocAsync), which keeps up to kPoolKeep bytes (env GLP_POOL_KEEP_GB) of freed memory mapped
 // between graphs: create/destroy of a multi-GB graph then costs no driver
 // map/unmap (plain cudaMalloc/cudaFree made end-to-end create times vary from
 // 0.1 to 2 s on the B200 box).
@@ -64,6 +64,7 @@ cudaError_t pool_malloc(void** p, size_t bytes, cudaStream_t s) {
       cudaMemPool_t pool;
       if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
         uint64_t keep = kPoolKeep;
+        if (const char* e = getenv("GLP_POOL_KEEP_GB")) keep = (uint64_t)(atof(e) * (double)(1ull << 30));
         cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
       }
       ready.push_back(dev);

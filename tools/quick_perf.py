@@ -8,7 +8,10 @@ import os
 VAR = os.environ.get('GLP_VARIANT', 'classic')
 GAMMA = float(os.environ.get('GLP_GAMMA', '1.0' if VAR == 'llp' else '0'))
 t0 = time.time()
-csr = graphs.rmat(scale, seed=1, device='cuda', buckets=16 if scale >= 27 else 0)
+if os.environ.get('GLP_GRAPH'):
+    csr, _seeds = graphs.make(os.environ['GLP_GRAPH'], device='cuda')
+else:
+    csr = graphs.rmat(scale, seed=1, device='cuda', buckets=16 if scale >= 27 else 0)
 torch.cuda.synchronize()
 print('gen', scale, csr.nnz, round(time.time() - t0, 2), 's', flush=True)
 g = glp.Graph(csr)
