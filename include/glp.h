@@ -81,7 +81,10 @@ typedef struct {
   const int32_t *col_idx;      /* nnz_local entries in [0, n_global); a row
                                   may list a neighbour twice (two votes, R3)   */
   int32_t on_device;           /* 1: device pointers, BORROWED for the graph's
-                                     lifetime (e.g. torch tensors);
+                                     lifetime (e.g. torch tensors); their
+                                     contents must be complete when create is
+                                     called, or be produced on the stream
+                                     passed in glp_dist.cuda_stream;
                                   0: host pointers, copied during create       */
   int32_t symmetric;           /* 1: caller asserts the global graph is
                                   symmetric (u in N(v) <=> v in N(u)); the

@@ -191,6 +191,10 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
             uid_buf = (ctypes.c_uint8 * 128).from_buffer_copy(nccl_unique_id)
             d.nccl_unique_id = ctypes.cast(uid_buf, ctypes.c_void_p)
         d.cuda_stream = stream.cuda_stream if stream is not None else None
+    if on_device and stream is None:
+        # borrowed tensors are read on the library's own stream: they must be
+        # complete (torch may still be producing them on its current stream)
+        torch.cuda.current_stream(row_offsets.device).synchronize()
     h = ctypes.c_void_p()
     prm = make_params(validate=validate)
     st = lib.glp_graph_create(ctypes.byref(c), None if d is None else ctypes.byref(d), ctypes.byref(prm),
