@@ -518,6 +518,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     {
       const char* ser = getenv("GLP_SERIAL");
       g->concurrent = !(ser && ser[0] == '1');
+      const char* novl = getenv("GLP_NO_VL");
+      g->use_vl = !(novl && novl[0] == '1');
     }
 
     const int sms = g->sms;
@@ -735,6 +737,11 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
     k_hist<<<ga, 256, 0, s>>>(g->L[0], g->n, g->V);
     g->init_launches += 1;
+    if (g->use_vl) {
+      if (!g->VL) g->VL = dalloc<int32_t>(g, std::max<int64_t>(g->n, 1));
+      k_vl<<<ga, 256, 0, s>>>(g->L[0], g->V, g->n, g->VL);
+      g->init_launches += 1;
+    }
     CK(cudaGetLastError());
   }
   if (g->n_rows) {
@@ -820,6 +827,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     // L_0 = PickLabel's identity labelling (a permutation): its histogram V is
     // all ones (k_hist still writes it), so t = 1 needs no V gathers
     a.v_ones = (variant == GLP_VARIANT_LLP && t == 1) ? 1 : 0;
+    a.VL = (variant == GLP_VARIANT_LLP && g->use_vl) ? g->VL : nullptr;
     switch (variant) {
       case GLP_VARIANT_CLASSIC: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
@@ -884,7 +892,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       timed(g, prof, 5, pend, used, s, [&] {
         CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
         k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb], g->n, g->V);
+        if (g->use_vl) k_vl<<<ga, 256, 0, s>>>(g->L[1 - rb], g->V, g->n, g->VL);
       });
+      launches += g->use_vl ? 1 : 0;
     }
     g->iter_stats.push_back(st);
     g->pb = (g->pb + 1) % 3;

@@ -113,6 +113,11 @@ __device__ __forceinline__ int ld_label(const int32_t* p) {
 }
 __device__ __forceinline__ int gather(const MflArgs& a, int u) { return u >= 0 ? ld_label(a.R + u) : -1; }
 
+// LLP: V[L_{t-1}[u]] carried next to the label of u (a.VL, computed once per
+// vertex after the histogram): gathered at the same index as the label, so a
+// candidate's V arrives with it instead of a random V[l] gather per label.
+__device__ __forceinline__ int gather_v(const MflArgs& a, int u) { return u >= 0 ? ld_label(a.VL + u) : -1; }
+
 // LLP score val = k - gamma * (v - k) [P:119], double, no contraction (R11).
 __device__ __forceinline__ double llp_score(unsigned k, int v, double gamma) {
   double kd = (double)k;
@@ -133,11 +138,14 @@ template <int VAR>
 struct Best {
   unsigned long long key = 0ull;
   unsigned lab = kNoLabel;
-  __device__ __forceinline__ void observe(unsigned cnt, unsigned l, const MflArgs& a) {
+  int bv = -1;  // LLP: V of the best label
+  // vl: V[l] when the caller has it (carried with the label, a.VL), else -1
+  __device__ __forceinline__ void observe(unsigned cnt, unsigned l, const MflArgs& a, int vl = -1) {
     if (VAR == V_LLP) {
-      const int vl = a.v_ones ? 1 : ld_label(a.V + l);  // V of a permutation labelling is all ones (t = 1)
-      const unsigned long long k = dkey(llp_score(cnt, vl, a.gamma));
-      if (k > key || (k == key && l < lab)) { key = k; lab = l; }
+      // V of a permutation labelling is all ones (t = 1)
+      const int v = vl >= 0 ? vl : (a.v_ones ? 1 : ld_label(a.V + l));
+      const unsigned long long k = dkey(llp_score(cnt, v, a.gamma));
+      if (k > key || (k == key && l < lab)) { key = k; lab = l; bv = v; }
     } else {
       const unsigned long long k = ((unsigned long long)cnt << 32) | (unsigned long long)(~l);
       key = k > key ? k : key;
@@ -277,16 +285,25 @@ __device__ __forceinline__ unsigned ht_add(const Table& t, unsigned lab, unsigne
 // claimed slots.
 template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
-                                                  const int (&labin)[N], Best<VAR>& b, volatile int* overflow) {
+                                                  const int (&labin)[N], Best<VAR>& b, volatile int* overflow,
+                                                  const int (&vin)[N], bool use_v) {
+  // use_v (LLP with a.VL): labels carry their V, so LLP observes at insert
+  // like CLASSIC; otherwise LLP scores from the final table (table_scan)
+  const bool obs = VAR != V_LLP || use_v;
   const int lane = threadIdx.x & 31;
   int lab[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) lab[j] = labin[j];
   unsigned nfresh = 0;
   int cand = b.have() ? (int)b.label() : -1;
+  int candv = b.have() ? b.bv : -1;
 #pragma unroll
-  for (int j = N - 1; j >= 0; --j) cand = (cand < 0 && lab[j] >= 0) ? lab[j] : cand;
+  for (int j = N - 1; j >= 0; --j) {
+    candv = (cand < 0 && lab[j] >= 0) ? (use_v ? vin[j] : -1) : candv;
+    cand = (cand < 0 && lab[j] >= 0) ? lab[j] : cand;
+  }
   const int hot = __shfl_sync(kFull, cand, 0);
+  const int hotv = __shfl_sync(kFull, candv, 0);
   if (hot >= 0) {  // warp-uniform
     unsigned hc = 0;
 #pragma unroll
@@ -298,7 +315,7 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
     if (lane == 0 && tot) {
       const unsigned cnt = ht_add(t, (unsigned)hot, tot, max_probe, &nfresh);
       if (cnt == 0u) *overflow = 1;
-      else if (VAR != V_LLP) b.observe(cnt, (unsigned)hot, a);
+      else if (obs) b.observe(cnt, (unsigned)hot, a, hotv);
     }
   }
   unsigned h[N], k[N];
@@ -317,10 +334,10 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
       if (cnt[j] == 0u) *overflow = 1;
     }
   }
-  if (VAR != V_LLP) {
+  if (obs) {
 #pragma unroll
     for (int j = 0; j < N; ++j)
-      if (cnt[j]) b.observe(cnt[j], (unsigned)lab[j], a);
+      if (cnt[j]) b.observe(cnt[j], (unsigned)lab[j], a, use_v ? vin[j] : -1);
   }
   return nfresh;
 }
@@ -482,6 +499,7 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       // every vertex of the chunk has degree d; nv vertices, lanes [0, total)
       const int nv = __popc(segs);
       int lab = gather(a, u);
+      const int lv = (VAR == V_LLP && a.VL != nullptr) ? gather_v(a, u) : -1;
       int r = 0;
       int2 so = make_int2(0, 0);
       if (lane < nv) {
@@ -505,7 +523,7 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       Best<VAR> h;
       if (VAR == V_LLP || !GLP_LOW_REDUX) {
         Best<VAR> b;
-        if (vote && first) b.observe(k, (unsigned)lab, a);
+        if (vote && first) b.observe(k, (unsigned)lab, a, lv);
         // segmented arg-max toward the segment head: ceil(log2 d) steps (d is
         // warp-uniform)
         const int send = sstart + d;
@@ -684,8 +702,12 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           load_round(a.col, nstart, 0, nd, p0, p1);  // nd == 0: no loads
           next_loaded = true;
         }
-        int l[8];
+        int l[8], lv[8];
         l[0] = gather(a, x0.x); l[1] = gather(a, x0.y); l[2] = gather(a, x0.z); l[3] = gather(a, x0.w);
+        const bool use_v = VAR == V_LLP && a.VL != nullptr;
+        lv[0] = use_v ? gather_v(a, x0.x) : -1; lv[1] = use_v ? gather_v(a, x0.y) : -1;
+        lv[2] = use_v ? gather_v(a, x0.z) : -1; lv[3] = use_v ? gather_v(a, x0.w) : -1;
+        lv[4] = lv[5] = lv[6] = lv[7] = -1;
         if (kWRound == 256) {
           l[4] = gather(a, x1.x); l[5] = gather(a, x1.y); l[6] = gather(a, x1.z); l[7] = gather(a, x1.w);
         } else {
@@ -702,7 +724,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           if (okm) {  // every label of this round occurs once in the row so far
 #pragma unroll
             for (int j = 0; j < 8; ++j)
-              if (l[j] >= 0) { b.observe(1u, (unsigned)l[j], a); ++fresh; }
+              if (l[j] >= 0) { b.observe(1u, (unsigned)l[j], a, lv[j]); ++fresh; }
             prev = end;
             continue;
           }
@@ -715,14 +737,19 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
             load_round(a.col, start, b2, d, v0, v1);
             const int m8[8] = {gather(a, v0.x), gather(a, v0.y), gather(a, v0.z), gather(a, v0.w),
                                gather(a, v1.x), gather(a, v1.y), gather(a, v1.z), gather(a, v1.w)};
-            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid]);
+            const int mv8[8] = {use_v ? gather_v(a, v0.x) : -1, use_v ? gather_v(a, v0.y) : -1,
+                                use_v ? gather_v(a, v0.z) : -1, use_v ? gather_v(a, v0.w) : -1,
+                                use_v ? gather_v(a, v1.x) : -1, use_v ? gather_v(a, v1.y) : -1,
+                                use_v ? gather_v(a, v1.z) : -1, use_v ? gather_v(a, v1.w) : -1};
+            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v);
           }
         }
         if (kWRound == 256 && d - off > 128) {  // warp-uniform
-          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid]);
+          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v);
         } else {
           const int l4[4] = {l[0], l[1], l[2], l[3]};
-          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid]);
+          const int v4[4] = {lv[0], lv[1], lv[2], lv[3]};
+          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v);
         }
         __syncwarp();
         over = s_over[wid] != 0;
@@ -732,7 +759,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       if (over) {
         if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = base + jl * nwarps + gw;
       } else {
-        table_scan<VAR>(tab, lane, 32, a, b);  // LLP (s_over's __syncwarp ended the count)
+        if (a.VL == nullptr) table_scan<VAR>(tab, lane, 32, a, b);  // LLP (s_over's __syncwarp ended the count)
         b.warp_reduce();
         fresh = __reduce_add_sync(kFull, fresh);
         if (lane == jl) {
@@ -796,13 +823,18 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
     int4 un[UNROLL];
     if (!IPF && base > 0) block_load_round<BLOCK, UNROLL>(a.col, start, d, base, u);
     if (IPF) block_load_round<BLOCK, UNROLL>(a.col, start, d, base + STEP, un);
-    int lab[4 * UNROLL];
+    int lab[4 * UNROLL], lv[4 * UNROLL];
+    const bool use_v = VAR == V_LLP && a.VL != nullptr;
 #pragma unroll
     for (int j = 0; j < UNROLL; ++j) {
       lab[4 * j + 0] = gather(a, u[j].x);
       lab[4 * j + 1] = gather(a, u[j].y);
       lab[4 * j + 2] = gather(a, u[j].z);
       lab[4 * j + 3] = gather(a, u[j].w);
+      lv[4 * j + 0] = use_v ? gather_v(a, u[j].x) : -1;
+      lv[4 * j + 1] = use_v ? gather_v(a, u[j].y) : -1;
+      lv[4 * j + 2] = use_v ? gather_v(a, u[j].z) : -1;
+      lv[4 * j + 3] = use_v ? gather_v(a, u[j].w) : -1;
       const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
       if (stage_out != nullptr && idx < d)
         __stcg((int4*)(stage_out + idx), make_int4(lab[4 * j], lab[4 * j + 1], lab[4 * j + 2], lab[4 * j + 3]));
@@ -811,7 +843,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
     }
-    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow);
+    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v);
     if (GLP_MAJORITY && VAR != V_LLP && major != nullptr && base + STEP < d) {
       // a strict-majority observation ends the row for every warp (they poll the flag)
       const bool m = strict_majority(b, d);
@@ -878,7 +910,7 @@ __device__ __forceinline__ bool block_mono(const MflArgs& a, int64_t start, int 
       const int wb = base + j * 4 * BLOCK + 128 * wid;
 #pragma unroll
       for (int k = 0; k < 4; ++k)
-        if (wb + 4 * lane + k < d) { b.observe(1u, (unsigned)x[j][k], a); ++*fresh; }
+        if (wb + 4 * lane + k < d) { b.observe(1u, (unsigned)x[j][k], a); ++*fresh; }  // (V gathered: t = 1 has v_ones)
     }
   }
   return true;
@@ -915,7 +947,8 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
       const int j = j0 + k * BLOCK + (int)threadIdx.x;
       lab[k] = j < cnt ? __ldcg(stage + j) : -1;
     }
-    fresh += warp_insert_n<VAR, 4>(a, tab, max_probe, lab, b, overflow);
+    const int nov[4] = {-1, -1, -1, -1};
+    fresh += warp_insert_n<VAR, 4>(a, tab, max_probe, lab, b, overflow, nov, false);
     if (__any_sync(kFull, *overflow != 0)) break;
   }
   fresh = __reduce_add_sync(kFull, fresh);
@@ -1057,7 +1090,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
                                       may_over ? nullptr : &s_major);
       __syncthreads();
       over = s_over != 0;
-      if (!over) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
+      if (!over && a.VL == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
       __syncthreads();
       if (over && PART) {
         nparts = min(max(2u, ((unsigned)d + SLOTS / 2 - 1) / (SLOTS / 2)), 255u);
@@ -1210,7 +1243,7 @@ __global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
     Best<VAR> b;
     unsigned fresh = 0;
     for (int base = sg.begin; base < end; base += kGBlock * 4 * kGUnroll) {
-      int lab[4 * kGUnroll];
+      int lab[4 * kGUnroll], gv[4 * kGUnroll];
 #pragma unroll
       for (int j = 0; j < kGUnroll; ++j) {
         const int idx = base + (j * kGBlock + (int)threadIdx.x) * 4;
@@ -1219,6 +1252,11 @@ __global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
         lab[4 * j + 1] = gather(a, u.y);
         lab[4 * j + 2] = gather(a, u.z);
         lab[4 * j + 3] = gather(a, u.w);
+        const bool use_v = VAR == V_LLP && a.VL != nullptr;
+        gv[4 * j + 0] = use_v ? gather_v(a, u.x) : -1;
+        gv[4 * j + 1] = use_v ? gather_v(a, u.y) : -1;
+        gv[4 * j + 2] = use_v ? gather_v(a, u.z) : -1;
+        gv[4 * j + 3] = use_v ? gather_v(a, u.w) : -1;
       }
       const int cand0 = b.have() ? (int)b.label() : -2;
 #pragma unroll
@@ -1231,7 +1269,7 @@ __global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
           bool fr = false;
           const unsigned cnt = giant_add(tab, tsz, (unsigned)lab[j], c, a.epoch, &fr);
           fresh += fr ? 1u : 0u;
-          b.observe(cnt, (unsigned)lab[j], a);
+          b.observe(cnt, (unsigned)lab[j], a, (VAR == V_LLP && a.VL != nullptr) ? gv[j] : -1);
         }
       }
     }
