@@ -125,13 +125,14 @@ __global__ void k_init_pred(const BinItem* __restrict__ rows, int32_t n_rows, un
 }
 
 // LLP: V[l] = #{w : L[w] = l} [P:119].
-// LLP: VL[q] = V[L[q]], the histogram value of each vertex's label, so that
-// the MFL kernels read a neighbour's V at the neighbour's index (one gather
-// per vertex here instead of one random V[l] gather per candidate label).
-__global__ void k_vl(const int32_t* __restrict__ L, const int32_t* __restrict__ V, int64_t n, int32_t* __restrict__ VL) {
+// LLP: LV[q] = (L[q], V[L[q]]): each vertex's label next to its histogram
+// value, so that the MFL kernels read a neighbour's label and V with one
+// 8-byte gather at the neighbour's index (one random V gather per vertex here
+// instead of one per candidate label there).
+__global__ void k_vl(const int32_t* __restrict__ L, const int32_t* __restrict__ V, int64_t n, int2* __restrict__ LV) {
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
     const int32_t l = L[q];
-    VL[q] = l >= 0 ? V[l] : 0;
+    LV[q] = make_int2(l, l >= 0 ? V[l] : 0);
   }
 }
 

@@ -738,8 +738,8 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     k_hist<<<ga, 256, 0, s>>>(g->L[0], g->n, g->V);
     g->init_launches += 1;
     if (g->use_vl) {
-      if (!g->VL) g->VL = dalloc<int32_t>(g, std::max<int64_t>(g->n, 1));
-      k_vl<<<ga, 256, 0, s>>>(g->L[0], g->V, g->n, g->VL);
+      if (!g->LV) g->LV = dalloc<int2>(g, std::max<int64_t>(g->n, 1));
+      k_vl<<<ga, 256, 0, s>>>(g->L[0], g->V, g->n, g->LV);
       g->init_launches += 1;
     }
     CK(cudaGetLastError());
@@ -827,7 +827,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     // L_0 = PickLabel's identity labelling (a permutation): its histogram V is
     // all ones (k_hist still writes it), so t = 1 needs no V gathers
     a.v_ones = (variant == GLP_VARIANT_LLP && t == 1) ? 1 : 0;
-    a.VL = (variant == GLP_VARIANT_LLP && g->use_vl) ? g->VL : nullptr;
+    a.LV = (variant == GLP_VARIANT_LLP && g->use_vl) ? g->LV : nullptr;
     switch (variant) {
       case GLP_VARIANT_CLASSIC: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
@@ -892,7 +892,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       timed(g, prof, 5, pend, used, s, [&] {
         CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
         k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb], g->n, g->V);
-        if (g->use_vl) k_vl<<<ga, 256, 0, s>>>(g->L[1 - rb], g->V, g->n, g->VL);
+        if (g->use_vl) k_vl<<<ga, 256, 0, s>>>(g->L[1 - rb], g->V, g->n, g->LV);
       });
       launches += g->use_vl ? 1 : 0;
     }

@@ -191,7 +191,7 @@ struct MflArgs {
   double gamma;
   int32_t t;                            // iteration number (1-based)
   int32_t dense;                        // 1: process every listed vertex
-  const int32_t* __restrict__ VL;       // LLP: VL[u] = V[L_{t-1}[u]] (carried with the label), or null
+  const int2* __restrict__ LV;          // LLP: (L_{t-1}[u], V[L_{t-1}[u]]) interleaved, or null
   int32_t v_ones;                       // LLP: V[l] == 1 for every l (L_{t-1} is PickLabel's permutation)
 };
 
@@ -263,7 +263,7 @@ struct glp_graph {
   int32_t* L[2] = {nullptr, nullptr};
   int2* so = nullptr;
   int32_t* V = nullptr;
-  int32_t* VL = nullptr;  // LLP: V of each vertex's current label
+  int2* LV = nullptr;  // LLP: (label, V of the label) of each vertex
   uint8_t* is_seed = nullptr;
   uint8_t* flag[2] = {nullptr, nullptr};
   bool flag_clean[2] = {true, true};
@@ -287,7 +287,7 @@ struct glp_graph {
   // concurrent class kernels within an iteration (GLP_SERIAL=1 disables):
   // xs[0] giant, xs[1] L, xs[2] M, xs[3] low; W and the redo chain on `stream`
   bool concurrent = true;
-  bool use_vl = true;  // LLP carries V[L[u]] with the labels (GLP_NO_VL=1 disables)
+  bool use_vl = true;  // LLP gathers (label, V[label]) pairs from LV (GLP_NO_VL=1 disables)
   int* col_bad = nullptr;  // create: col_idx range check flag (side stream)
   cudaStream_t xs[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaEvent_t xev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};

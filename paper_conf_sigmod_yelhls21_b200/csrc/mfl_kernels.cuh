@@ -113,10 +113,20 @@ __device__ __forceinline__ int ld_label(const int32_t* p) {
 }
 __device__ __forceinline__ int gather(const MflArgs& a, int u) { return u >= 0 ? ld_label(a.R + u) : -1; }
 
-// LLP: V[L_{t-1}[u]] carried next to the label of u (a.VL, computed once per
-// vertex after the histogram): gathered at the same index as the label, so a
-// candidate's V arrives with it instead of a random V[l] gather per label.
-__device__ __forceinline__ int gather_v(const MflArgs& a, int u) { return u >= 0 ? ld_label(a.VL + u) : -1; }
+// LLP: (L_{t-1}[u], V[L_{t-1}[u]]) interleaved in a.LV (rebuilt once per
+// vertex after the histogram): one 8-byte gather at the neighbour's index
+// returns its label and the label's V, so a candidate's V arrives with it
+// instead of a random V[l] gather per label.  Without LV: the plain label.
+__device__ __forceinline__ int gather_lv(const MflArgs& a, int u, bool use_v, int& lv) {
+  if (u < 0) { lv = -1; return -1; }
+  if (use_v) {
+    const int2 x = __ldg(a.LV + u);
+    lv = x.y;
+    return x.x;
+  }
+  lv = -1;
+  return ld_label(a.R + u);
+}
 
 // LLP score val = k - gamma * (v - k) [P:119], double, no contraction (R11).
 __device__ __forceinline__ double llp_score(unsigned k, int v, double gamma) {
@@ -139,7 +149,7 @@ struct Best {
   unsigned long long key = 0ull;
   unsigned lab = kNoLabel;
   int bv = -1;  // LLP: V of the best label
-  // vl: V[l] when the caller has it (carried with the label, a.VL), else -1
+  // vl: V[l] when the caller has it (carried with the label, a.LV), else -1
   __device__ __forceinline__ void observe(unsigned cnt, unsigned l, const MflArgs& a, int vl = -1) {
     if (VAR == V_LLP) {
       // V of a permutation labelling is all ones (t = 1)
@@ -287,7 +297,7 @@ template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
                                                   const int (&labin)[N], Best<VAR>& b, volatile int* overflow,
                                                   const int (&vin)[N], bool use_v) {
-  // use_v (LLP with a.VL): labels carry their V, so LLP observes at insert
+  // use_v (LLP with a.LV): labels carry their V, so LLP observes at insert
   // like CLASSIC; otherwise LLP scores from the final table (table_scan)
   const bool obs = VAR != V_LLP || use_v;
   const int lane = threadIdx.x & 31;
@@ -498,8 +508,8 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       }
       // every vertex of the chunk has degree d; nv vertices, lanes [0, total)
       const int nv = __popc(segs);
-      int lab = gather(a, u);
-      const int lv = (VAR == V_LLP && a.VL != nullptr) ? gather_v(a, u) : -1;
+      int lv;
+      int lab = gather_lv(a, u, VAR == V_LLP && a.LV != nullptr, lv);
       int r = 0;
       int2 so = make_int2(0, 0);
       if (lane < nv) {
@@ -703,10 +713,9 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           next_loaded = true;
         }
         int l[8], lv[8];
-        l[0] = gather(a, x0.x); l[1] = gather(a, x0.y); l[2] = gather(a, x0.z); l[3] = gather(a, x0.w);
-        const bool use_v = VAR == V_LLP && a.VL != nullptr;
-        lv[0] = use_v ? gather_v(a, x0.x) : -1; lv[1] = use_v ? gather_v(a, x0.y) : -1;
-        lv[2] = use_v ? gather_v(a, x0.z) : -1; lv[3] = use_v ? gather_v(a, x0.w) : -1;
+        const bool use_v = VAR == V_LLP && a.LV != nullptr;
+        l[0] = gather_lv(a, x0.x, use_v, lv[0]); l[1] = gather_lv(a, x0.y, use_v, lv[1]);
+        l[2] = gather_lv(a, x0.z, use_v, lv[2]); l[3] = gather_lv(a, x0.w, use_v, lv[3]);
         lv[4] = lv[5] = lv[6] = lv[7] = -1;
         if (kWRound == 256) {
           l[4] = gather(a, x1.x); l[5] = gather(a, x1.y); l[6] = gather(a, x1.z); l[7] = gather(a, x1.w);
@@ -735,12 +744,11 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           for (int b2 = 0; b2 < off; b2 += kWRound) {
             int4 v0, v1;
             load_round(a.col, start, b2, d, v0, v1);
-            const int m8[8] = {gather(a, v0.x), gather(a, v0.y), gather(a, v0.z), gather(a, v0.w),
-                               gather(a, v1.x), gather(a, v1.y), gather(a, v1.z), gather(a, v1.w)};
-            const int mv8[8] = {use_v ? gather_v(a, v0.x) : -1, use_v ? gather_v(a, v0.y) : -1,
-                                use_v ? gather_v(a, v0.z) : -1, use_v ? gather_v(a, v0.w) : -1,
-                                use_v ? gather_v(a, v1.x) : -1, use_v ? gather_v(a, v1.y) : -1,
-                                use_v ? gather_v(a, v1.z) : -1, use_v ? gather_v(a, v1.w) : -1};
+            int m8[8], mv8[8];
+            m8[0] = gather_lv(a, v0.x, use_v, mv8[0]); m8[1] = gather_lv(a, v0.y, use_v, mv8[1]);
+            m8[2] = gather_lv(a, v0.z, use_v, mv8[2]); m8[3] = gather_lv(a, v0.w, use_v, mv8[3]);
+            m8[4] = gather_lv(a, v1.x, use_v, mv8[4]); m8[5] = gather_lv(a, v1.y, use_v, mv8[5]);
+            m8[6] = gather_lv(a, v1.z, use_v, mv8[6]); m8[7] = gather_lv(a, v1.w, use_v, mv8[7]);
             fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v);
           }
         }
@@ -759,7 +767,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       if (over) {
         if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = base + jl * nwarps + gw;
       } else {
-        if (a.VL == nullptr) table_scan<VAR>(tab, lane, 32, a, b);  // LLP (s_over's __syncwarp ended the count)
+        if (a.LV == nullptr) table_scan<VAR>(tab, lane, 32, a, b);  // LLP (s_over's __syncwarp ended the count)
         b.warp_reduce();
         fresh = __reduce_add_sync(kFull, fresh);
         if (lane == jl) {
@@ -824,17 +832,13 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
     if (!IPF && base > 0) block_load_round<BLOCK, UNROLL>(a.col, start, d, base, u);
     if (IPF) block_load_round<BLOCK, UNROLL>(a.col, start, d, base + STEP, un);
     int lab[4 * UNROLL], lv[4 * UNROLL];
-    const bool use_v = VAR == V_LLP && a.VL != nullptr;
+    const bool use_v = VAR == V_LLP && a.LV != nullptr;
 #pragma unroll
     for (int j = 0; j < UNROLL; ++j) {
-      lab[4 * j + 0] = gather(a, u[j].x);
-      lab[4 * j + 1] = gather(a, u[j].y);
-      lab[4 * j + 2] = gather(a, u[j].z);
-      lab[4 * j + 3] = gather(a, u[j].w);
-      lv[4 * j + 0] = use_v ? gather_v(a, u[j].x) : -1;
-      lv[4 * j + 1] = use_v ? gather_v(a, u[j].y) : -1;
-      lv[4 * j + 2] = use_v ? gather_v(a, u[j].z) : -1;
-      lv[4 * j + 3] = use_v ? gather_v(a, u[j].w) : -1;
+      lab[4 * j + 0] = gather_lv(a, u[j].x, use_v, lv[4 * j + 0]);
+      lab[4 * j + 1] = gather_lv(a, u[j].y, use_v, lv[4 * j + 1]);
+      lab[4 * j + 2] = gather_lv(a, u[j].z, use_v, lv[4 * j + 2]);
+      lab[4 * j + 3] = gather_lv(a, u[j].w, use_v, lv[4 * j + 3]);
       const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
       if (stage_out != nullptr && idx < d)
         __stcg((int4*)(stage_out + idx), make_int4(lab[4 * j], lab[4 * j + 1], lab[4 * j + 2], lab[4 * j + 3]));
@@ -1090,7 +1094,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
                                       may_over ? nullptr : &s_major);
       __syncthreads();
       over = s_over != 0;
-      if (!over && a.VL == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
+      if (!over && a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
       __syncthreads();
       if (over && PART) {
         nparts = min(max(2u, ((unsigned)d + SLOTS / 2 - 1) / (SLOTS / 2)), 255u);
@@ -1248,15 +1252,11 @@ __global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
       for (int j = 0; j < kGUnroll; ++j) {
         const int idx = base + (j * kGBlock + (int)threadIdx.x) * 4;
         const int4 u = idx < end ? ld_stream4(a.col + it.start + idx) : make_int4(-1, -1, -1, -1);
-        lab[4 * j + 0] = gather(a, u.x);
-        lab[4 * j + 1] = gather(a, u.y);
-        lab[4 * j + 2] = gather(a, u.z);
-        lab[4 * j + 3] = gather(a, u.w);
-        const bool use_v = VAR == V_LLP && a.VL != nullptr;
-        gv[4 * j + 0] = use_v ? gather_v(a, u.x) : -1;
-        gv[4 * j + 1] = use_v ? gather_v(a, u.y) : -1;
-        gv[4 * j + 2] = use_v ? gather_v(a, u.z) : -1;
-        gv[4 * j + 3] = use_v ? gather_v(a, u.w) : -1;
+        const bool use_v = VAR == V_LLP && a.LV != nullptr;
+        lab[4 * j + 0] = gather_lv(a, u.x, use_v, gv[4 * j + 0]);
+        lab[4 * j + 1] = gather_lv(a, u.y, use_v, gv[4 * j + 1]);
+        lab[4 * j + 2] = gather_lv(a, u.z, use_v, gv[4 * j + 2]);
+        lab[4 * j + 3] = gather_lv(a, u.w, use_v, gv[4 * j + 3]);
       }
       const int cand0 = b.have() ? (int)b.label() : -2;
 #pragma unroll
@@ -1269,7 +1269,7 @@ __global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
           bool fr = false;
           const unsigned cnt = giant_add(tab, tsz, (unsigned)lab[j], c, a.epoch, &fr);
           fresh += fr ? 1u : 0u;
-          b.observe(cnt, (unsigned)lab[j], a, (VAR == V_LLP && a.VL != nullptr) ? gv[j] : -1);
+          b.observe(cnt, (unsigned)lab[j], a, (VAR == V_LLP && a.LV != nullptr) ? gv[j] : -1);
         }
       }
     }
