@@ -72,6 +72,9 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_M_LOAD
 #define GLP_M_LOAD 4
 #endif
+#ifndef GLP_FEWER_BARRIERS
+#define GLP_FEWER_BARRIERS 1
+#endif
 #ifndef GLP_ADD_ALWAYS
 #define GLP_ADD_ALWAYS 1
 #endif
@@ -1095,7 +1098,9 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       __syncthreads();
       over = s_over != 0;
       if (!over && a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
-      __syncthreads();
+      // (s_over is next reset by the partition passes below or at the next row,
+      // which every thread reaches only through block_best's barrier)
+      if (!GLP_FEWER_BARRIERS || (over && PART)) __syncthreads();
       if (over && PART) {
         nparts = min(max(2u, ((unsigned)d + SLOTS / 2 - 1) / (SLOTS / 2)), 255u);
         over = false;
@@ -1189,7 +1194,11 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       a.pred_next[i] = max(dist, 1u) | (mono_done ? kMonoTried : 0u);
       update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty);
     }
-    __syncthreads();
+    // No barrier here: every shared value of this row (table, flags, the
+    // block_best scratch) was last read before block_best's barrier, and the
+    // next row rewrites them only after its own clear barrier; thread 0 alone
+    // reads s_distinct / s_major above and resets them itself.
+    if (!GLP_FEWER_BARRIERS) __syncthreads();
     }  // selected rows
   }
   tally_flush(ty, a.cnt);
