@@ -331,3 +331,15 @@ def test_nccl_exchange_path_single_rank():
         lab = g.labels("cpu").numpy()
     ref = oracle.run(csr, oracle.SEEDED, 30, seeds=seeds.numpy(), threads=8)
     assert info.iterations == ref.iterations and (lab == ref.labels).all()
+
+
+@pytest.mark.parametrize("env", [{"GLP_NO_VL": "1"}, {"GLP_SERIAL": "1"}])
+def test_alternate_execution_modes(env, monkeypatch):
+    """The A/B switches read at graph create (LLP without the interleaved
+    label/V array, serialised class kernels) give the same exact runs."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    csr = graphs.rmat(13, seed=4)
+    assert_same_run(csr, 0, 20)
+    for gamma in (1.0, 0.37):
+        assert_same_run(csr, 2, 8, gamma=gamma)
