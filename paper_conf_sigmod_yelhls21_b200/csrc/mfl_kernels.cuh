@@ -66,6 +66,9 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_L_IPF
 #define GLP_L_IPF 0
 #endif
+#ifndef GLP_L_FILTER
+#define GLP_L_FILTER 4  // L rows split into at most this many label parts count by filtering, not scattering
+#endif
 #ifndef GLP_L_EST
 #define GLP_L_EST 40
 #endif
@@ -827,7 +830,7 @@ template <int VAR, int BLOCK, int UNROLL, bool IPF>
 __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int d, const Table& tab,
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
                                             volatile int* overflow, int* distinct, Best<VAR>& b,
-                                            volatile int* major) {
+                                            volatile int* major, unsigned fparts = 1u) {
   constexpr int STEP = BLOCK * 4 * UNROLL;
   unsigned fresh = 0;
   for (int base = 0; base < d; base += STEP) {
@@ -845,6 +848,11 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
       const int idx = base + (j * BLOCK + (int)threadIdx.x) * 4;
       if (stage_out != nullptr && idx < d)
         __stcg((int4*)(stage_out + idx), make_int4(lab[4 * j], lab[4 * j + 1], lab[4 * j + 2], lab[4 * j + 3]));
+    }
+    if (fparts > 1u) {  // filtered count: only labels of hash partition 0 vote (the row is staged whole)
+#pragma unroll
+      for (int k = 0; k < 4 * UNROLL; ++k)
+        lab[k] = (lab[k] >= 0 && label_part((unsigned)lab[k], fparts) == 0u) ? lab[k] : -1;
     }
     if (IPF) {
 #pragma unroll
@@ -945,7 +953,7 @@ __device__ __forceinline__ Best<VAR> block_best(Best<VAR> b) {
 template <int VAR, int BLOCK>
 __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* stage, int cnt, const Table& tab,
                                              unsigned max_probe, volatile int* overflow, int* distinct,
-                                             Best<VAR>& b) {
+                                             Best<VAR>& b, unsigned fparts = 1u, unsigned part = 0u) {
   unsigned fresh = 0;
   for (int j0 = 0; j0 < cnt; j0 += 4 * BLOCK) {
     int lab[4];
@@ -953,6 +961,8 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
     for (int k = 0; k < 4; ++k) {
       const int j = j0 + k * BLOCK + (int)threadIdx.x;
       lab[k] = j < cnt ? __ldcg(stage + j) : -1;
+      // filtered count: only labels of hash partition `part` of `fparts` vote
+      if (fparts > 1u && lab[k] >= 0 && label_part((unsigned)lab[k], fparts) != part) lab[k] = -1;
     }
     const int nov[4] = {-1, -1, -1, -1};
     fresh += warp_insert_n<VAR, 4>(a, tab, max_probe, lab, b, overflow, nov, false);
@@ -1114,6 +1124,41 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     if (PART) {
       nparts = min(nparts, 255u);
       while (nparts > 1u) {
+        if (nparts <= (unsigned)GLP_L_FILTER) {
+          // Few parts: no partition histogram and scatter.  Part 0 is counted
+          // while the row is gathered and staged (labels of other parts are
+          // skipped), parts 1.. re-read the staged row and count only their
+          // own labels.  Every label lives in exactly one part, so the best
+          // over the parts is the row's MFL.
+          b = Best<VAR>();
+          bool pover = false;
+          unsigned p = 0;
+          for (; p < nparts && !pover; ++p) {
+            const Table tab{smem_tab, (unsigned)SLOTS};
+            tab.clear(threadIdx.x, BLOCK);
+            if (threadIdx.x == 0) {
+              s_over = 0;
+              if (p == 0) s_distinct = 0;
+            }
+            __syncthreads();
+            const bool gather_pass = p == 0 && !staged;
+            if (gather_pass) {
+              block_load_round<BLOCK, UNROLL>(a.col, it.start, d, 0, cur);
+              block_count<VAR, BLOCK, UNROLL, GLP_L_IPF>(a, it.start, d, tab, kLProbe, cur, stageA, &s_over,
+                                                         &s_distinct, b, nullptr, nparts);
+            } else {
+              count_staged<VAR, BLOCK>(a, stageA, d, tab, kLProbe, &s_over, &s_distinct, b, nparts, p);
+            }
+            __syncthreads();
+            pover = s_over != 0;
+            if (!pover && !(gather_pass && a.LV != nullptr)) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
+            if (!pover && gather_pass) staged = true;  // a gather pass that did not overflow staged the whole row
+            __syncthreads();
+          }
+          if (!pover) break;
+          nparts = nparts * 2u;  // a part overflowed: finer partitions (exact recount)
+          continue;
+        }
         // (a) histogram of partitions (gathering + staging the row if needed)
         if (threadIdx.x < 256) s_hist[threadIdx.x] = 0;
         if (threadIdx.x == 0) { s_over = 0; s_distinct = 0; }
