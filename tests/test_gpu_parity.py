@@ -343,3 +343,45 @@ def test_alternate_execution_modes(env, monkeypatch):
     assert_same_run(csr, 0, 20)
     for gamma in (1.0, 0.37):
         assert_same_run(csr, 2, 8, gamma=gamma)
+
+
+def _label_part(lab, nparts):
+    """Host copy of the L kernel's label-partition hash (mfl_kernels.cuh
+    label_part), used only to build inputs that load chosen parts."""
+    h = (lab.astype(np.uint64) * np.uint64(0x85EBCA77) + np.uint64(0x165667B1)) & np.uint64(0xFFFFFFFF)
+    return ((h * np.uint64(nparts)) >> np.uint64(32)).astype(np.int64)
+
+
+def _hub_distinct_t2(labels_of_leaves):
+    """A hub whose leaf i also touches a private vertex p_i with a smaller id:
+    at t = 1 leaf i takes label p_i, so at t = 2 the hub sees one distinct
+    label per arc (its row took the sorted fast path at t = 1, so its
+    distinct-count estimate is a fraction of its degree)."""
+    p = np.asarray(labels_of_leaves, dtype=np.int64)
+    n = int(p.max()) + 1 + p.size + 1
+    used = np.zeros(n, dtype=bool)
+    used[p] = True
+    used[n - 1] = True
+    leaves = np.flatnonzero(~used)[: p.size]
+    hub = n - 1
+    src = np.concatenate([leaves, leaves])
+    dst = np.concatenate([p, np.full(p.size, hub)])
+    return from_edges(n, torch.from_numpy(src), torch.from_numpy(dst), "hub_t2")
+
+
+@pytest.mark.parametrize("case", ["part1_heavy", "d20000", "d40000"])
+def test_l_partition_retries_exact(case):
+    """L rows whose t = 2 labels are all distinct: the filtered part counts,
+    an overflow in the gather pass, an overflow in a later part (staged row,
+    finer partitions) and the histogram path all give the oracle's labels."""
+    if case == "part1_heavy":
+        ids = np.arange(60000)
+        part = _label_part(ids, 2)
+        lab = np.concatenate([ids[part == 1][:10000], ids[part == 0][:500]])
+    else:
+        d = 20000 if case == "d20000" else 40000
+        lab = np.random.default_rng(d).permutation(3 * d)[:d]
+    csr = _hub_distinct_t2(np.sort(lab))
+    assert_same_run(csr, 0, 6)
+    assert_same_run(csr, 2, 4, gamma=0.5)
+    assert_same_run(csr, 1, 6, seeds=[0, int(lab.min()), csr.n - 1])
