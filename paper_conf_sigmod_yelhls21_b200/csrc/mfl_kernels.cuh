@@ -69,6 +69,15 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_L_FILTER
 #define GLP_L_FILTER 4  // L rows split into at most this many label parts count by filtering, not scattering
 #endif
+#ifndef GLP_L_STAGE1
+#define GLP_L_STAGE1 0
+#endif
+#ifndef GLP_L_MAJ
+#define GLP_L_MAJ 1
+#endif
+#ifndef GLP_M_EST
+#define GLP_M_EST 100  // M rows after a sorted-row pass: table sized for this % of the degree (x GLP_M_LOAD)
+#endif
 #ifndef GLP_L_EST
 #define GLP_L_EST 40
 #endif
@@ -1088,14 +1097,17 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     // [P:130] (RMAT probe at t = 2: 26-36 % distinct for deg > 2048); the
     // labels are staged, so an overflow recounts them in partitions
     const unsigned est = a.mode ? (unsigned)d
-                                : (PART && (praw & kMonoTried))
-                                      ? max(1u, (unsigned)(((unsigned long long)pred * GLP_L_EST) / 100ull))
+                                : (praw & kMonoTried)
+                                      ? max(1u, (unsigned)(((unsigned long long)pred * (PART ? GLP_L_EST : GLP_M_EST)) / 100ull))
                                       : pred;
     unsigned nparts = PART ? max(1u, (min(est, (unsigned)d) + SLOTS / 2 - 1) / (SLOTS / 2)) : 1u;
     bool staged = false;  // stageA holds the row's gathered labels
     bool over = false;
     if (nparts == 1u) {
-      // single pass: gather + count (L: stage the labels if an overflow is possible)
+      // single pass: gather + count.  Nothing is staged: an overflow stops the
+      // count early, so the partition passes below gather the row again
+      // (GLP_L_STAGE1 = 1 restores the old, never-read staging writes), and a
+      // strict majority may end the row (GLP_L_MAJ)
       const unsigned want = PART ? 2u * (unsigned)d : GLP_M_LOAD * est;
       const unsigned tsz = min(max(64u, 1u << (32 - __clz(want - 1u))), (unsigned)SLOTS);
       const Table tab{smem_tab, tsz};
@@ -1103,8 +1115,8 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       __syncthreads();
       const bool may_over = PART && 2u * (unsigned)d > (unsigned)SLOTS;
       block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : (PART ? tsz : kTabProbe), cur,
-                                      may_over ? stageA : nullptr, &s_over, &s_distinct, b,
-                                      may_over ? nullptr : &s_major);
+                                      (GLP_L_STAGE1 && may_over) ? stageA : nullptr, &s_over, &s_distinct, b,
+                                      (may_over && !GLP_L_MAJ) ? nullptr : &s_major);
       __syncthreads();
       over = s_over != 0;
       if (!over && a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
