@@ -7,9 +7,13 @@ device-resident graph: PickLabel, then synchronous MFL iterations (gather ->
 count -> arg-max -> update, active-vertex frontier, exact stop rule) until a
 fixed point, a two-cycle or the paper's 20 iterations [P:270].
 
-  value  = GTEPS = (arcs of the graph x iterations) / device time of the run
-           (the paper's "average elapsed time for one iteration" [P:355] as a
-           rate over the graph's edges; arcs = symmetrised CSR entries)
+  value  = GTEPS = arcs actually scanned over the run / device time of the run
+           (GTEPS_t = sum of the degrees of the vertices scanned
+           at t, counting only the arcs whose labels were gathered -- a row
+           that stops on a strict majority is credited with the arcs it
+           read); the paper's "average elapsed time for one iteration"
+           [P:355] as a rate.  nnz x iterations / time is reported beside it
+           as `nnz_x_iterations_gteps` (it credits arcs the frontier skipped)
   e2e    = the same metric through the public C ABI with HOST buffers:
            glp_graph_create(host CSR) + glp_run + glp_labels_get(host) per step
 
@@ -139,6 +143,45 @@ def cpu_reference(csr_cpu, variant, seeds, gamma, iters_per_sample, reps, warmup
     return value, threads, tot_t / max(len(times), 1), tot_it
 
 
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
+def cpu_sequential(csr_cpu, variant, seeds, gamma, arc_budget=150_000_000):
+    """The oracle's per-vertex rule on ONE core (oracle.step, threads=1) for
+    iteration 1 from PickLabel, on the first rows holding ~arc_budget arcs
+    (a bounded sample; arcs/s of the sequential program)."""
+    import numpy as np
+
+    import oracle
+    vid = {"classic": oracle.CLASSIC, "seeded": oracle.SEEDED, "llp": oracle.LLP}[variant]
+    n = csr_cpu.n
+    off, _ = csr_cpu.numpy()
+    v_end = int(np.searchsorted(off, min(arc_budget, int(off[-1])), side="left"))
+    v_end = max(1, min(n, v_end))
+    sd = None if seeds is None else seeds.cpu().numpy()
+    L0 = oracle.init_labels(n, vid, sd)
+    V = np.ones(n, dtype=np.int32) if vid == oracle.LLP else None
+    is_seed = None
+    if vid == oracle.SEEDED:
+        is_seed = np.zeros(n, dtype=np.uint8)
+        if sd is not None and len(sd):
+            is_seed[sd] = 1
+    t0 = time.perf_counter()
+    oracle.step(csr_cpu, vid, L0, 0, v_end, V=V, is_seed=is_seed, gamma=gamma, threads=1)
+    dt = time.perf_counter() - t0
+    arcs = int(off[v_end])
+    return {"value": round(arcs / dt / 1e9, 5), "unit": UNIT, "cores": 1, "arcs": arcs, "seconds": round(dt, 2),
+            "sample": f"iteration 1 from PickLabel on rows [0, {v_end}) ({arcs} arcs), oracle.step, 1 thread"}
+
+
 def flush_l2(buf):
     buf.fill_(1)  # 256 MB write > 126 MB L2
 
@@ -184,12 +227,12 @@ def bench_gpu(args):
         col_h = csr.col_idx.cpu().pin_memory()
         seeds_h = None if seeds is None else seeds.cpu()
         out_h = torch.empty(n, dtype=torch.int32).pin_memory()
-        e2e_ms, e2e_iters, phases = [], 0, []
+        e2e_ms, e2e_arcs, phases = [], 0, []
         e2e_warm = 2  # the first creates grow the stream-ordered pool
         for r in range(e2e_warm + min(args.steps, 3)):
             torch.cuda.synchronize()
             t0 = time.perf_counter()
-            g2 = glp.Graph(n=n, row_offsets=off_h, col_idx=col_h, stream=stream)
+            g2 = glp.Graph(n=n, row_offsets=off_h, col_idx=col_h, symmetric=csr.symmetric, stream=stream)
             t1 = time.perf_counter()
             ri = g2.run(variant, max_iters, seeds_h, gamma=gamma)
             t2 = time.perf_counter()
@@ -199,9 +242,9 @@ def bench_gpu(args):
             g2.close()
             if r >= e2e_warm:
                 e2e_ms.append(dt)
-                e2e_iters += ri.iterations
+                e2e_arcs += ri.arcs_processed
                 phases.append(((t1 - t0) * 1e3, (t2 - t1) * 1e3, (t3 - t2) * 1e3))
-        e2e = {"value": round(nnz * e2e_iters / (sum(e2e_ms) / 1e3) / 1e9, 3), "unit": UNIT,
+        e2e = {"value": round(e2e_arcs / (sum(e2e_ms) / 1e3) / 1e9, 3), "unit": UNIT,
                "h2d_bytes_per_step": int((n + 1) * 8 + nnz * 4 + (0 if seeds is None else 4 * seeds.numel())),
                "d2h_bytes_per_step": int(4 * n), "ms_per_step": round(statistics.mean(e2e_ms), 3),
                "includes": "graph create (H2D copy, relayout) + run + labels D2H",
@@ -275,7 +318,13 @@ def bench_gpu(args):
         t = torch.tensor([csr.nnz], dtype=torch.int64, device=dev)
         arcs_total = csr.nnz  # every rank generated the full graph
     ms_per_step = total_ms / args.steps
-    value = arcs_total * sum(i.iterations for i in infos) / (total_ms / 1e3) / 1e9
+    scanned = sum(i.arcs_processed for i in infos)
+    if world > 1:
+        t = torch.tensor([scanned], dtype=torch.int64, device=dev)
+        dist.all_reduce(t)  # every rank scans its own rows
+        scanned = int(t.item())
+    value = scanned / (total_ms / 1e3) / 1e9
+    nnz_iters = arcs_total * sum(i.iterations for i in infos) / (total_ms / 1e3) / 1e9
 
     # ---- roofline of the dominant kernel (algorithmic bytes / event time) ----
     peak, peak_src = measured_peaks()
@@ -323,6 +372,18 @@ def bench_gpu(args):
         # whole-iteration roofline (SURVEY §8(d) model incl. 4n label first touch)
         it_bytes = [4.0 * s["active_arcs"] + 8.0 * s["active_vertices"] + 4.0 * n + 4.0 * s["changed"] for s in st]
         it1 = st[0] if st else None
+        if roof is not None and st:
+            # every iteration of the last timed run against the same HBM peak:
+            # B_t (4 arcs + 8 vertices + 4n + 4 changed) / t_iter
+            roof["per_iteration"] = [
+                {"t": i + 1, "ms": round(x["ms"], 4), "active_arcs": x["active_arcs"],
+                 "bytes": int(b), "gbps": round(b / (x["ms"] / 1e3) / 1e9, 1),
+                 "frac": round(b / (x["ms"] / 1e3) / 1e9 / peak, 4),
+                 "gteps": round(x["active_arcs"] / (x["ms"] / 1e3) / 1e9, 2)}
+                for i, (x, b) in enumerate(zip(st, it_bytes)) if x["ms"] > 0]
+            tot_ms = sum(x["ms"] for x in st)
+            roof["whole_run"] = {"bytes": int(sum(it_bytes)), "ms": round(tot_ms, 4),
+                                 "frac": round(sum(it_bytes) / (tot_ms / 1e3) / 1e9 / peak, 4) if tot_ms else None}
         out = {
             "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
@@ -339,7 +400,8 @@ def bench_gpu(args):
             "iteration_active_arcs": [s["active_arcs"] for s in st],
             "iteration1_gteps": round(nnz / (it1["ms"] / 1e3) / 1e9, 2) if it1 else None,
             "iteration1_hbm_frac": round(it_bytes[0] / (it1["ms"] / 1e3) / 1e9 / peak, 4) if it1 else None,
-            "scanned_arcs_gteps": round(sum(i.arcs_processed for i in infos) / (total_ms / 1e3) / 1e9, 3),
+            "nnz_x_iterations_gteps": round(nnz_iters, 3),
+            "scanned_arcs_per_step": int(scanned / args.steps),
             "roofline": roof,
             "gpu_launches": int(sum(i.kernel_launches for i in infos)),
             "clocks": clk.summary(),
@@ -352,8 +414,11 @@ def bench_gpu(args):
         samp_iters = 1 if nnz > 50_000_000 else max_iters
         v, cores, sec, its = cpu_reference(csr_cpu, variant, seeds, gamma, samp_iters, reps=1)
         out["cpu_baseline"] = {"value": round(v, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
+                               "cpu_model": cpu_model(),
                                "sample": f"{args.workload}: first {its} LP iteration(s) from PickLabel, "
-                                         f"oracle/glp_oracle.c OpenMP over {cores} threads, {sec:.1f} s"}
+                                         f"oracle/glp_oracle.c OpenMP over {cores} threads, {sec:.1f} s "
+                                         "(the oracle scans every arc each iteration)",
+                               "sequential": cpu_sequential(csr_cpu, variant, seeds, gamma)}
     if rank == 0:
         print(json.dumps(out), flush=True)
     g.close()
@@ -371,16 +436,29 @@ def bench_reference(args):
     dev = "cuda" if torch.cuda.is_available() else "cpu"
     csr, seeds = make_graph(spec, dev)
     csr_cpu = csr.to("cpu")
+    del csr
     seeds = None if seeds is None else seeds.cpu()
-    samp = 1 if csr.nnz > 50_000_000 else max_iters
+    # each step = one whole run of the workload (same config as the GPU arm)
+    # when K+W of them fit the budget, else the first `samp` iterations
+    _, _, probe_s, probe_it = cpu_reference(csr_cpu, variant, seeds, gamma, 1, reps=1)
+    budget_s = float(os.environ.get("GLP_REF_BUDGET_S", "200"))
+    per_it = probe_s / max(probe_it, 1)
+    samp = max_iters if per_it * max_iters * (args.steps + args.warmup) <= budget_s else \
+        max(1, int(budget_s / (per_it * (args.steps + args.warmup))))
+    samp = min(samp, max_iters)
     v, cores, sec, its = cpu_reference(csr_cpu, variant, seeds, gamma, samp, reps=args.steps, warmup=args.warmup)
+    same = samp == max_iters
     out = {"metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": round(sec * 1e3, 2), "higher_is_better": True,
            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic", "impl": "reference",
            "config": {"workload": args.workload, "generator": spec, "variant": variant, "gamma": gamma,
-                      "n": csr.n, "arcs": csr.nnz},
+                      "max_iters": max_iters, "n": csr_cpu.n, "arcs": csr_cpu.nnz, "same_config": same},
            "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
-                            "sample": f"each step = first {samp} LP iteration(s) of {args.workload} from PickLabel"},
+                            "cpu_model": cpu_model(),
+                            "sample": (f"each step = one whole run of {args.workload} (stop rule, <= {max_iters} "
+                                       "iterations)" if same else
+                                       f"each step = first {samp} LP iteration(s) of {args.workload} from "
+                                       "PickLabel") + f"; {its} iterations timed over {args.steps} steps"},
            "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 

@@ -23,13 +23,14 @@ class CSR:
     row_offsets: torch.Tensor  # int64 [n+1]
     col_idx: torch.Tensor      # int32 [nnz]
     name: str = ""
+    symmetric: bool = False    # builder-asserted u in N(v) <=> v in N(u)
 
     @property
     def nnz(self) -> int:
         return int(self.col_idx.numel())
 
     def to(self, device) -> "CSR":
-        return CSR(self.n, self.row_offsets.to(device), self.col_idx.to(device), self.name)
+        return CSR(self.n, self.row_offsets.to(device), self.col_idx.to(device), self.name, self.symmetric)
 
     def numpy(self):
         return (self.row_offsets.cpu().numpy().astype(np.int64, copy=False),
@@ -74,14 +75,15 @@ def from_edges(n: int, src: torch.Tensor, dst: torch.Tensor, name: str = "",
     off = torch.zeros(n + 1, dtype=torch.int64, device=device)
     if n > 0:
         off[1:] = torch.cumsum(counts, 0)
-    return CSR(n, off, cols.contiguous(), name)
+    return CSR(n, off, cols.contiguous(), name, symmetrize)
 
 
-def from_arrays(n: int, row_offsets, col_idx, name: str = "") -> CSR:
-    """Wrap raw (possibly non-symmetric / unvalidated) arrays as a CSR."""
+def from_arrays(n: int, row_offsets, col_idx, name: str = "", symmetric: bool = False) -> CSR:
+    """Wrap raw (possibly non-symmetric / unvalidated) arrays as a CSR; the
+    caller states whether it is symmetric (default: not asserted)."""
     off = torch.as_tensor(np.asarray(row_offsets, dtype=np.int64))
     col = torch.as_tensor(np.asarray(col_idx, dtype=np.int32))
-    return CSR(n, off, col, name)
+    return CSR(n, off, col, name, symmetric)
 
 
 def relabel(csr: CSR, new_id: torch.Tensor) -> CSR:
@@ -91,14 +93,18 @@ def relabel(csr: CSR, new_id: torch.Tensor) -> CSR:
     rows = torch.repeat_interleave(torch.arange(csr.n, device=off.device), deg)
     src = new_id[rows]
     dst = new_id[csr.col_idx.to(torch.int64)]
-    return from_edges(csr.n, src, dst, csr.name, symmetrize=False)
+    out = from_edges(csr.n, src, dst, csr.name, symmetrize=False)
+    out.symmetric = csr.symmetric  # a permutation keeps (a)symmetry
+    return out
 
 
 def save_npz(csr: CSR, path: str) -> None:
     off, col = csr.numpy()
-    np.savez(path, n=np.int64(csr.n), row_offsets=off, col_idx=col, name=np.str_(csr.name))
+    np.savez(path, n=np.int64(csr.n), row_offsets=off, col_idx=col, name=np.str_(csr.name),
+             symmetric=np.bool_(csr.symmetric))
 
 
 def load_npz(path: str) -> CSR:
     z = np.load(path)
-    return CSR(int(z["n"]), torch.from_numpy(z["row_offsets"]), torch.from_numpy(z["col_idx"]), str(z["name"]))
+    return CSR(int(z["n"]), torch.from_numpy(z["row_offsets"]), torch.from_numpy(z["col_idx"]), str(z["name"]),
+               bool(z["symmetric"]) if "symmetric" in z else False)

@@ -229,7 +229,7 @@ def rmat(scale: int, edge_factor: int = 16, seed: int = 1, device="cpu", scrambl
         del key, rows, counts
     col = torch.cat(cols) if len(cols) > 1 else cols[0]
     del cols
-    return CSR(n, off, col.contiguous(), f"rmat{scale}ef{edge_factor}")
+    return CSR(n, off, col.contiguous(), f"rmat{scale}ef{edge_factor}", True)
 
 
 def _trunc_powerlaw_quantiles(count: int, alpha: float, lo: float, hi: float, device):

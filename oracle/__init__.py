@@ -45,7 +45,7 @@ def _load():
                                        ctypes.c_int32, P, P, P, P]
         lib.glp_oracle_step.restype = ctypes.c_int
         lib.glp_oracle_step.argtypes = [ctypes.c_int64, P, P, ctypes.c_int32, P, P, P, ctypes.c_double,
-                                        ctypes.c_int64, ctypes.c_int64, P]
+                                        ctypes.c_int64, ctypes.c_int64, P, ctypes.c_int32]
         lib.glp_oracle_modularity.restype = ctypes.c_double
         lib.glp_oracle_modularity.argtypes = [ctypes.c_int64, P, P, P]
         _lib = lib
@@ -104,7 +104,7 @@ def run(csr, variant: int = CLASSIC, max_iters: int = 20, seeds=None, gamma: flo
 
 
 def step(csr, variant: int, labels_prev, v_begin: int = 0, v_end=None, V=None, is_seed=None,
-         gamma: float = 0.0, out=None) -> np.ndarray:
+         gamma: float = 0.0, out=None, threads: int = 1) -> np.ndarray:
     """One synchronous iteration for rows [v_begin, v_end) (see glp_oracle.c)."""
     lib = _load()
     n, off, col = _csr_np(csr)
@@ -114,7 +114,7 @@ def step(csr, variant: int, labels_prev, v_begin: int = 0, v_end=None, V=None, i
     Vh = None if V is None else np.ascontiguousarray(V, dtype=np.int32)
     sd = None if is_seed is None else np.ascontiguousarray(is_seed, dtype=np.uint8)
     rc = lib.glp_oracle_step(n, _ptr(off), _ptr(col), int(variant), _ptr(Lp), _ptr(Vh), _ptr(sd),
-                             float(gamma), int(v_begin), int(v_end), _ptr(out))
+                             float(gamma), int(v_begin), int(v_end), _ptr(out), int(threads))
     if rc != 0:
         raise ValueError(f"glp_oracle_step failed rc={rc}")
     return out

@@ -156,7 +156,7 @@ def glp_partition(n: int, nranks: int, row_offsets=None, edge_balanced: bool = F
 
 
 def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Tensor, *,
-                     v_begin: int = 0, v_end: int | None = None, symmetric: bool = True,
+                     v_begin: int = 0, v_end: int | None = None, symmetric: bool = False,
                      rank: int = 0, nranks: int = 1, device: int | None = None,
                      nccl_unique_id: bytes | None = None, stream: torch.cuda.Stream | None = None,
                      validate: bool = True):
@@ -200,8 +200,9 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
     st = lib.glp_graph_create(ctypes.byref(c), None if d is None else ctypes.byref(d), ctypes.byref(prm),
                               ctypes.byref(h))
     if st == 3 and torch.cuda.is_available():
-        # GLP_ERR_OUT_OF_MEMORY: the library allocates with cudaMalloc, so
-        # return torch's cached blocks to the driver and try once more
+        # GLP_ERR_OUT_OF_MEMORY: the library already trimmed its private pool
+        # and retried; torch's caching allocator may still hold freed blocks,
+        # so return them to the driver and try once more
         torch.cuda.empty_cache()
         st = lib.glp_graph_create(ctypes.byref(c), None if d is None else ctypes.byref(d), ctypes.byref(prm),
                                   ctypes.byref(h))
@@ -298,10 +299,16 @@ class Graph:
     copied to the device by the library.
     """
 
-    def __init__(self, csr=None, *, n=None, row_offsets=None, col_idx=None, symmetric=True,
+    def __init__(self, csr=None, *, n=None, row_offsets=None, col_idx=None, symmetric=None,
                  validate=True, **dist):
+        # symmetric: None = the CSR's own flag (glp_inputs.CSR.symmetric), else
+        # False -- the frontier push is exact only on symmetric graphs, so it
+        # is never assumed (the C ABI's zero default)
         if csr is not None:
             n, row_offsets, col_idx = csr.n, csr.row_offsets, csr.col_idx
+            if symmetric is None:
+                symmetric = bool(getattr(csr, "symmetric", False))
+        symmetric = bool(symmetric) if symmetric is not None else False
         self.n = int(n)
         self._off = row_offsets
         self._col = col_idx

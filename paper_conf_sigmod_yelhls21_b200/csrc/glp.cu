@@ -47,30 +47,52 @@ thread_local std::string g_last_error = "";
     }                                                                                      \
   } while (0)
 
-// Device memory comes from the device's stream-ordered memory pool
-// (cudaMallocAsync), which keeps up to kPoolKeep bytes (env GLP_POOL_KEEP_GB) of freed memory mapped
-// between graphs: create/destroy of a multi-GB graph then costs no driver
-// map/unmap (plain cudaMalloc/cudaFree made end-to-end create times vary from
-// 0.1 to 2 s on the B200 box).
+// Device memory comes from a PRIVATE stream-ordered memory pool per device
+// (cudaMemPoolCreate; not the device's default pool, which torch's
+// cudaMallocAsync backend may share), which keeps up to kPoolKeep bytes (env
+// GLP_POOL_KEEP_GB) of freed memory mapped between graphs: create/destroy of
+// a multi-GB graph then costs no driver map/unmap (plain cudaMalloc/cudaFree
+// made end-to-end create times vary from 0.1 to 2 s on the B200 box).  When an
+// allocation fails, the pool's unused reserve is returned to the driver
+// (cudaMemPoolTrimTo) and the allocation is retried once.
 constexpr uint64_t kPoolKeep = 16ull << 30;
-cudaError_t pool_malloc(void** p, size_t bytes, cudaStream_t s) {
+cudaMemPool_t device_pool(int dev) {
   static std::mutex mu;
-  static std::vector<int> ready;
+  static std::vector<cudaMemPool_t> pools;
+  std::lock_guard<std::mutex> lock(mu);
+  if ((int)pools.size() <= dev) pools.resize(dev + 1, nullptr);
+  if (!pools[dev]) {
+    cudaMemPoolProps props;
+    memset(&props, 0, sizeof(props));
+    props.allocType = cudaMemAllocationTypePinned;
+    props.handleTypes = cudaMemHandleTypeNone;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t pool = nullptr;
+    if (cudaMemPoolCreate(&pool, &props) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    uint64_t keep = kPoolKeep;
+    if (const char* e = getenv("GLP_POOL_KEEP_GB")) keep = (uint64_t)(atof(e) * (double)(1ull << 30));
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    pools[dev] = pool;
+  }
+  return pools[dev];
+}
+cudaError_t pool_malloc(void** p, size_t bytes, cudaStream_t s) {
   int dev = 0;
   cudaGetDevice(&dev);
-  {
-    std::lock_guard<std::mutex> lock(mu);
-    if (std::find(ready.begin(), ready.end(), dev) == ready.end()) {
-      cudaMemPool_t pool;
-      if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-        uint64_t keep = kPoolKeep;
-        if (const char* e = getenv("GLP_POOL_KEEP_GB")) keep = (uint64_t)(atof(e) * (double)(1ull << 30));
-        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
-      }
-      ready.push_back(dev);
-    }
+  cudaMemPool_t pool = device_pool(dev);
+  if (!pool) return cudaMallocAsync(p, bytes, s);
+  cudaError_t e = cudaMallocFromPoolAsync(p, bytes, pool, s);
+  if (e == cudaErrorMemoryAllocation) {
+    cudaGetLastError();
+    cudaStreamSynchronize(s);  // frees queued on this stream complete first
+    cudaMemPoolTrimTo(pool, 0);
+    e = cudaMallocFromPoolAsync(p, bytes, pool, s);
   }
-  return cudaMallocAsync(p, bytes, s);
+  return e;
 }
 void pool_free(void* p, cudaStream_t s) {
   if (p) cudaFreeAsync(p, s);
@@ -541,10 +563,13 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->grid_g = grid_for(sms, (const void*)mfl_giant_count<V_LLP>, kGBlock, 0);
     g->grid_aux = sms * 8;
     if (g->n_rows > 0) {
-      // L staging: two row-sized buffers per resident L block
+      // L staging: two row-sized buffers per resident L block, in two regions:
+      // the static L launch (side stream) and the redo L launch (main stream)
+      // may run at the same time, so each has its own (a shared
+      // region let a redo row overwrite a static row's staged labels).
       // L never takes giant rows (deg > kGiantMin)
       g->stage_stride = (std::min<int64_t>(g->max_deg, kGiantMin) + 3) & ~(int64_t)3;
-      g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 2 * g->grid_l);
+      g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 4 * g->grid_l);
     }
     CK(cudaStreamSynchronize(g->stream));
   } catch (...) {
@@ -671,6 +696,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     if (used_x[2]) CK(cudaStreamWaitEvent(s0, g->xev[1], 0));
     MflArgs q = r;
     q.mode = 1; q.cnt = c + 3; q.redo_in = g->redo_l; q.redo_in_n = &sc->n_redo_l; q.work = &sc->work_lr;
+    q.stage = g->stage + (size_t)g->stage_stride * 2 * g->grid_l;  // redo region (runs beside static L)
     timed(g, prof, 3, pend, used, s0, [&] { GLP_L_KERNEL(VAR)<<<g->grid_l, kLBlock, ls_, s0>>>(q); });
     n += 2;
   }

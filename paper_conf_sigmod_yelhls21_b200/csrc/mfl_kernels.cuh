@@ -425,9 +425,11 @@ __device__ __forceinline__ void tally_flush(Tally t, Counters* cnt) {
 //   r   = L_{t-1}[v];  have = some neighbour voted;  best = winning label.
 // Writes W[v] unconditionally (the frontier invariant of DESIGN.md §Frontier),
 // and records (t, r) in so[v] when the label changed.
+// `scanned` = arcs whose labels were gathered (< deg after a majority exit);
+// `deg` feeds the frontier-size estimate (sum of changed degrees).
 template <int VAR>
 __device__ __forceinline__ void update_vertex(const MflArgs& a, int v, int deg, bool have, unsigned best,
-                                              Tally& ty) {
+                                              Tally& ty, int scanned) {
   const int64_t gv = a.vb + v;
   const int r = ld_label(a.R + gv);
   int nw = have ? (int)best : r;
@@ -436,7 +438,7 @@ __device__ __forceinline__ void update_vertex(const MflArgs& a, int v, int deg, 
   const int l2 = (so.x == a.t - 1) ? so.y : r;  // L_{t-2}[v]
   a.W[gv] = nw;
   ty.verts += 1;
-  ty.arcs += (unsigned long long)deg;
+  ty.arcs += (unsigned long long)scanned;
   ty.d2 += (nw != l2);
   if (nw != r) {
     ty.changed += 1;
@@ -686,6 +688,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
     bool rdone = false;
     unsigned long long rkey = 0ull;
     unsigned rlab = kNoLabel, rpred = 0u;
+    int rscan = 0;
     int jl = __ffs(todo) - 1;
     todo &= todo - 1;
     int64_t start = __shfl_sync(kFull, mine.start, jl);
@@ -719,7 +722,9 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       int prev = -1;
       bool next_loaded = false;  // x0/x1 hold the next row's first round
       bool major = false;        // a strict-majority label was observed: the rest of the row cannot change the MFL
+      int scanned = 0;           // arcs gathered so far
       for (int off = 0; off < d && !over && !major; off += kWRound) {
+        scanned = min(d, off + kWRound);
         int4 p0, p1;
         if (off + kWRound < d) {
           load_round(a.col, start, off + kWRound, d, p0, p1);
@@ -789,6 +794,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           rdone = true;
           rkey = b.key;
           rlab = b.lab;
+          rscan = scanned;
           // a row that just took the sorted fast path is not retried next time
           // (a majority exit saw part of the row: keep the old prediction if larger)
           rpred = max(major ? max(fresh, pred & kPredMask) : fresh, 1u) | (tried && mono ? kMonoTried : 0u);
@@ -806,7 +812,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       r.key = rkey;
       r.lab = rlab;
       a.pred_next[il] = rpred;
-      update_vertex<VAR>(a, mine.v, mine.d, r.have(), r.label(), ty);
+      update_vertex<VAR>(a, mine.v, mine.d, r.have(), r.label(), ty, rscan);
     }
   }
   tally_flush(ty, a.cnt);
@@ -839,10 +845,11 @@ template <int VAR, int BLOCK, int UNROLL, bool IPF>
 __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int d, const Table& tab,
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
                                             volatile int* overflow, int* distinct, Best<VAR>& b,
-                                            volatile int* major, unsigned fparts = 1u) {
+                                            volatile int* major, unsigned fparts = 1u, int* scanned = nullptr) {
   constexpr int STEP = BLOCK * 4 * UNROLL;
   unsigned fresh = 0;
-  for (int base = 0; base < d; base += STEP) {
+  int base = 0;
+  for (; base < d; base += STEP) {
     int4 un[UNROLL];
     if (!IPF && base > 0) block_load_round<BLOCK, UNROLL>(a.col, start, d, base, u);
     if (IPF) block_load_round<BLOCK, UNROLL>(a.col, start, d, base + STEP, un);
@@ -877,7 +884,11 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
     if (__any_sync(kFull, *overflow != 0)) break;  // warp-uniform exit
   }
   fresh = __reduce_add_sync(kFull, fresh);
-  if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
+  if ((threadIdx.x & 31) == 0) {
+    if (fresh) atomicAdd(distinct, (int)fresh);
+    // arcs this warp gathered: rounds up to the one it stopped in
+    if (scanned != nullptr) atomicMax(scanned, min(d, base + STEP));
+  }
 }
 
 // Block-level sorted-row fast path (see warp_quads_increasing): rounds of
@@ -1004,7 +1015,7 @@ template <int VAR, int BLOCK, int SLOTS, bool PART, int UNROLL, int CLS>
 #endif
 __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_block(MflArgs a) {
   extern __shared__ __align__(16) unsigned long long smem_tab[];  // SLOTS
-  __shared__ int s_over, s_distinct, s_major;
+  __shared__ int s_over, s_distinct, s_major, s_scan;
   __shared__ int s_hist[PART ? 256 : 1], s_cur[PART ? 256 : 1];
   Tally ty;
   int32_t* stageA = PART ? a.stage + (int64_t)blockIdx.x * 2 * a.stage_stride : nullptr;
@@ -1075,7 +1086,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     const unsigned pred = s_pe[q];
     const int d = it.d;
     Best<VAR> b;
-    if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; s_major = 0; }
+    if (threadIdx.x == 0) { s_distinct = 0; s_over = 0; s_major = 0; s_scan = 0; }
     bool mono_done = false;
     if (!a.mode && cand) {
       __syncthreads();
@@ -1116,7 +1127,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       const bool may_over = PART && 2u * (unsigned)d > (unsigned)SLOTS;
       block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : (PART ? tsz : kTabProbe), cur,
                                       (GLP_L_STAGE1 && may_over) ? stageA : nullptr, &s_over, &s_distinct, b,
-                                      (may_over && !GLP_L_MAJ) ? nullptr : &s_major);
+                                      (may_over && !GLP_L_MAJ) ? nullptr : &s_major, 1u, &s_scan);
       __syncthreads();
       over = s_over != 0;
       if (!over && a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
@@ -1249,7 +1260,8 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     if (threadIdx.x == 0) {
       const unsigned dist = s_major ? max((unsigned)s_distinct, pred) : (unsigned)s_distinct;  // partial on a majority exit
       a.pred_next[i] = max(dist, 1u) | (mono_done ? kMonoTried : 0u);
-      update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty);
+      // arcs gathered: the whole row unless the single pass stopped on a majority
+      update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty, s_major ? s_scan : d);
     }
     // No barrier here: every shared value of this row (table, flags, the
     // block_best scratch) was last read before block_best's barrier, and the
@@ -1364,7 +1376,7 @@ __global__ void __launch_bounds__(256) mfl_giant_finish(MflArgs a, const int32_t
     if (threadIdx.x == 0) {
       a.pred_next[i] = max(a.gdistinct[i], 1u);
       a.gdistinct[i] = 0u;
-      update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty);
+      update_vertex<VAR>(a, it.v, it.d, b.have(), b.label(), ty, it.d);
     }
   } else if (threadIdx.x == 0) {
     a.pred_next[i] = a.pred[i];

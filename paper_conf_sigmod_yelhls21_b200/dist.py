@@ -47,5 +47,6 @@ def distributed_graph(csr, group=None, edge_balanced: bool = False, stream=None)
     off, col = local_rows(csr.row_offsets, csr.col_idx, vb, ve)
     uid = broadcast_unique_id(group) if world > 1 else None
     dev = torch.cuda.current_device()
-    return Graph(n=csr.n, row_offsets=off, col_idx=col, rank=rank, nranks=world, nccl_unique_id=uid,
+    return Graph(n=csr.n, row_offsets=off, col_idx=col, symmetric=csr.symmetric, rank=rank, nranks=world,
+                 nccl_unique_id=uid,
                  v_begin=vb, v_end=ve, device=dev, stream=stream)

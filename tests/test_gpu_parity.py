@@ -48,7 +48,7 @@ def assert_same_run(csr, variant=0, max_iters=20, seeds=None, gamma=0.0, frontie
 # --------------------------------------------------------------------------- small, per iteration
 def test_bowtie_golden_trajectories(golden_dir):
     g = json.load(open(os.path.join(golden_dir, "bowtie.json")))
-    csr = from_arrays(g["graph"]["n"], g["graph"]["row_offsets"], g["graph"]["col_idx"])
+    csr = from_arrays(g["graph"]["n"], g["graph"]["row_offsets"], g["graph"]["col_idx"], symmetric=True)
     for case, variant in [("classic", 0), ("llp_gamma_1", 2), ("seeded_4", 1), ("seeded_1_4", 1)]:
         exp = g[case]
         for t, row in enumerate(exp["trajectory"], start=1):
@@ -176,7 +176,7 @@ def _perturb_rows(csr, mode, seed=0):
             col[a:b] = g.permutation(col[a:b])
         else:
             col[b - 2], col[b - 1] = col[b - 1], col[b - 2]
-    return from_arrays(csr.n, off, col)
+    return from_arrays(csr.n, off, col, symmetric=csr.symmetric)
 
 
 @pytest.mark.parametrize("mode", ["shuffle", "tail"])
