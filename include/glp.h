@@ -92,15 +92,26 @@ typedef struct {
                                   0: the frontier is disabled (full sweeps)    */
 } glp_csr;
 
-/* Multi-GPU placement (1-D vertex-range partition, one process per GPU).
- * NULL = single GPU, device = current device. */
+/* In-process rank group: P ranks (P graphs, one host thread each) in ONE
+ * process exchange labels through each other's device buffers instead of NCCL
+ * (glp_local_group_create).  Used to run the partitioned path on one GPU. */
+typedef struct glp_local_group glp_local_group;
+
+/* Multi-GPU placement (1-D vertex-range partition, one process per GPU, or P
+ * ranks of one local group).  NULL = single GPU, device = current device.
+ * Creating and running a partitioned graph are COLLECTIVE: every rank calls
+ * glp_graph_create / glp_run with the same arguments (except its own rows),
+ * concurrently (separate processes or separate host threads). */
 typedef struct {
   int32_t rank, nranks;        /* this process's rank and the world size      */
   int32_t device;              /* CUDA ordinal for this rank                   */
   const void *nccl_unique_id;  /* 128 bytes from glp_nccl_unique_id() on rank 0,
-                                  broadcast by the caller; NULL if nranks == 1 */
+                                  broadcast by the caller; NULL if nranks == 1
+                                  or local_group is set                        */
   void *cuda_stream;           /* cudaStream_t to run on, or NULL = a stream
                                   owned by the library                         */
+  glp_local_group *local_group;/* non-NULL: exchange through this in-process
+                                  group (borrowed; must outlive the graph)     */
 } glp_dist;
 
 /* Run parameters.  Zero-initialise, set struct_size = sizeof(glp_params),
@@ -119,7 +130,14 @@ typedef struct {
   int32_t debug_pred_cap;      /* testing only: clamp each row's predicted
                                   distinct-label count (forces the overflow /
                                   re-queue paths; results are unchanged); 0 off */
-  int32_t reserved[6];
+  int32_t llp_hist;            /* LLP label histogram with nranks > 1:
+                                  0 default (= 2), 1 replicated (every rank
+                                  counts all n labels after the label
+                                  all-gather), 2 sharded (each rank counts its
+                                  own rows, the counts are all-reduced, and the
+                                  (label, V) pairs of the owned rows are
+                                  all-gathered instead of the labels)          */
+  int32_t reserved[5];
 } glp_params;
 
 typedef struct {
@@ -150,6 +168,13 @@ typedef struct {
   double bytes;                /* algorithmic bytes       */
   double arcs;                 /* arcs processed                                */
 } glp_kernel_stat;
+
+/* In-process group of nranks ranks (1 <= nranks <= 16); owned by the caller,
+ * destroyed after every graph that uses it.  A rank that fails inside a
+ * collective aborts the group: the other ranks' calls then return
+ * GLP_ERR_STATE instead of waiting (and the group cannot be reused). */
+glp_status glp_local_group_create(int32_t nranks, glp_local_group **out);
+glp_status glp_local_group_destroy(glp_local_group *grp); /* NULL-safe */
 
 /* 128-byte NCCL unique id; rank 0 calls it and broadcasts the bytes. */
 glp_status glp_nccl_unique_id(uint8_t out[128]);

@@ -47,7 +47,8 @@ class glp_csr(ctypes.Structure):
 
 class glp_dist(ctypes.Structure):
     _fields_ = [("rank", ctypes.c_int32), ("nranks", ctypes.c_int32), ("device", ctypes.c_int32),
-                ("nccl_unique_id", ctypes.c_void_p), ("cuda_stream", ctypes.c_void_p)]
+                ("nccl_unique_id", ctypes.c_void_p), ("cuda_stream", ctypes.c_void_p),
+                ("local_group", ctypes.c_void_p)]
 
 
 class glp_params(ctypes.Structure):
@@ -55,7 +56,7 @@ class glp_params(ctypes.Structure):
                 ("frontier", ctypes.c_int32), ("stop_on_2cycle", ctypes.c_int32),
                 ("validate", ctypes.c_int32), ("profile", ctypes.c_int32),
                 ("dense_divisor", ctypes.c_int32), ("debug_pred_cap", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 6)]
+                ("llp_hist", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5)]
 
 
 class glp_run_info(ctypes.Structure):
@@ -77,7 +78,7 @@ class glp_kernel_stat(ctypes.Structure):
 
 EXPORTS = ["glp_nccl_unique_id", "glp_partition", "glp_graph_create", "glp_run", "glp_labels_get",
            "glp_iter_stats", "glp_kernel_stats", "glp_graph_info", "glp_graph_destroy",
-           "glp_last_error", "glp_version"]
+           "glp_local_group_create", "glp_local_group_destroy", "glp_last_error", "glp_version"]
 
 _lib = None
 
@@ -103,6 +104,8 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "glp_kernel_stats": [P, P, I32, P],
         "glp_graph_info": [P, P, I32],
         "glp_graph_destroy": [P],
+        "glp_local_group_create": [I32, P],
+        "glp_local_group_destroy": [P],
     }
     for name, args in sig.items():
         fn = getattr(lib, name)
@@ -123,7 +126,7 @@ def _check(st: int):
 
 def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = True,
                 validate: bool = True, profile: bool = False, dense_divisor: int = 0,
-                debug_pred_cap: int = 0) -> glp_params:
+                debug_pred_cap: int = 0, llp_hist: int = 0) -> glp_params:
     p = glp_params()
     p.struct_size = ctypes.sizeof(glp_params)
     p.gamma = float(gamma)
@@ -133,6 +136,7 @@ def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = T
     p.profile = int(bool(profile))
     p.dense_divisor = int(dense_divisor)
     p.debug_pred_cap = int(debug_pred_cap)
+    p.llp_hist = int(llp_hist)
     return p
 
 
@@ -159,7 +163,7 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
                      v_begin: int = 0, v_end: int | None = None, symmetric: bool = False,
                      rank: int = 0, nranks: int = 1, device: int | None = None,
                      nccl_unique_id: bytes | None = None, stream: torch.cuda.Stream | None = None,
-                     validate: bool = True):
+                     validate: bool = True, local_group=None):
     """Create a device graph.  CUDA tensors are borrowed (keep them alive);
     CPU tensors are copied.  Returns an opaque handle (ctypes.c_void_p)."""
     lib = load_library()
@@ -182,7 +186,7 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
     c.symmetric = int(bool(symmetric))
     d = None
     uid_buf = None
-    if nranks > 1 or device is not None or stream is not None:
+    if nranks > 1 or device is not None or stream is not None or local_group is not None:
         d = glp_dist()
         d.rank, d.nranks = int(rank), int(nranks)
         d.device = int(device if device is not None else
@@ -191,6 +195,7 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
             uid_buf = (ctypes.c_uint8 * 128).from_buffer_copy(nccl_unique_id)
             d.nccl_unique_id = ctypes.cast(uid_buf, ctypes.c_void_p)
         d.cuda_stream = stream.cuda_stream if stream is not None else None
+        d.local_group = local_group
     if on_device and stream is None:
         # borrowed tensors are read on the library's own stream: they must be
         # complete (torch may still be producing them on its current stream)
@@ -212,7 +217,7 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
 
 def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, gamma: float = 0.0,
             frontier: int = -1, stop_on_2cycle: bool = True, profile: bool = False,
-            dense_divisor: int = 0, debug_pred_cap: int = 0) -> dict:
+            dense_divisor: int = 0, debug_pred_cap: int = 0, llp_hist: int = 0) -> dict:
     import numpy as np
     lib = load_library()
     sd = None
@@ -222,7 +227,7 @@ def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, 
         ns = int(sd.size)
     info = glp_run_info()
     prm = make_params(gamma=gamma, frontier=frontier, stop_on_2cycle=stop_on_2cycle, profile=profile,
-                      dense_divisor=dense_divisor, debug_pred_cap=debug_pred_cap)
+                      dense_divisor=dense_divisor, debug_pred_cap=debug_pred_cap, llp_hist=llp_hist)
     _check(lib.glp_run(handle, int(variant), int(max_iters), None if sd is None else sd.ctypes.data, ns,
                        ctypes.byref(prm), ctypes.byref(info)))
     return dict(iterations=info.iterations, stop_reason=info.stop_reason,
@@ -265,6 +270,18 @@ def glp_graph_info(handle) -> dict:
     names = ["isolated", "low", "mid", "high", "huge"]
     bins = {nm: dict(vertices=int(out[2 + 2 * i]), arcs=int(out[3 + 2 * i])) for i, nm in enumerate(names)}
     return dict(n=int(out[0]), nnz=int(out[1]), bins=bins, max_degree=int(out[12]), low_chunks=int(out[13]))
+
+
+def glp_local_group_create(nranks: int):
+    """An in-process rank group (see glp.h): handle for glp_graph_create(local_group=...)."""
+    h = ctypes.c_void_p()
+    _check(load_library().glp_local_group_create(int(nranks), ctypes.byref(h)))
+    return h
+
+
+def glp_local_group_destroy(handle) -> None:
+    if handle:
+        _check(load_library().glp_local_group_destroy(handle))
 
 
 def glp_graph_destroy(handle) -> None:

@@ -136,6 +136,12 @@ __global__ void k_vl(const int32_t* __restrict__ L, const int32_t* __restrict__ 
   }
 }
 
+// LLP at t = 0: L_0 is a permutation, so V[L_0[q]] = 1 for every q.
+__global__ void k_lv_ones(const int32_t* __restrict__ L, int64_t n, int2* __restrict__ LV) {
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x)
+    LV[q] = make_int2(L[q], 1);
+}
+
 __global__ void k_hist(const int32_t* __restrict__ L, int64_t n, int32_t* __restrict__ V) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
     const int32_t l = L[v];

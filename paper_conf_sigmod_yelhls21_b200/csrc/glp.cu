@@ -3,7 +3,8 @@
 // Per LP iteration t, all on the graph's stream:
 //   1. reset per-bin counters                                  (memset 256 B)
 //   2. MFL kernels huge, high, mid, low        R = L_{t-1} -> W = L_t
-//   3. [P > 1] ncclAllGather of the owned label slice, counters all-reduce
+//   3. [P > 1] all-gather of the owned label slice, counters all-reduce
+//      (comm.cuh: NCCL across processes, or an in-process local group)
 //   4. read the counters (changed, d2, sum of changed degrees) -> stop rule R8
 //   5. frontier decision: dense when sum_{changed} deg > nnz / dense_divisor,
 //      else k_push marks N(v) + v for changed v (exact for CLASSIC/SEEDED, R9)
@@ -24,10 +25,10 @@
 #include <vector>
 
 #include "aux_kernels.cuh"
+#include "comm.cuh"
 #include "glp_internal.cuh"
 #include "layout.cuh"
 #include "mfl_kernels.cuh"
-#include "nccl_dyn.cuh"
 
 using namespace glp;
 
@@ -190,7 +191,8 @@ void free_graph(glp_graph* g) {
   if (g->ev_b) cudaEventDestroy(g->ev_b);
   for (auto& e : g->ev_pool) cudaEventDestroy(e);
   for (auto& e : g->xev) if (e) cudaEventDestroy(e);
-  nccl_destroy(g);
+  delete g->comm;
+  g->comm = nullptr;
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
   delete g;
 }
@@ -379,9 +381,9 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
   if (nl) k_perm<<<gb, 256, 0, s>>>(orig_local, nl, g->vb, g->pos, g->orig);
   if (g->npad > g->n) k_iota2<<<1, 256, 0, s>>>(g->pos, g->orig, g->n, g->npad);
   CK(cudaGetLastError());
-  if (g->nccl) {
-    nccl_exchange(g, g->pos);
-    nccl_exchange(g, g->orig);
+  if (g->comm) {
+    g->comm->allgather(g, g->pos, sizeof(int32_t));
+    g->comm->allgather(g, g->orig, sizeof(int32_t));
   }
   // ---- the arcs themselves (copied and checked on the side stream)
   CK(cudaStreamWaitEvent(s, g->xev[1], 0));
@@ -417,7 +419,10 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     rank = dist->rank;
     nranks = dist->nranks;
     if (nranks < 1 || rank < 0 || rank >= nranks) fail(GLP_ERR_INVALID_ARGUMENT, "bad rank/nranks");
-    if (nranks > 1 && !dist->nccl_unique_id) fail(GLP_ERR_INVALID_ARGUMENT, "nccl_unique_id required for nranks > 1");
+    if (nranks > 1 && !dist->nccl_unique_id && !dist->local_group)
+      fail(GLP_ERR_INVALID_ARGUMENT, "nccl_unique_id or local_group required for nranks > 1");
+    if (dist->nccl_unique_id && dist->local_group)
+      fail(GLP_ERR_INVALID_ARGUMENT, "set nccl_unique_id or local_group, not both");
   }
   if (nranks == 1 && (csr->v_begin != 0 || csr->v_end != n))
     fail(GLP_ERR_INVALID_ARGUMENT, "single GPU: owned range must be [0, n_global)");
@@ -519,15 +524,19 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     const int64_t npad = ((n + nranks - 1) / nranks) * nranks;
     g->npad = npad;
     g->nnz_global = g->nnz;
-    // NCCL exchange for nranks > 1; with nranks == 1 a unique id still selects
-    // the NCCL path (a one-rank communicator), which tests its plumbing on one GPU
-    if (nranks > 1 || (dist && dist->nccl_unique_id)) nccl_init(g, dist->nccl_unique_id);
+    // exchange for nranks > 1: an in-process local group, else NCCL; with
+    // nranks == 1 a unique id or group still selects that path (a one-rank
+    // communicator), which tests its plumbing on one GPU
+    if (dist && dist->local_group) g->comm = new LocalComm(g, dist->local_group);
+    else if (nranks > 1 || (dist && dist->nccl_unique_id)) g->comm = new NcclComm(g, dist->nccl_unique_id);
+    if (g->comm) g->comm->setup(g);
     build_layout(g, off_d, col_d);
 
     g->L[0] = dalloc<int32_t>(g, npad);
     g->L[1] = dalloc<int32_t>(g, npad);
     g->so = dalloc<int2>(g, g->nl);
     g->V = dalloc<int32_t>(g, std::max<int64_t>(n, 1));
+    if (g->comm) g->Vloc = dalloc<int32_t>(g, std::max<int64_t>(n, 1));
     g->is_seed = dalloc<uint8_t>(g, g->nl);
     g->flag[0] = dalloc<uint8_t>(g, npad);
     g->flag[1] = dalloc<uint8_t>(g, npad);
@@ -572,7 +581,12 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 4 * g->grid_l);
     }
     CK(cudaStreamSynchronize(g->stream));
+  } catch (const Err& e) {
+    if (g->comm) g->comm->abort(e.msg);  // release the other ranks of a local group
+    free_graph(g);
+    throw;
   } catch (...) {
+    if (g->comm) g->comm->abort("rank failed in glp_graph_create");
     free_graph(g);
     throw;
   }
@@ -758,14 +772,15 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     g->init_launches += 1;
     CK(cudaGetLastError());
   }
+  // LLP histogram with several ranks: sharded (each rank counts its rows,
+  // all-reduce, all-gather of the owned (label, V) pairs) or replicated
+  const bool llp_shard = variant == GLP_VARIANT_LLP && g->comm && g->use_vl && p.llp_hist != 1;
   if (variant == GLP_VARIANT_LLP) {
-    // V[l] = #{w : L_0[w] = l} = 1 for every l (L_0[v] = v)
-    CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
-    k_hist<<<ga, 256, 0, s>>>(g->L[0], g->n, g->V);
-    g->init_launches += 1;
+    // V[l] = #{w : L_0[w] = l} = 1 for every l (L_0 is a permutation): t = 1
+    // reads no V (v_ones), and LV = (L_0[q], 1) needs no histogram
     if (g->use_vl) {
-      if (!g->LV) g->LV = dalloc<int2>(g, std::max<int64_t>(g->n, 1));
-      k_vl<<<ga, 256, 0, s>>>(g->L[0], g->V, g->n, g->LV);
+      if (!g->LV) g->LV = dalloc<int2>(g, std::max<int64_t>(g->npad, 1));  // npad: equal-slice all-gather
+      k_lv_ones<<<ga, 256, 0, s>>>(g->L[0], g->n, g->LV);
       g->init_launches += 1;
     }
     CK(cudaGetLastError());
@@ -789,7 +804,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       g->init_launches += 1;
       CK(cudaGetLastError());
       g->flag_clean[fb] = false;
-      if (g->nccl) nccl_merge_flags(g, g->flag[fb]);
+      if (g->comm) g->comm->merge_flags(g, g->flag[fb]);
       if (g->n_chunks) {
         k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_base, g->flag[fb], g->vb, g->cflag);
         g->init_launches += 1;
@@ -854,14 +869,16 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     // all ones (k_hist still writes it), so t = 1 needs no V gathers
     a.v_ones = (variant == GLP_VARIANT_LLP && t == 1) ? 1 : 0;
     a.LV = (variant == GLP_VARIANT_LLP && g->use_vl) ? g->LV : nullptr;
+    a.lv_labels = llp_shard ? 1 : 0;  // non-owned labels live only in LV
     switch (variant) {
       case GLP_VARIANT_CLASSIC: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
       default: launches += launch_mfl<V_LLP>(g, a, prof, pend, used); break;
     }
-    if (g->nccl) {
-      timed(g, prof, 6, pend, used, s, [&] { nccl_exchange(g, g->L[1 - rb]); });
-      nccl_sum_counters(g, g->d_cnt, 5 * sizeof(Counters) / sizeof(unsigned long long));
+    if (g->comm) {
+      // sharded LLP replicates (label, V) pairs after the histogram instead
+      if (!llp_shard) timed(g, prof, 6, pend, used, s, [&] { g->comm->allgather(g, g->L[1 - rb], sizeof(int32_t)); });
+      g->comm->allreduce_u64(g, (unsigned long long*)g->d_cnt, 5 * sizeof(Counters) / sizeof(unsigned long long));
     }
     CK(cudaMemcpyAsync(g->h_cnt, g->d_cnt, 5 * sizeof(Counters), cudaMemcpyDeviceToHost, s));
     CK(cudaEventRecord(e1, s));
@@ -896,13 +913,15 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     // frontier of t+1: dense when the changed vertices touch > nnz/divisor arcs
     const int nf = 1 - fb;
     bool next_dense = true;
-    if (!stop && use_frontier)
+    // nothing of t+1 is prepared after the last iteration (stop or max_iters)
+    const bool last = stop || t == max_iters;
+    if (!last && use_frontier)
       next_dense = (double)tot.chdeg * (double)p.dense_divisor > (double)g->nnz_global;
-    if (!stop && !next_dense) {
+    if (!last && !next_dense) {
       launches += 1;
       timed(g, prof, 4, pend, used, s, [&] {
         k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, g->flag[nf]);
-        if (g->nccl) nccl_merge_flags(g, g->flag[nf]);
+        if (g->comm) g->comm->merge_flags(g, g->flag[nf]);
         if (g->n_chunks)
           k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_base, g->flag[nf], g->vb, g->cflag);
       });
@@ -913,14 +932,30 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       CK(cudaMemsetAsync(g->flag[fb], 0, std::max<int64_t>(g->npad, 1), s));
       g->flag_clean[fb] = true;
     }
-    if (!stop && variant == GLP_VARIANT_LLP) {
+    if (!last && variant == GLP_VARIANT_LLP) {
       launches += 1;
-      timed(g, prof, 5, pend, used, s, [&] {
-        CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
-        k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb], g->n, g->V);
-        if (g->use_vl) k_vl<<<ga, 256, 0, s>>>(g->L[1 - rb], g->V, g->n, g->LV);
-      });
-      launches += g->use_vl ? 1 : 0;
+      if (llp_shard) {
+        // this rank's rows only: V = sum over ranks of the owned counts, then
+        // LV of the owned rows, all-gathered (replaces the label all-gather)
+        timed(g, prof, 5, pend, used, s, [&] {
+          CK(cudaMemsetAsync(g->Vloc, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
+          if (g->nl) k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb] + g->vb, g->nl, g->Vloc);
+          CK(cudaGetLastError());
+          g->comm->allreduce_i32(g, g->Vloc, g->V, (size_t)g->n);
+          if (g->nl) k_vl<<<ga, 256, 0, s>>>(g->L[1 - rb] + g->vb, g->V, g->nl, g->LV + g->vb);
+        });
+        timed(g, prof, 6, pend, used, s, [&] { g->comm->allgather(g, g->LV, sizeof(int2)); });
+        launches += 1;
+        g->kstats[5].arcs += (double)g->nl;  // labels histogrammed by this rank
+      } else {
+        timed(g, prof, 5, pend, used, s, [&] {
+          CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
+          k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb], g->n, g->V);
+          if (g->use_vl) k_vl<<<ga, 256, 0, s>>>(g->L[1 - rb], g->V, g->n, g->LV);
+        });
+        launches += g->use_vl ? 1 : 0;
+        g->kstats[5].arcs += (double)g->n;
+      }
     }
     g->iter_stats.push_back(st);
     g->pb = (g->pb + 1) % 3;
@@ -929,6 +964,8 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     dense = next_dense;
     if (stop) break;
   }
+  // sharded LLP exchanged (label, V) pairs only: replicate the final labels
+  if (llp_shard && iters > 0) g->comm->allgather(g, g->L[rb], sizeof(int32_t));
   if (!pend.empty()) {
     CK(cudaStreamSynchronize(s));
     drain(false);
@@ -961,7 +998,24 @@ glp_status glp_graph_create(const glp_csr* csr, const glp_dist* dist, const glp_
 
 glp_status glp_run(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_t* seeds, int64_t n_seeds,
                    const glp_params* params, glp_run_info* info) {
-  return guard([&] { run_impl(g, variant, max_iters, seeds, n_seeds, params, info); });
+  const glp_status st = guard([&] { run_impl(g, variant, max_iters, seeds, n_seeds, params, info); });
+  // a failed rank releases the others of its local group (they would wait
+  // at the next exchange forever)
+  if (st != GLP_OK && g && g->comm) g->comm->abort(g_last_error);
+  return st;
+}
+
+glp_status glp_local_group_create(int32_t nranks, glp_local_group** out) {
+  return guard([&] {
+    if (!out) fail(GLP_ERR_INVALID_ARGUMENT, "out is NULL");
+    *out = nullptr;
+    if (nranks < 1 || nranks > kMaxLocalRanks) fail(GLP_ERR_INVALID_ARGUMENT, "nranks must be in [1, 16]");
+    *out = new glp_local_group(nranks);
+  });
+}
+
+glp_status glp_local_group_destroy(glp_local_group* grp) {
+  return guard([&] { delete grp; });
 }
 
 glp_status glp_labels_get(const glp_graph* g, int32_t* out, int64_t out_len, int32_t out_on_device) {

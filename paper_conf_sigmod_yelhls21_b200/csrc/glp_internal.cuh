@@ -23,6 +23,8 @@
 
 namespace glp {
 
+struct Comm;  // comm.cuh: the exchange of the 1-D partition (NCCL or in-process)
+
 // Degree bin of the packed-warp kernel (PAPER §4.2): deg <= 32.
 constexpr int kLowMax = 32;
 constexpr int kLowBlock = 256;
@@ -193,6 +195,7 @@ struct MflArgs {
   int32_t dense;                        // 1: process every listed vertex
   const int2* __restrict__ LV;          // LLP: (L_{t-1}[u], V[L_{t-1}[u]]) interleaved, or null
   int32_t v_ones;                       // LLP: V[l] == 1 for every l (L_{t-1} is PickLabel's permutation)
+  int32_t lv_labels;                    // LLP sharded: neighbour labels are read from LV (R holds owned rows only)
 };
 
 // Internal error: thrown inside the library, converted to glp_status at the ABI.
@@ -214,7 +217,7 @@ struct glp_graph {
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   int rank = 0, nranks = 1;
-  void* nccl = nullptr;  // ncclComm_t when nranks > 1
+  glp::Comm* comm = nullptr;  // exchange when nranks > 1 (or a one-rank NCCL comm)
 
   int64_t n = 0, vb = 0, ve = 0, nl = 0, nnz = 0;
   int64_t npad = 0;        // label arrays padded to a multiple of nranks
@@ -263,6 +266,7 @@ struct glp_graph {
   int32_t* L[2] = {nullptr, nullptr};
   int2* so = nullptr;
   int32_t* V = nullptr;
+  int32_t* Vloc = nullptr;  // LLP, sharded histogram: this rank's counts (summed into V)
   int2* LV = nullptr;  // LLP: (label, V of the label) of each vertex
   uint8_t* is_seed = nullptr;
   uint8_t* flag[2] = {nullptr, nullptr};

@@ -126,7 +126,10 @@ __device__ __forceinline__ int ld_label(const int32_t* p) {
   return __ldg(p);
 #endif
 }
-__device__ __forceinline__ int gather(const MflArgs& a, int u) { return u >= 0 ? ld_label(a.R + u) : -1; }
+__device__ __forceinline__ int gather(const MflArgs& a, int u) {
+  if (u < 0) return -1;
+  return a.lv_labels ? __ldg(&a.LV[u].x) : ld_label(a.R + u);
+}
 
 // LLP: (L_{t-1}[u], V[L_{t-1}[u]]) interleaved in a.LV (rebuilt once per
 // vertex after the histogram): one 8-byte gather at the neighbour's index

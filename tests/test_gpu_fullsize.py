@@ -55,11 +55,14 @@ def test_rmat24_iteration1_closed_form(rmat24):
     assert (lab == exp).all()
 
 
-def test_rmat24_llp_first_iterations(rmat24):
+def test_rmat24_llp_full_run(rmat24):
+    """The bench's LLP configuration end to end: 20 iterations (the thrash
+    regime where one flipped decision would cascade)."""
     dev, cpu = rmat24
-    lab, info, _ = _run(dev, "llp", 4, gamma=1.0)
-    ref = oracle.run(cpu, oracle.LLP, 4, gamma=1.0, threads=THREADS)
-    assert info.iterations == ref.iterations
+    lab, info, st = _run(dev, "llp", 20, gamma=1.0)
+    ref = oracle.run(cpu, oracle.LLP, 20, gamma=1.0, threads=THREADS)
+    assert (info.iterations, info.stop_reason) == (ref.iterations, ref.stop_reason)
+    assert [s["changed"] for s in st] == list(ref.changed)
     agree = (lab == ref.labels).mean()
     assert agree >= 0.9999
     assert abs(oracle.modularity(cpu, lab) - oracle.modularity(cpu, ref.labels)) <= 1e-9
@@ -75,12 +78,14 @@ def test_sbm1m_classic_to_convergence():
     assert (lab == ref.labels).all()
 
 
-def test_taobao100m_seeded_first_iterations():
+def test_taobao100m_seeded_to_fixed_point():
+    """configs[3] as bench.py runs it: seeded LP to its stop rule."""
     dev, seeds = graphs.taobao(device="cuda")
     cpu = dev.to("cpu")
     s = seeds.cpu().numpy()
-    lab, info, st = _run(dev, "seeded", 4, s)
-    ref = oracle.run(cpu, oracle.SEEDED, 4, seeds=s, threads=THREADS)
+    lab, info, st = _run(dev, "seeded", 20, s)
+    ref = oracle.run(cpu, oracle.SEEDED, 20, seeds=s, threads=THREADS)
+    assert (info.iterations, info.stop_reason) == (ref.iterations, ref.stop_reason)
     assert [x["changed"] for x in st] == list(ref.changed)
     assert (lab == ref.labels).all()
     assert (lab[s] == s).all()
@@ -148,3 +153,31 @@ def test_rmat28_llp_iteration2_sampled_oracle(rmat28):
     V = torch.bincount(L1.to(torch.int64), minlength=n).to(torch.int32).cpu().numpy()
     out = oracle.step((S + A, offc.cpu().numpy(), colc.cpu().numpy()), oracle.LLP, Lp, 0, S, V=V, gamma=1.0)
     assert (out[:S] == L2[samp].cpu().numpy()).all()
+
+
+@pytest.mark.parametrize("t", [2, 3, 4, 20])
+def test_rmat28_llp_iteration_all_vertices(rmat28, t):
+    """Every vertex of iteration t recomputed by the oracle (oracle.step over
+    all n rows, host threads) from the GPU's own L_{t-1} and its histogram:
+    the GPU's L_t must equal it bit for bit.  t = 2..4 are the dense,
+    distinct-heavy iterations; t = 20 the late oscillating regime."""
+    csr, g = rmat28
+    cpu = _r28_cpu(csr)
+    g.run("llp", t - 1, gamma=1.0)
+    Lp = g.labels("cuda")
+    V = torch.bincount(Lp.to(torch.int64), minlength=csr.n).to(torch.int32).cpu().numpy()
+    Lp = Lp.cpu().numpy()
+    g.run("llp", t, gamma=1.0)
+    Lt = g.labels("cpu").numpy()
+    out = oracle.step(cpu, oracle.LLP, Lp, 0, csr.n, V=V, gamma=1.0, threads=THREADS)
+    mism = np.flatnonzero(out != Lt)
+    assert mism.size == 0, f"t={t}: {mism.size} labels differ, first {mism[:10]}"
+
+
+_R28_CPU = {}
+
+
+def _r28_cpu(csr):
+    if "c" not in _R28_CPU:
+        _R28_CPU["c"] = csr.to("cpu")
+    return _R28_CPU["c"]
