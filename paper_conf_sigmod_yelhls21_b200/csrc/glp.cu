@@ -542,8 +542,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->flag[1] = dalloc<uint8_t>(g, npad);
     CK(cudaMemsetAsync(g->flag[0], 0, std::max<int64_t>(npad, 1), g->stream));
     CK(cudaMemsetAsync(g->flag[1], 0, std::max<int64_t>(npad, 1), g->stream));
-    g->d_cnt = dalloc<Counters>(g, 5);
-    CK(cudaMallocHost(&g->h_cnt, 5 * sizeof(Counters)));
+    g->d_cnt = dalloc<Counters>(g, kNumCounters);
+    CK(cudaMallocHost(&g->h_cnt, kNumCounters * sizeof(Counters)));
     CK(cudaEventCreate(&g->ev_a));
     CK(cudaEventCreate(&g->ev_b));
     {
@@ -551,6 +551,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       g->concurrent = !(ser && ser[0] == '1');
       const char* novl = getenv("GLP_NO_VL");
       g->use_vl = !(novl && novl[0] == '1');
+      const char* nomono = getenv("GLP_NO_MONO");
+      g->use_mono = !(nomono && nomono[0] == '1');
     }
 
     const int sms = g->sms;
@@ -568,6 +570,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaFuncSetAttribute(mfl_warp<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
     g->grid_w = grid_for(sms, (const void*)mfl_warp<V_LLP>, kWBlock, ws_);
     g->grid_m = grid_for(sms, (const void*)GLP_M_KERNEL(V_LLP), kMBlock, ms_);
+    g->grid_mono = grid_for(sms, (const void*)mfl_mono<V_LLP>, kMonoBlock, 0);
     g->grid_l = grid_for(sms, (const void*)GLP_L_KERNEL(V_LLP), kLBlock, ls_);
     g->grid_g = grid_for(sms, (const void*)mfl_giant_count<V_LLP>, kGBlock, 0);
     g->grid_aux = sms * 8;
@@ -610,8 +613,8 @@ cudaEvent_t pool_event(glp_graph* g, size_t& used) {
 }
 
 const char* kKernelNames[] = {"mfl_low", "mfl_warp", "mfl_block_m", "mfl_block_l", "push", "llp_hist", "exchange",
-                              "mfl_giant"};
-constexpr int kNumKernelNames = 8;
+                              "mfl_giant", "mfl_mono"};
+constexpr int kNumKernelNames = 9;
 
 template <class F>
 void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t& used, cudaStream_t st, F f) {
@@ -682,6 +685,13 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     const int grid = std::min<int>(g->grid_m, g->n_ge8k + (g->n_gt256 - g->n_ge8k + 31) / 32);
     timed(g, prof, 2, pend, used, cc ? g->xs[2] : s0, [&] { GLP_M_KERNEL(VAR)<<<grid, kMBlock, ms_, S(2)>>>(b); });
     if (cc) CK(cudaEventRecord(g->xev[1], g->xs[2]));
+    ++n;
+  }
+  if (g->n_rows && a.mono_kernel) {  // t = 1: sorted-row candidates, table-free; unsorted rows -> M redo list
+    MflArgs b = r;
+    b.n_items = g->n_rows; b.cnt = c + 5; b.redo_out = g->redo_m; b.redo_out_n = &sc->n_redo_m;
+    const int grid = std::min<int>(g->grid_mono, (g->n_rows + kMonoBlock - 1) / kMonoBlock);
+    timed(g, prof, 8, pend, used, s0, [&] { mfl_mono<VAR><<<grid, kMonoBlock, 0, s0>>>(b); });
     ++n;
   }
   if (g->n_rows) {  // W: every row of class W; overflowing rows -> M redo list
@@ -831,9 +841,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       KStat& ks = g->kstats[pe.kid];
       ks.launches += 1;
       ks.ms += kms;
-      if (with_counters && (pe.kid < 4 || pe.kid == 7) && pe.t == cur_t && !credited[pe.kid]) {
+      if (with_counters && (pe.kid < 4 || pe.kid >= 7) && pe.t == cur_t && !credited[pe.kid]) {
         credited[pe.kid] = true;
-        const Counters& c = g->h_cnt[pe.kid == 7 ? 4 : pe.kid];
+        const Counters& c = g->h_cnt[pe.kid == 7 ? 4 : pe.kid == 8 ? 5 : pe.kid];
         ks.arcs += (double)c.arcs;
         // 4 B/arc (col_idx) + 8 B/active vertex (row offsets) + 4 B/changed label
         ks.bytes += 4.0 * (double)c.arcs + 8.0 * (double)c.verts + 4.0 * (double)c.changed;
@@ -849,7 +859,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   for (int32_t t = 1; t <= max_iters; ++t) {
     cudaEvent_t e0 = pool_event(g, used), e1 = pool_event(g, used);
     CK(cudaEventRecord(e0, s));
-    CK(cudaMemsetAsync(g->d_cnt, 0, 5 * sizeof(Counters), s));
+    CK(cudaMemsetAsync(g->d_cnt, 0, kNumCounters * sizeof(Counters), s));
     CK(cudaMemsetAsync(g->d_sched, 0, sizeof(Sched), s));
     g->cur_t = t;
     if (g->n_giant) {
@@ -870,6 +880,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     a.v_ones = (variant == GLP_VARIANT_LLP && t == 1) ? 1 : 0;
     a.LV = (variant == GLP_VARIANT_LLP && g->use_vl) ? g->LV : nullptr;
     a.lv_labels = llp_shard ? 1 : 0;  // non-owned labels live only in LV
+    // t = 1: every row is a sorted-row candidate (unique labels); they go to
+    // the table-free mono kernel (SEEDED never takes the sorted path)
+    a.mono_kernel = (t == 1 && variant != GLP_VARIANT_SEEDED && g->use_mono) ? 1 : 0;
     switch (variant) {
       case GLP_VARIANT_CLASSIC: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
@@ -878,14 +891,14 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     if (g->comm) {
       // sharded LLP replicates (label, V) pairs after the histogram instead
       if (!llp_shard) timed(g, prof, 6, pend, used, s, [&] { g->comm->allgather(g, g->L[1 - rb], sizeof(int32_t)); });
-      g->comm->allreduce_u64(g, (unsigned long long*)g->d_cnt, 5 * sizeof(Counters) / sizeof(unsigned long long));
+      g->comm->allreduce_u64(g, (unsigned long long*)g->d_cnt, kNumCounters * sizeof(Counters) / sizeof(unsigned long long));
     }
-    CK(cudaMemcpyAsync(g->h_cnt, g->d_cnt, 5 * sizeof(Counters), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(g->h_cnt, g->d_cnt, kNumCounters * sizeof(Counters), cudaMemcpyDeviceToHost, s));
     CK(cudaEventRecord(e1, s));
     CK(cudaStreamSynchronize(s));
     Counters tot;
     memset(&tot, 0, sizeof(tot));
-    for (int b = 0; b < 5; ++b) {
+    for (int b = 0; b < kNumCounters; ++b) {
       tot.changed += g->h_cnt[b].changed; tot.d2 += g->h_cnt[b].d2; tot.chdeg += g->h_cnt[b].chdeg;
       tot.arcs += g->h_cnt[b].arcs; tot.verts += g->h_cnt[b].verts;
     }

@@ -93,16 +93,17 @@ constexpr int kGBlock = 512;
 constexpr int kGUnroll = 2;
 constexpr int kGCountBits = 25;  // count field of a giant-table slot (deg < 2^25)
 constexpr int kGEpochBits = 64 - 31 - kGCountBits;
-enum RowClass { CLS_W = 0, CLS_M = 1, CLS_L = 2, CLS_G = 3 };
+enum RowClass { CLS_W = 0, CLS_M = 1, CLS_L = 2, CLS_G = 3, CLS_MONO = 4 };
 // pred word: low 31 bits = predicted distinct labels; bit 31 = the row took
 // the sorted-row fast path last time (do not retry it)
 constexpr unsigned kPredMask = 0x7fffffffu, kMonoTried = 0x80000000u;
 // A sorted-row candidate (`mono`: its labels were all distinct last time and
 // it has not tried the fast path yet, e.g. every row at t = 1) needs no table:
-// it goes to the barrier-free warp kernel whatever its size.
-__host__ __device__ __forceinline__ int row_class(unsigned pred, int d, bool mono) {
+// it goes to the barrier-free warp kernel whatever its size (to the table-free
+// mono kernel when that one is launched: mono_k, t = 1).
+__host__ __device__ __forceinline__ int row_class(unsigned pred, int d, bool mono, bool mono_k = false) {
   if (d > kGiantMin) return CLS_G;
-  if (mono) return d > kMonoWMax ? CLS_L : CLS_W;
+  if (mono) return d > kMonoWMax ? CLS_L : (mono_k ? CLS_MONO : CLS_W);
   if (pred <= kWPred && d <= kWMaxDeg) return CLS_W;
   if (pred <= kMPred && d <= kMMaxDeg) return CLS_M;
   return CLS_L;
@@ -152,6 +153,9 @@ struct Counters {
   unsigned long long pad[2];
 };
 
+// per-kernel iteration counters: low, W, M, L, giant, mono
+constexpr int kNumCounters = 6;
+
 // Arguments shared by the MFL kernels (passed by value).
 struct MflArgs {
   const int32_t* __restrict__ col;      // col2: bin-major arcs (global ids, -1 = padding)
@@ -196,6 +200,7 @@ struct MflArgs {
   const int2* __restrict__ LV;          // LLP: (L_{t-1}[u], V[L_{t-1}[u]]) interleaved, or null
   int32_t v_ones;                       // LLP: V[l] == 1 for every l (L_{t-1} is PickLabel's permutation)
   int32_t lv_labels;                    // LLP sharded: neighbour labels are read from LV (R holds owned rows only)
+  int32_t mono_kernel;                  // sorted-row candidates go to mfl_mono (launched this iteration)
 };
 
 // Internal error: thrown inside the library, converted to glp_status at the ABI.
@@ -279,7 +284,7 @@ struct glp_graph {
   int64_t seeds_cap = 0;
 
   // launch geometry
-  int grid_low = 0, grid_w = 0, grid_m = 0, grid_l = 0, grid_g = 0, grid_aux = 0;
+  int grid_low = 0, grid_w = 0, grid_m = 0, grid_l = 0, grid_g = 0, grid_aux = 0, grid_mono = 0;
 
   int cur = 0;  // index of L holding the result of the last run
   int cur_t = 0;  // iteration being launched (profiling)
@@ -292,6 +297,7 @@ struct glp_graph {
   // xs[0] giant, xs[1] L, xs[2] M, xs[3] low; W and the redo chain on `stream`
   bool concurrent = true;
   bool use_vl = true;  // LLP gathers (label, V[label]) pairs from LV (GLP_NO_VL=1 disables)
+  bool use_mono = true;  // t = 1 sorted-row candidates in mfl_mono (GLP_NO_MONO=1: in the W kernel)
   int* col_bad = nullptr;  // create: col_idx range check flag (side stream)
   cudaStream_t xs[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaEvent_t xev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};

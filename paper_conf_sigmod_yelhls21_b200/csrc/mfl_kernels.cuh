@@ -60,6 +60,10 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_LOW_REDUX
 #define GLP_LOW_REDUX 0
 #endif
+#ifndef GLP_LOW_MATCH
+#define GLP_LOW_MATCH 6  // low segments of at least this degree count with match.any (33 = never);
+                         // A/B: 6 / 12 / 17 all -2.8 % per R24 run vs never (shuffle loop)
+#endif
 #ifndef GLP_L_OPT
 #define GLP_L_OPT 0
 #endif
@@ -311,10 +315,25 @@ __device__ __forceinline__ unsigned ht_add(const Table& t, unsigned lab, unsigne
 // match) with predicated atomics; only labels whose home slot holds another
 // label fall back to the probing loop.  Returns this lane's count of newly
 // claimed slots.
+// Rows predicted to hold more than d / GLP_HOT_DIV distinct labels (few
+// repeats per label: t = 2..3) skip the hot-label pass, whose single-lane
+// insert costs more than it saves there (0 = always take it).
+#ifndef GLP_HOT_DIV
+#define GLP_HOT_DIV 0
+#endif
+// GLP_MATCH_INSERT: 1 = equal labels of one batch slot are merged across the
+// warp with match.any (the lowest lane inserts the group's count); 2 = the
+// same without the hot-label pass
+#ifndef GLP_MATCH_INSERT
+#define GLP_MATCH_INSERT 0
+#endif
+__device__ __forceinline__ bool hot_pass(unsigned pred, int d) {
+  return GLP_HOT_DIV == 0 || (unsigned long long)pred * GLP_HOT_DIV <= (unsigned long long)d;
+}
 template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
                                                   const int (&labin)[N], Best<VAR>& b, volatile int* overflow,
-                                                  const int (&vin)[N], bool use_v) {
+                                                  const int (&vin)[N], bool use_v, bool hot_ok = true) {
   // use_v (LLP with a.LV): labels carry their V, so LLP observes at insert
   // like CLASSIC; otherwise LLP scores from the final table (table_scan)
   const bool obs = VAR != V_LLP || use_v;
@@ -330,7 +349,7 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
     candv = (cand < 0 && lab[j] >= 0) ? (use_v ? vin[j] : -1) : candv;
     cand = (cand < 0 && lab[j] >= 0) ? lab[j] : cand;
   }
-  const int hot = __shfl_sync(kFull, cand, 0);
+  const int hot = (hot_ok && GLP_MATCH_INSERT != 2) ? __shfl_sync(kFull, cand, 0) : -1;
   const int hotv = __shfl_sync(kFull, candv, 0);
   if (hot >= 0) {  // warp-uniform
     unsigned hc = 0;
@@ -346,6 +365,17 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
       else if (obs) b.observe(cnt, (unsigned)hot, a, hotv);
     }
   }
+  unsigned mc[N];  // occurrences this lane inserts for slot j
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    mc[j] = 1u;
+    if (GLP_MATCH_INSERT) {
+      const unsigned m = __match_any_sync(kFull, lab[j]);
+      const bool lead = (m & ((1u << lane) - 1u)) == 0u;
+      mc[j] = __popc(m);
+      lab[j] = lead ? lab[j] : -1;
+    }
+  }
   unsigned h[N], k[N];
 #pragma unroll
   for (int j = 0; j < N; ++j) {
@@ -354,11 +384,11 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
   }
   unsigned cnt[N];
 #pragma unroll
-  for (int j = 0; j < N; ++j) cnt[j] = lab[j] >= 0 ? slot_try(t, h[j], (unsigned)lab[j], 1u, k[j], &nfresh) : 0u;
+  for (int j = 0; j < N; ++j) cnt[j] = lab[j] >= 0 ? slot_try(t, h[j], (unsigned)lab[j], mc[j], k[j], &nfresh) : 0u;
 #pragma unroll
   for (int j = 0; j < N; ++j) {
     if (lab[j] >= 0 && cnt[j] == 0u) {
-      cnt[j] = ht_probe_from(t, (unsigned)lab[j], 1u, h[j], max_probe, &nfresh);
+      cnt[j] = ht_probe_from(t, (unsigned)lab[j], mc[j], h[j], max_probe, &nfresh);
       if (cnt[j] == 0u) *overflow = 1;
     }
   }
@@ -540,17 +570,36 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       if (!vote) lab = -1;
       // first lane of this lane's segment (vmask [P:230])
       const int sstart = 31 - __clz(segs & ((2u << lane) - 1u));
+      const int head = (lane < nv ? lane * d : 0) & 31;  // lane jv takes segment jv
+      Best<VAR> h;
+      // Every segment's labels valid and strictly increasing (t = 1's unique
+      // labels on sorted rows): all counts are 1, so the MFL is the segment
+      // head's label (R4) and nothing needs counting.  CLASSIC/SEEDED at any
+      // t; LLP only while V == 1 (equal scores).
+      const int up = __shfl_up_sync(kFull, lab, 1);
+      const bool inc = lane >= total || (vote && (lane == sstart || up < lab));
+      if ((VAR != V_LLP || a.v_ones) && __all_sync(kFull, inc)) {
+        const int hl = __shfl_sync(kFull, lab, head);
+        h.observe(1u, (unsigned)hl, a, 1);
+      } else {
       // label frequency inside the vertex's lanes [P:231-232]
       unsigned k = 0;
       bool first = true;  // LLP: only a label's first lane scores it (one V[l] gather per distinct label)
+      if (d >= GLP_LOW_MATCH) {
+        // long segments: one match.any over the warp, restricted to the
+        // segment's lanes (d warp-uniform), instead of d shuffles
+        const unsigned segm = d >= 32 ? kFull : (((1u << d) - 1u) << sstart);
+        const unsigned m = __match_any_sync(kFull, lab) & segm;
+        k = __popc(m);
+        if (VAR == V_LLP) first = (m & ((1u << lane) - 1u)) == 0u;
+      } else {
 #pragma unroll 4
-      for (int i = 0; i < d; ++i) {
-        const bool eq = __shfl_sync(kFull, lab, sstart + i) == lab;
-        k += eq ? 1u : 0u;
-        if (VAR == V_LLP) first = first && !(eq && sstart + i < lane);
+        for (int i = 0; i < d; ++i) {
+          const bool eq = __shfl_sync(kFull, lab, sstart + i) == lab;
+          k += eq ? 1u : 0u;
+          if (VAR == V_LLP) first = first && !(eq && sstart + i < lane);
+        }
       }
-      const int head = (lane < nv ? lane * d : 0) & 31;  // lane jv takes segment jv
-      Best<VAR> h;
       if (VAR == V_LLP || !GLP_LOW_REDUX) {
         Best<VAR> b;
         if (vote && first) b.observe(k, (unsigned)lab, a, lv);
@@ -576,6 +625,7 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
         const unsigned hl = __shfl_sync(kFull, lmin, head);
         h.key = hk ? (((unsigned long long)hk << 32) | (unsigned long long)(~hl)) : 0ull;
       }
+      }  // counted
       if (lane < nv) update_vertex_pre<VAR>(a, v, d, h.have(), h.label(), r, so, ty);
       if (!more) break;
       u = nu;
@@ -679,7 +729,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       // in this kernel bit 31 of mpred marks a sorted-row candidate
       const bool cand = mono_cand<VAR>(raw, a.pred_cap, mine.d);
       mpred = pred_est(raw, a.pred_prev[il], a.pred_cap) | (cand ? kMonoTried : 0u);
-      ok = row_class(mpred & kPredMask, mine.d, cand) == CLS_W;
+      ok = row_class(mpred & kPredMask, mine.d, cand, a.mono_kernel) == CLS_W;
       if (ok && !a.dense && !a.flag[a.vb + mine.v]) {
         ok = false;
         a.pred_next[il] = raw;  // inactive: carry the prediction forward
@@ -726,6 +776,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       bool next_loaded = false;  // x0/x1 hold the next row's first round
       bool major = false;        // a strict-majority label was observed: the rest of the row cannot change the MFL
       int scanned = 0;           // arcs gathered so far
+      const bool hot = hot_pass(pred & kPredMask, d);
       for (int off = 0; off < d && !over && !major; off += kWRound) {
         scanned = min(d, off + kWRound);
         int4 p0, p1;
@@ -772,15 +823,15 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
             m8[2] = gather_lv(a, v0.z, use_v, mv8[2]); m8[3] = gather_lv(a, v0.w, use_v, mv8[3]);
             m8[4] = gather_lv(a, v1.x, use_v, mv8[4]); m8[5] = gather_lv(a, v1.y, use_v, mv8[5]);
             m8[6] = gather_lv(a, v1.z, use_v, mv8[6]); m8[7] = gather_lv(a, v1.w, use_v, mv8[7]);
-            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v);
+            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v, hot);
           }
         }
         if (kWRound == 256 && d - off > 128) {  // warp-uniform
-          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v);
+          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v, hot);
         } else {
           const int l4[4] = {l[0], l[1], l[2], l[3]};
           const int v4[4] = {lv[0], lv[1], lv[2], lv[3]};
-          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v);
+          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v, hot);
         }
         __syncwarp();
         over = s_over[wid] != 0;
@@ -822,6 +873,99 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
 }
 
 // ---------------------------------------------------------------------------
+// mfl_mono: the sorted-row fast path alone (t = 1: unique labels L0[u] = u
+// [P:68]), without the W kernel's shared tables, so it runs at full occupancy
+// with two rounds of label gathers in flight per lane (the path is bound by
+// gather latency, not by counting).  One warp per sorted-row candidate of at
+// most kMonoWMax arcs; a row whose labels turn out not to be strictly
+// increasing (unsorted input rows, repeated arcs) is re-queued to the M
+// kernel's redo list, which counts it exactly.
+#ifndef GLP_MONO_MINB
+#define GLP_MONO_MINB 6
+#endif
+constexpr int kMonoBlock = 256;
+template <int VAR>
+__global__ void __launch_bounds__(kMonoBlock, GLP_MONO_MINB) mfl_mono(MflArgs a) {
+  const int lane = threadIdx.x & 31;
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int nwarps = (gridDim.x * blockDim.x) >> 5;
+  Tally ty;
+  for (int base = 0; base < a.n_items; base += nwarps * 32) {
+    const int il = base + lane * nwarps + gw;
+    BinItem mine;
+    mine.start = 0; mine.v = 0; mine.d = 0;
+    bool ok = il < a.n_items;
+    if (ok) {
+      mine = a.items[il];
+      const unsigned raw = a.pred[il];
+      ok = mono_cand<VAR>(raw, a.pred_cap, mine.d) &&
+           row_class(raw & kPredMask, mine.d, true, true) == CLS_MONO;
+      if (ok && !a.dense && !a.flag[a.vb + mine.v]) {
+        ok = false;
+        a.pred_next[il] = raw;
+      }
+    }
+    unsigned todo = __ballot_sync(kFull, ok);
+    bool rdone = false;
+    unsigned long long rkey = 0ull;
+    unsigned rlab = kNoLabel, rpred = 0u;
+    while (todo) {
+      const int jl = __ffs(todo) - 1;
+      todo &= todo - 1;
+      const int64_t start = __shfl_sync(kFull, mine.start, jl);
+      const int d = __shfl_sync(kFull, mine.d, jl);
+      Best<VAR> b;
+      unsigned fresh = 0;
+      int prev = -1;
+      bool sorted = true;
+      // round r's labels in l[], round r+1's gathers in flight in nl[]
+      int4 x = make_int4(-1, -1, -1, -1);
+      if (4 * lane < d) x = ld_stream4(a.col + start + 4 * lane);
+      int l[4] = {gather(a, x.x), gather(a, x.y), gather(a, x.z), gather(a, x.w)};
+      for (int off = 0; off < d; off += 128) {
+        int nl[4] = {-1, -1, -1, -1};
+        if (off + 128 < d) {
+          int4 y = make_int4(-1, -1, -1, -1);
+          if (off + 128 + 4 * lane < d) y = ld_stream4(a.col + start + off + 128 + 4 * lane);
+          nl[0] = gather(a, y.x); nl[1] = gather(a, y.y); nl[2] = gather(a, y.z); nl[3] = gather(a, y.w);
+        }
+        int end = -1;
+        if (!warp_quads_increasing(l, off, d, prev, &end)) {
+          sorted = false;
+          break;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          if (l[j] >= 0) { b.observe(1u, (unsigned)l[j], a); ++fresh; }  // (t = 1: V == 1, v_ones)
+        prev = end;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) l[j] = nl[j];
+      }
+      if (!sorted) {
+        if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = base + jl * nwarps + gw;
+        continue;
+      }
+      b.warp_reduce();
+      fresh = __reduce_add_sync(kFull, fresh);
+      if (lane == jl) {
+        rdone = true;
+        rkey = b.key;
+        rlab = b.lab;
+        rpred = max(fresh, 1u) | kMonoTried;
+      }
+    }
+    if (rdone) {
+      Best<VAR> r;
+      r.key = rkey;
+      r.lab = rlab;
+      a.pred_next[il] = rpred;
+      update_vertex<VAR>(a, mine.v, mine.d, r.have(), r.label(), ty, mine.d);
+    }
+  }
+  tally_flush(ty, a.cnt);
+}
+
+// ---------------------------------------------------------------------------
 // Block-per-vertex counting of one row into `tab` (UNROLL 128-bit loads per
 // thread in flight).  Only labels of hash partition `part` of `nparts` vote
 // (multi-pass counting of rows with more distinct labels than the table
@@ -848,7 +992,8 @@ template <int VAR, int BLOCK, int UNROLL, bool IPF>
 __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int d, const Table& tab,
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
                                             volatile int* overflow, int* distinct, Best<VAR>& b,
-                                            volatile int* major, unsigned fparts = 1u, int* scanned = nullptr) {
+                                            volatile int* major, unsigned fparts = 1u, int* scanned = nullptr,
+                                            bool hot = true) {
   constexpr int STEP = BLOCK * 4 * UNROLL;
   unsigned fresh = 0;
   int base = 0;
@@ -877,7 +1022,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
     }
-    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v);
+    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot);
     if (GLP_MAJORITY && VAR != V_LLP && major != nullptr && base + STEP < d) {
       // a strict-majority observation ends the row for every warp (they poll the flag)
       const bool m = strict_majority(b, d);
@@ -988,7 +1133,7 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
       if (fparts > 1u && lab[k] >= 0 && label_part((unsigned)lab[k], fparts) != part) lab[k] = -1;
     }
     const int nov[4] = {-1, -1, -1, -1};
-    fresh += warp_insert_n<VAR, 4>(a, tab, max_probe, lab, b, overflow, nov, false);
+    fresh += warp_insert_n<VAR, 4>(a, tab, max_probe, lab, b, overflow, nov, false, GLP_HOT_DIV == 0);
     if (__any_sync(kFull, *overflow != 0)) break;
   }
   fresh = __reduce_add_sync(kFull, fresh);
@@ -1059,7 +1204,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
         pe = pred_est(raw, a.pred_prev[ik], a.pred_cap);
         cnd = mono_cand<VAR>(raw, a.pred_cap, itk.d);
         if (!a.mode) {
-          ok = row_class(pe, itk.d, cnd) == CLS;
+          ok = row_class(pe, itk.d, cnd, a.mono_kernel) == CLS;
           if (ok && !a.dense && !a.flag[a.vb + itk.v]) {
             ok = false;
             a.pred_next[ik] = raw;  // inactive: carry the prediction forward
@@ -1130,7 +1275,8 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       const bool may_over = PART && 2u * (unsigned)d > (unsigned)SLOTS;
       block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : (PART ? tsz : kTabProbe), cur,
                                       (GLP_L_STAGE1 && may_over) ? stageA : nullptr, &s_over, &s_distinct, b,
-                                      (may_over && !GLP_L_MAJ) ? nullptr : &s_major, 1u, &s_scan);
+                                      (may_over && !GLP_L_MAJ) ? nullptr : &s_major, 1u, &s_scan,
+                                      hot_pass(est, d));
       __syncthreads();
       over = s_over != 0;
       if (!over && a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
@@ -1171,7 +1317,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
             if (gather_pass) {
               block_load_round<BLOCK, UNROLL>(a.col, it.start, d, 0, cur);
               block_count<VAR, BLOCK, UNROLL, GLP_L_IPF>(a, it.start, d, tab, kLProbe, cur, stageA, &s_over,
-                                                         &s_distinct, b, nullptr, nparts);
+                                                         &s_distinct, b, nullptr, nparts, nullptr, GLP_HOT_DIV == 0);
             } else {
               count_staged<VAR, BLOCK>(a, stageA, d, tab, kLProbe, &s_over, &s_distinct, b, nparts, p);
             }

@@ -109,7 +109,10 @@ def test_explicit_uneven_bounds_and_empty_slice():
 
 
 def test_group_ranks_agree_with_single_gpu_stats():
-    """Per-iteration active vertices and changes summed over ranks equal the 1-GPU run's."""
+    """Iterations and per-iteration changes of a 4-rank run equal the 1-GPU
+    run's.  (Scanned vertices and arcs may differ: a low-degree chunk is
+    scanned whole when any of its vertices is active, and chunks are packed
+    per rank; a block stops on a strict majority when its warps poll.)"""
     csr = graphs.rmat(13, seed=21)
     c = csr.to("cuda")
     with glp.Graph(c) as g:
@@ -117,10 +120,8 @@ def test_group_ranks_agree_with_single_gpu_stats():
         st1 = g.iter_stats()
     labs, infos, st, ks, b = run_group(c, 4, "classic", 20)
     assert infos[0].iterations == info1.iterations
-    # (active arcs can differ by a few: a block stops on a strict majority when
-    # its warps poll the flag, so the rounds read past it vary run to run)
-    assert [s["active_vertices"] for s in st[0]] == [s["active_vertices"] for s in st1]
     assert [s["changed"] for s in st[0]] == [s["changed"] for s in st1]
+    assert [s["dense"] for s in st[0]] == [s["dense"] for s in st1]
 
 
 def test_failed_rank_releases_group():
