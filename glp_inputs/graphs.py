@@ -240,6 +240,13 @@ def _trunc_powerlaw_quantiles(count: int, alpha: float, lo: float, hi: float, de
     return (a + q * (b - a)) ** (1.0 / e)
 
 
+def _cdf(w: torch.Tensor):
+    """Normalised running sum of w, accumulated sequentially (numpy)."""
+    import numpy as np
+    c = np.cumsum(w.numpy())
+    return c / c[-1]
+
+
 def taobao(users: int = 80_000_000, items: int = 20_000_000, pairs: int = 1_000_000_000,
            rings: int = 10_000, ring_users: int = 20, ring_items: int = 5,
            seeds_per_ring: int = 4, seed_frac: float = 0.001, seed: int = 7,
@@ -255,13 +262,11 @@ def taobao(users: int = 80_000_000, items: int = 20_000_000, pairs: int = 1_000_
     ``seed_frac`` of all users.  Returns (CSR, seeds int32 tensor).
     """
     n = users + items
-    wu = _trunc_powerlaw_quantiles(users, 2.5, 1.0, 2000.0, device).flip(0)
-    wi = _trunc_powerlaw_quantiles(items, 2.0, 1.0, 5e6, device).flip(0)
-    cu = torch.cumsum(wu, 0)
-    cu /= cu[-1].clone()
-    ci = torch.cumsum(wi, 0)
-    ci /= ci[-1].clone()
-    del wu, wi
+    # the inverse-CDF tables are built on the host (sequential float64
+    # cumsum): a parallel device scan rounds in a run-dependent order, which
+    # made the 100M-vertex graph differ from run to run
+    cu = torch.from_numpy(_cdf(_trunc_powerlaw_quantiles(users, 2.5, 1.0, 2000.0, "cpu").flip(0))).to(device)
+    ci = torch.from_numpy(_cdf(_trunc_powerlaw_quantiles(items, 2.0, 1.0, 5e6, "cpu").flip(0))).to(device)
     srcs, dsts = [], []
     for s0 in range(0, pairs, chunk):
         s1 = min(pairs, s0 + chunk)

@@ -63,10 +63,22 @@ __global__ void k_init_seeds(const int32_t* __restrict__ seeds, int64_t ns, cons
 // Frontier push: for every owned vertex changed at iteration t (so.x == t),
 // mark itself and its neighbours (global ids) active for t+1 (DESIGN.md
 // §Frontier: marking the changed vertex itself keeps the unconditional-write
-// invariant).  One warp scans 32 stamps, then walks each changed row.
+// invariant).  One warp scans 32 stamps, then walks each changed row; rows of
+// at least kPushBig arcs are only listed, and k_push_big spreads each of them
+// over the whole grid (a changed hub -- TaoBao's 10.9M-arc item -- would
+// otherwise keep one warp busy for milliseconds).
+constexpr int kPushBig = 8192;
+// GLP_PUSH_CHECK: read a mark before writing it (most marks of a large push
+// are already set: a read costs less than a partial-sector write)
+#ifndef GLP_PUSH_CHECK
+#define GLP_PUSH_CHECK 1
+#endif
+__device__ __forceinline__ void mark(uint8_t* flag, int32_t x) {
+  if (!GLP_PUSH_CHECK || !flag[x]) flag[x] = 1;
+}
 __global__ void k_push(const int64_t* __restrict__ ioff, const int32_t* __restrict__ ideg,
                        const int32_t* __restrict__ col2, const int2* __restrict__ so, int64_t nl, int64_t vb,
-                       int32_t t, uint8_t* __restrict__ flag) {
+                       int32_t t, uint8_t* __restrict__ flag, int32_t* __restrict__ big, unsigned* __restrict__ n_big) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -74,14 +86,31 @@ __global__ void k_push(const int64_t* __restrict__ ioff, const int32_t* __restri
     const int64_t v = base + lane;
     const bool ch = v < nl && so[v].x == t;
     unsigned m = __ballot_sync(0xffffffffu, ch);
+    if (ch) flag[vb + v] = 1;
+    const bool isbig = ch && ideg[v] >= kPushBig;
+    if (isbig) big[atomicAdd(n_big, 1u)] = (int32_t)v;
+    m &= ~__ballot_sync(0xffffffffu, isbig);
     while (m) {
       const int j = __ffs(m) - 1;
       m &= m - 1;
       const int64_t u = base + j;
-      if (lane == 0) flag[vb + u] = 1;
       const int64_t e0 = ioff[u], e1 = e0 + ideg[u];
-      for (int64_t e = e0 + lane; e < e1; e += 32) flag[col2[e]] = 1;  // global ids
+      for (int64_t e = e0 + lane; e < e1; e += 32) mark(flag, col2[e]);  // global ids
     }
+  }
+}
+// the listed long rows: every thread of the grid takes a stride of each row
+__global__ void k_push_big(const int64_t* __restrict__ ioff, const int32_t* __restrict__ ideg,
+                           const int32_t* __restrict__ col2, const int32_t* __restrict__ big,
+                           const unsigned* __restrict__ n_big, uint8_t* __restrict__ flag) {
+  const unsigned nb = *n_big;
+  const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+  for (unsigned i = 0; i < nb; ++i) {
+    const int32_t u = big[i];
+    const int64_t e0 = ioff[u];
+    const int32_t d = ideg[u];
+    for (int64_t e = tid; e < d; e += nth) mark(flag, col2[e0 + e]);
   }
 }
 

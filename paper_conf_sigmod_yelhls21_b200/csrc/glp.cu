@@ -572,7 +572,11 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->grid_m = grid_for(sms, (const void*)GLP_M_KERNEL(V_LLP), kMBlock, ms_);
     g->grid_mono = grid_for(sms, (const void*)mfl_mono<V_LLP>, kMonoBlock, 0);
     g->grid_l = grid_for(sms, (const void*)GLP_L_KERNEL(V_LLP), kLBlock, ls_);
-    g->grid_g = grid_for(sms, (const void*)mfl_giant_count<V_LLP>, kGBlock, 0);
+    const int gs_ = GLP_GIANT_SMEM ? kGSlots * 8 : 0;
+    CK(cudaFuncSetAttribute(mfl_giant_count<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
+    CK(cudaFuncSetAttribute(mfl_giant_count<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
+    CK(cudaFuncSetAttribute(mfl_giant_count<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
+    g->grid_g = grid_for(sms, (const void*)mfl_giant_count<V_LLP>, kGBlock, gs_);
     g->grid_aux = sms * 8;
     if (g->n_rows > 0) {
       // L staging: two row-sized buffers per resident L block, in two regions:
@@ -634,6 +638,20 @@ void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t&
 }
 
 // ---------------------------------------------------------------- run
+// frontier push of the vertices changed at t (k_push + its long-row pass)
+void push(glp_graph* g, int32_t t, uint8_t* flag) {
+  cudaStream_t s = g->stream;
+  if (!g->push_big) {
+    g->push_big = dalloc<int32_t>(g, std::max<int64_t>(g->nl, 1));
+    g->push_nbig = dalloc<unsigned>(g, 1);
+  }
+  CK(cudaMemsetAsync(g->push_nbig, 0, sizeof(unsigned), s));
+  k_push<<<g->grid_aux, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, flag, g->push_big,
+                                     g->push_nbig);
+  if (g->max_deg >= kPushBig) k_push_big<<<g->sms * 4, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->push_big, g->push_nbig, flag);
+  CK(cudaGetLastError());
+}
+
 template <int VAR>
 int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, size_t& used) {
   Counters* c = g->d_cnt;
@@ -666,7 +684,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     b.gsegs = g->gsegs; b.n_gsegs = g->n_gsegs; b.gtab = g->gtab; b.gtab_off = g->gtab_off;
     b.gcand_key = g->gcand_key; b.gcand_lab = g->gcand_lab; b.gdistinct = g->gdistinct; b.epoch = g->gepoch;
     timed(g, prof, 7, pend, used, cc ? g->xs[0] : s0, [&] {
-      mfl_giant_count<VAR><<<std::min(g->grid_g, g->n_gsegs), kGBlock, 0, S(0)>>>(b);
+      mfl_giant_count<VAR><<<std::min(g->grid_g, g->n_gsegs), kGBlock, GLP_GIANT_SMEM ? kGSlots * 8 : 0, S(0)>>>(b);
       mfl_giant_finish<VAR><<<g->n_giant, 256, 0, S(0)>>>(b, g->gseg_first);
     });
     n += 2;
@@ -810,8 +828,8 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   if (variant == GLP_VARIANT_SEEDED) {
     // frontier of t = 1 is N(S) (+ S): push from the seeds (stamped t = 0)
     if (use_frontier) {
-      k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, 0, g->flag[fb]);
-      g->init_launches += 1;
+      push(g, 0, g->flag[fb]);
+      g->init_launches += g->max_deg >= kPushBig ? 2 : 1;
       CK(cudaGetLastError());
       g->flag_clean[fb] = false;
       if (g->comm) g->comm->merge_flags(g, g->flag[fb]);
@@ -931,9 +949,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     if (!last && use_frontier)
       next_dense = (double)tot.chdeg * (double)p.dense_divisor > (double)g->nnz_global;
     if (!last && !next_dense) {
-      launches += 1;
+      launches += g->max_deg >= kPushBig ? 2 : 1;
       timed(g, prof, 4, pend, used, s, [&] {
-        k_push<<<ga, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, g->flag[nf]);
+        push(g, t, g->flag[nf]);
         if (g->comm) g->comm->merge_flags(g, g->flag[nf]);
         if (g->n_chunks)
           k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_base, g->flag[nf], g->vb, g->cflag);

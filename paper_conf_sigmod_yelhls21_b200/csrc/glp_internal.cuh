@@ -261,6 +261,8 @@ struct glp_graph {
   int pb = 0;                                        // pred[pb] is read this iteration
   int32_t* redo_m = nullptr;                         // [n_rows]
   int32_t* redo_l = nullptr;                         // [n_rows]
+  int32_t* push_big = nullptr;                       // [nl] changed rows of >= kPushBig arcs (push)
+  unsigned* push_nbig = nullptr;
   glp::Sched* d_sched = nullptr;
   int64_t bin_verts[glp::NBINS] = {0}, bin_arcs[glp::NBINS] = {0};
 

@@ -82,3 +82,15 @@ def test_rmat_bucketed_build_matches_plain():
             b = graphs.rmat(scale, seed=1, buckets=buckets)
             assert torch.equal(a.row_offsets, b.row_offsets)
             assert torch.equal(a.col_idx, b.col_idx)
+
+
+@pytest.mark.gpu
+def test_taobao_generation_repeatable_on_gpu():
+    """Two generations of a mid-size TaoBao window are identical (the
+    inverse-CDF tables once came from a device float scan whose rounding
+    order varied run to run)."""
+    import torch
+    a, sa = graphs.taobao(users=20_000_000, items=5_000_000, pairs=40_000_000, rings=100, device="cuda")
+    b, sb = graphs.taobao(users=20_000_000, items=5_000_000, pairs=40_000_000, rings=100, device="cuda")
+    assert torch.equal(a.row_offsets, b.row_offsets) and torch.equal(a.col_idx, b.col_idx)
+    assert torch.equal(sa, sb)

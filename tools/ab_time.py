@@ -29,15 +29,19 @@ flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device="cuda")
 stream = torch.cuda.current_stream()
 for _ in range(3):
     g.run(variant, max_iters, seeds, gamma=gamma)
-ms, its = [], []
+ms, its, shas = [], [], set()
 for _ in range(reps):
     flush.fill_(1)
     info = g.run(variant, max_iters, seeds, gamma=gamma)
     ms.append(info.elapsed_ms)
     its.append([round(s["ms"], 3) for s in g.iter_stats()])
+    shas.add(hashlib.sha1(g.labels("cpu").numpy().tobytes()).hexdigest()[:12])
 lab = g.labels("cpu").numpy()
+w = (torch.arange(csr.col_idx.numel(), device="cuda", dtype=torch.int64) % 1000003) + 1
+graph_sum = int((csr.col_idx.to(torch.int64) * w).sum()) ^ int(csr.row_offsets.sum())
 med = statistics.median(ms)
 i = ms.index(sorted(ms)[len(ms) // 2])
 print(json.dumps({"lib": os.environ.get("GLP_LIB", "in-tree"), "workload": wl, "median_ms": round(med, 3),
                   "min_ms": round(min(ms), 3), "iterations": info.iterations, "iter_ms": its[i],
-                  "labels_sha": hashlib.sha1(lab.tobytes()).hexdigest()[:12]}), flush=True)
+                  "labels_sha": hashlib.sha1(lab.tobytes()).hexdigest()[:12], "distinct_runs": len(shas),
+                  "graph_sum": graph_sum}), flush=True)
