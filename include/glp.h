@@ -137,7 +137,16 @@ typedef struct {
                                   own rows, the counts are all-reduced, and the
                                   (label, V) pairs of the owned rows are
                                   all-gathered instead of the labels)          */
-  int32_t reserved[5];
+  int32_t host_arcs;           /* create only.  1: CPU-GPU hybrid mode for
+                                  graphs whose arcs exceed device memory
+                                  [P:103]: the library's arc array lives in
+                                  pinned, mapped HOST memory and every
+                                  iteration streams it over the host link;
+                                  labels, counters and tables stay on the
+                                  device.  Needs a host CSR (on_device = 0),
+                                  whose col_idx is registered (pinned) during
+                                  create.  Results are identical.  Default 0 */
+  int32_t reserved[4];
 } glp_params;
 
 typedef struct {

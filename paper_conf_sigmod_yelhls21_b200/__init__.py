@@ -56,7 +56,7 @@ class glp_params(ctypes.Structure):
                 ("frontier", ctypes.c_int32), ("stop_on_2cycle", ctypes.c_int32),
                 ("validate", ctypes.c_int32), ("profile", ctypes.c_int32),
                 ("dense_divisor", ctypes.c_int32), ("debug_pred_cap", ctypes.c_int32),
-                ("llp_hist", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5)]
+                ("llp_hist", ctypes.c_int32), ("host_arcs", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
 
 
 class glp_run_info(ctypes.Structure):
@@ -126,7 +126,7 @@ def _check(st: int):
 
 def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = True,
                 validate: bool = True, profile: bool = False, dense_divisor: int = 0,
-                debug_pred_cap: int = 0, llp_hist: int = 0) -> glp_params:
+                debug_pred_cap: int = 0, llp_hist: int = 0, host_arcs: bool = False) -> glp_params:
     p = glp_params()
     p.struct_size = ctypes.sizeof(glp_params)
     p.gamma = float(gamma)
@@ -137,6 +137,7 @@ def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = T
     p.dense_divisor = int(dense_divisor)
     p.debug_pred_cap = int(debug_pred_cap)
     p.llp_hist = int(llp_hist)
+    p.host_arcs = int(bool(host_arcs))
     return p
 
 
@@ -163,7 +164,7 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
                      v_begin: int = 0, v_end: int | None = None, symmetric: bool = False,
                      rank: int = 0, nranks: int = 1, device: int | None = None,
                      nccl_unique_id: bytes | None = None, stream: torch.cuda.Stream | None = None,
-                     validate: bool = True, local_group=None):
+                     validate: bool = True, local_group=None, host_arcs: bool = False):
     """Create a device graph.  CUDA tensors are borrowed (keep them alive);
     CPU tensors are copied.  Returns an opaque handle (ctypes.c_void_p)."""
     lib = load_library()
@@ -201,7 +202,7 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
         # complete (torch may still be producing them on its current stream)
         torch.cuda.current_stream(row_offsets.device).synchronize()
     h = ctypes.c_void_p()
-    prm = make_params(validate=validate)
+    prm = make_params(validate=validate, host_arcs=host_arcs)
     st = lib.glp_graph_create(ctypes.byref(c), None if d is None else ctypes.byref(d), ctypes.byref(prm),
                               ctypes.byref(h))
     if st == 3 and torch.cuda.is_available():

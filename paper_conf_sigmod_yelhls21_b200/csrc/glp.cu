@@ -187,6 +187,8 @@ void free_graph(glp_graph* g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   g->allocs.clear();
   if (g->h_cnt) cudaFreeHost(g->h_cnt);
+  if (g->col2_host) cudaFreeHost(g->col2_host);
+  if (g->registered) cudaHostUnregister(g->registered);
   if (g->ev_a) cudaEventDestroy(g->ev_a);
   if (g->ev_b) cudaEventDestroy(g->ev_b);
   for (auto& e : g->ev_pool) cudaEventDestroy(e);
@@ -393,8 +395,25 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     CK(cudaStreamSynchronize(s));
     if (bad & 8) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
   }
-  g->col2 = dalloc<int32_t>(g, g->nnz2);
-  CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), s));  // padding = -1
+  if (g->host_arcs) {
+    // hybrid mode [P:103]: the bin-major arc array lives in pinned, mapped
+    // host memory; the MFL kernels stream it over the host link (labels,
+    // counters and tables stay in HBM)
+    void* hp = nullptr;
+    const size_t bytes = std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t);
+    if (cudaHostAlloc(&hp, bytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      fail(GLP_ERR_OUT_OF_MEMORY, "pinned host allocation of the arc array failed");
+    }
+    g->col2_host = hp;
+    memset(hp, 0xff, bytes);  // padding = -1
+    void* dp = nullptr;
+    CK(cudaHostGetDevicePointer(&dp, hp, 0));
+    g->col2 = (int32_t*)dp;
+  } else {
+    g->col2 = dalloc<int32_t>(g, g->nnz2);
+    CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), s));  // padding = -1
+  }
   if (nl > 0 && g->nnz > 0) {
     k_relayout<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, g->pos, nl, g->vb, g->col2);
     CK(cudaGetLastError());
@@ -459,6 +478,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->nl = g->ve - g->vb;
     g->nnz = csr->nnz_local;
     g->symmetric = csr->symmetric ? 1 : 0;
+    g->host_arcs = p.host_arcs != 0;
+    if (g->host_arcs && csr->on_device) fail(GLP_ERR_INVALID_ARGUMENT, "host_arcs needs a host CSR (on_device = 0)");
     if (g->nnz >= ((int64_t)1 << 40)) fail(GLP_ERR_INVALID_ARGUMENT, "nnz_local too large");
 
     g->sms = prop.multiProcessorCount;
@@ -470,6 +491,31 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     if (csr->on_device) {
       off_d = csr->row_offsets;
       col_d = csr->col_idx;
+    } else if (g->host_arcs) {
+      // hybrid mode: the caller's arcs stay in host memory (registered and
+      // mapped for the relayout, which reads them over the host link); only
+      // the offsets are staged on the device
+      void* po = nullptr;
+      if (pool_malloc(&po, (g->nl + 1) * sizeof(int64_t), g->stream) != cudaSuccess) {
+        cudaGetLastError();
+        fail(GLP_ERR_OUT_OF_MEMORY, "staging the row offsets on the device failed");
+      }
+      temps.push_back(po);
+      CK(cudaMemcpyAsync(po, csr->row_offsets, (g->nl + 1) * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
+      off_d = (const int64_t*)po;
+      if (g->nnz) {
+        void* hp = (void*)csr->col_idx;
+        void* dp = nullptr;
+        // already pinned (cudaHostAlloc / registered by the caller): mapped
+        // under UVA as it is; otherwise register it for the create
+        if (cudaHostGetDevicePointer(&dp, hp, 0) != cudaSuccess) {
+          cudaGetLastError();
+          CK(cudaHostRegister(hp, g->nnz * sizeof(int32_t), cudaHostRegisterMapped | cudaHostRegisterReadOnly));
+          g->registered = hp;
+          CK(cudaHostGetDevicePointer(&dp, hp, 0));
+        }
+        col_d = (const int32_t*)dp;
+      }
     } else {
       void *po = nullptr, *pc = nullptr;
       if (pool_malloc(&po, (g->nl + 1) * sizeof(int64_t), g->stream) != cudaSuccess ||
@@ -493,7 +539,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaMemsetAsync(dbad, 0, 2 * sizeof(int), g->stream));
     CK(cudaEventRecord(g->xev[0], g->stream));
     CK(cudaStreamWaitEvent(g->xs[0], g->xev[0], 0));
-    if (!csr->on_device && g->nnz)
+    if (!csr->on_device && !g->host_arcs && g->nnz)
       CK(cudaMemcpyAsync((void*)col_d, csr->col_idx, g->nnz * sizeof(int32_t), cudaMemcpyHostToDevice, g->xs[0]));
     if (p.validate && g->nnz) k_validate_col<<<g->sms * 4, 256, 0, g->xs[0]>>>(col_d, g->nnz, g->n, dbad + 1);
     CK(cudaGetLastError());
@@ -531,6 +577,11 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     else if (nranks > 1 || (dist && dist->nccl_unique_id)) g->comm = new NcclComm(g, dist->nccl_unique_id);
     if (g->comm) g->comm->setup(g);
     build_layout(g, off_d, col_d);
+    if (g->registered) {  // the caller's arcs are not read after the relayout
+      CK(cudaStreamSynchronize(g->stream));
+      cudaHostUnregister(g->registered);
+      g->registered = nullptr;
+    }
 
     g->L[0] = dalloc<int32_t>(g, npad);
     g->L[1] = dalloc<int32_t>(g, npad);

@@ -232,6 +232,9 @@ struct glp_graph {
   const int64_t* off = nullptr;
   const int32_t* col = nullptr;
   bool own_csr = false;
+  bool host_arcs = false;       // hybrid mode: col2 in pinned mapped host memory
+  void* col2_host = nullptr;    // its host allocation
+  void* registered = nullptr;   // caller's host arcs registered during create
   int symmetric = 1;
   int64_t max_deg = 0;
 
