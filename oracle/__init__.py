@@ -46,6 +46,9 @@ def _load():
         lib.glp_oracle_step.restype = ctypes.c_int
         lib.glp_oracle_step.argtypes = [ctypes.c_int64, P, P, ctypes.c_int32, P, P, P, ctypes.c_double,
                                         ctypes.c_int64, ctypes.c_int64, P, ctypes.c_int32]
+        lib.glp_oracle_run_w.restype = ctypes.c_int
+        lib.glp_oracle_run_w.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, ctypes.c_int32, P,
+                                         ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, P, P, P, P]
         lib.glp_oracle_modularity.restype = ctypes.c_double
         lib.glp_oracle_modularity.argtypes = [ctypes.c_int64, P, P, P]
         _lib = lib
@@ -98,6 +101,32 @@ def run(csr, variant: int = CLASSIC, max_iters: int = 20, seeds=None, gamma: flo
                             _ptr(changed), _ptr(tr), _ptr(info))
     if rc != 0:
         raise ValueError(f"glp_oracle_run failed rc={rc}")
+    it = int(info[0])
+    return OracleResult(labels[:n].copy(), changed[:it].copy(), it, int(info[1]),
+                        None if tr is None else tr[:it, :n].copy())
+
+
+def run_weighted(csr, weights, variant: int = CLASSIC, max_iters: int = 20, seeds=None,
+                 stop_on_2cycle: bool = True, threads: int = 1, trace: bool = False) -> OracleResult:
+    """Weighted LP (label frequency = sum of arc weights), CLASSIC/SEEDED."""
+    lib = _load()
+    n, off, col = _csr_np(csr)
+    w = np.ascontiguousarray(np.asarray(weights.cpu().numpy() if hasattr(weights, "cpu") else weights,
+                                        dtype=np.uint32))
+    assert w.size == col.size
+    labels = np.empty(max(n, 1), dtype=np.int32)
+    changed = np.zeros(max(max_iters, 1), dtype=np.int64)
+    tr = np.empty((max(max_iters, 1), max(n, 1)), dtype=np.int32) if trace else None
+    info = np.zeros(2, dtype=np.int32)
+    sd, ns = None, 0
+    if seeds is not None:
+        sd = np.ascontiguousarray(np.asarray(seeds, dtype=np.int32))
+        ns = int(sd.size)
+    rc = lib.glp_oracle_run_w(n, _ptr(off), _ptr(col), _ptr(w), int(variant), int(max_iters), _ptr(sd), ns,
+                              int(bool(stop_on_2cycle)), int(threads), _ptr(labels), _ptr(changed), _ptr(tr),
+                              _ptr(info))
+    if rc != 0:
+        raise ValueError(f"glp_oracle_run_w failed rc={rc}")
     it = int(info[0])
     return OracleResult(labels[:n].copy(), changed[:it].copy(), it, int(info[1]),
                         None if tr is None else tr[:it, :n].copy())
