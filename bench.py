@@ -57,6 +57,9 @@ WORKLOADS = {
     "rmat24_hostarcs": (dict(kind="rmat", scale=24, edge_factor=16, seed=1), "classic", 20, 0.0),
 }
 HOST_ARCS = {"rmat24_hostarcs"}
+# §8(f)3 weighted LP: RMAT-24 with symmetric integer arc weights in [1, 8]
+WORKLOADS["rmat24_weighted"] = (dict(kind="rmat", scale=24, edge_factor=16, seed=1), "classic", 20, 0.0)
+WEIGHTED = {"rmat24_weighted"}
 
 
 def host_link_gbs(dev) -> float:
@@ -145,7 +148,14 @@ def make_graph(spec, device):
     return csr, seeds
 
 
-def cpu_reference(csr_cpu, variant, seeds, gamma, iters_per_sample, reps, warmup=0):
+def workload_weights(name, csr):
+    if name not in WEIGHTED:
+        return None
+    from glp_inputs import graphs
+    return graphs.edge_weights(csr, seed=5, hi=8)
+
+
+def cpu_reference(csr_cpu, variant, seeds, gamma, iters_per_sample, reps, warmup=0, weights=None):
     """Time the CPU oracle (as it stands) on the host cores: `reps` samples of
     `iters_per_sample` LP iterations from PickLabel."""
     import oracle
@@ -154,8 +164,12 @@ def cpu_reference(csr_cpu, variant, seeds, gamma, iters_per_sample, reps, warmup
     times = []
     for r in range(warmup + reps):
         t0 = time.perf_counter()
-        res = oracle.run(csr_cpu, vid, iters_per_sample, seeds=None if seeds is None else seeds.cpu().numpy(),
-                         gamma=gamma, threads=threads)
+        sd = None if seeds is None else seeds.cpu().numpy()
+        if weights is not None:
+            res = oracle.run_weighted(csr_cpu, weights.cpu().numpy().astype("uint32"), vid, iters_per_sample,
+                                      seeds=sd, threads=threads)
+        else:
+            res = oracle.run(csr_cpu, vid, iters_per_sample, seeds=sd, gamma=gamma, threads=threads)
         dt = time.perf_counter() - t0
         if r >= warmup:
             times.append((dt, res.iterations))
@@ -235,6 +249,7 @@ def bench_gpu(args):
     t_gen = time.perf_counter() - t_gen
     n, nnz = csr.n, csr.nnz
     stream = torch.cuda.current_stream()
+    wts = workload_weights(args.workload, csr)
 
     # torch's cache of the generator's temporaries (~139 GB after TaoBao) is
     # released, so the library's memory pool can keep a whole graph mapped
@@ -255,7 +270,7 @@ def bench_gpu(args):
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             g2 = glp.Graph(n=n, row_offsets=off_h, col_idx=col_h, symmetric=csr.symmetric, stream=stream,
-                           host_arcs=args.workload in HOST_ARCS)
+                           host_arcs=args.workload in HOST_ARCS, weights=None if wts is None else wts.cpu())
             t1 = time.perf_counter()
             ri = g2.run(variant, max_iters, seeds_h, gamma=gamma)
             t2 = time.perf_counter()
@@ -268,7 +283,8 @@ def bench_gpu(args):
                 e2e_arcs += ri.arcs_processed
                 phases.append(((t1 - t0) * 1e3, (t2 - t1) * 1e3, (t3 - t2) * 1e3))
         e2e = {"value": round(e2e_arcs / (sum(e2e_ms) / 1e3) / 1e9, 3), "unit": UNIT,
-               "h2d_bytes_per_step": int((n + 1) * 8 + nnz * 4 + (0 if seeds is None else 4 * seeds.numel())),
+               "h2d_bytes_per_step": int((n + 1) * 8 + nnz * 4 + (0 if seeds is None else 4 * seeds.numel())
+                                         + (0 if wts is None else 4 * nnz)),
                "d2h_bytes_per_step": int(4 * n), "ms_per_step": round(statistics.mean(e2e_ms), 3),
                "includes": "graph create (H2D copy, relayout) + run + labels D2H",
                "phase_ms": {k: round(statistics.mean(p[i] for p in phases), 3)
@@ -284,7 +300,7 @@ def bench_gpu(args):
         if args.workload in HOST_ARCS:
             g = glp.Graph(csr.to("cpu"), device=local, stream=stream, host_arcs=True)
         else:
-            g = glp.Graph(csr, device=local, stream=stream)
+            g = glp.Graph(csr, device=local, stream=stream, weights=wts)
     info = g.info()
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
 
@@ -443,13 +459,14 @@ def bench_gpu(args):
     if rank == 0 and world == 1 and not args.no_cpu:
         csr_cpu = csr.to("cpu")
         samp_iters = 1 if nnz > 50_000_000 else max_iters
-        v, cores, sec, its = cpu_reference(csr_cpu, variant, seeds, gamma, samp_iters, reps=1)
+        v, cores, sec, its = cpu_reference(csr_cpu, variant, seeds, gamma, samp_iters, reps=1, weights=wts)
         out["cpu_baseline"] = {"value": round(v, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
                                "cpu_model": cpu_model(),
                                "sample": f"{args.workload}: first {its} LP iteration(s) from PickLabel, "
                                          f"oracle/glp_oracle.c OpenMP over {cores} threads, {sec:.1f} s "
                                          "(the oracle scans every arc each iteration)",
-                               "sequential": cpu_sequential(csr_cpu, variant, seeds, gamma)}
+                               "sequential": cpu_sequential(csr_cpu, variant, seeds, gamma) if wts is None
+                               else None}
     if rank == 0:
         print(json.dumps(out), flush=True)
     g.close()
@@ -466,18 +483,21 @@ def bench_reference(args):
     spec, variant, max_iters, gamma = WORKLOADS[args.workload]
     dev = "cuda" if torch.cuda.is_available() else "cpu"
     csr, seeds = make_graph(spec, dev)
+    wts = workload_weights(args.workload, csr)
+    wts = None if wts is None else wts.cpu()
     csr_cpu = csr.to("cpu")
     del csr
     seeds = None if seeds is None else seeds.cpu()
     # each step = one whole run of the workload (same config as the GPU arm)
     # when K+W of them fit the budget, else the first `samp` iterations
-    _, _, probe_s, probe_it = cpu_reference(csr_cpu, variant, seeds, gamma, 1, reps=1)
+    _, _, probe_s, probe_it = cpu_reference(csr_cpu, variant, seeds, gamma, 1, reps=1, weights=wts)
     budget_s = float(os.environ.get("GLP_REF_BUDGET_S", "200"))
     per_it = probe_s / max(probe_it, 1)
     samp = max_iters if per_it * max_iters * (args.steps + args.warmup) <= budget_s else \
         max(1, int(budget_s / (per_it * (args.steps + args.warmup))))
     samp = min(samp, max_iters)
-    v, cores, sec, its = cpu_reference(csr_cpu, variant, seeds, gamma, samp, reps=args.steps, warmup=args.warmup)
+    v, cores, sec, its = cpu_reference(csr_cpu, variant, seeds, gamma, samp, reps=args.steps, warmup=args.warmup,
+                                       weights=wts)
     same = samp == max_iters
     out = {"metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": round(sec * 1e3, 2), "higher_is_better": True,

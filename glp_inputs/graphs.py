@@ -350,3 +350,15 @@ def lcg_degrees_hint(csr: CSR) -> dict:
     out["max_degree"] = int(deg.max()) if deg.numel() else 0
     out["log2_n"] = math.log2(max(csr.n, 1))
     return out
+
+
+def edge_weights(csr: CSR, seed: int = 5, hi: int = 8) -> torch.Tensor:
+    """Integer arc weights in [1, hi] (weighted LP, §8(f)3), symmetric: arc
+    (u, v) and arc (v, u) get the same weight (a counter-based hash of the
+    unordered pair).  int32 tensor on the CSR's device."""
+    off = csr.row_offsets
+    deg = off[1:] - off[:-1]
+    rows = torch.repeat_interleave(torch.arange(csr.n, device=off.device), deg)
+    cols = csr.col_idx.to(torch.int64)
+    key = torch.minimum(rows, cols) * csr.n + torch.maximum(rows, cols)
+    return (rng.hash64(seed, 31, key) % hi + 1).to(torch.int32)

@@ -90,6 +90,15 @@ typedef struct {
                                   symmetric (u in N(v) <=> v in N(u)); the
                                   frontier push then walks the CSR itself.
                                   0: the frontier is disabled (full sweeps)    */
+  const uint32_t *weights;     /* NULL, or nnz_local arc weights in [1, 2^31)
+                                  (LoadNeighbor's weight [P:110, P:145]): a
+                                  label's frequency is the SUM of the weights
+                                  of the arcs carrying it (weighted LP,
+                                  CLASSIC / SEEDED; LLP -> UNSUPPORTED).
+                                  Same memory space as col_idx; copied into
+                                  the library's layout during create.  Every
+                                  row's weight total must be < 2^31
+                                  (GLP_ERR_INVALID_GRAPH otherwise)            */
 } glp_csr;
 
 /* In-process rank group: P ranks (P graphs, one host thread each) in ONE
@@ -228,6 +237,11 @@ glp_status glp_kernel_stats(const glp_graph *g, glp_kernel_stat *out, int32_t ma
 glp_status glp_graph_info(const glp_graph *g, int64_t *out, int32_t max_entries);
 
 glp_status glp_graph_destroy(glp_graph *g); /* NULL-safe */
+
+/* ABI self-check for bindings: out[0..5] = sizeof(glp_csr), sizeof(glp_dist),
+ * sizeof(glp_params), sizeof(glp_run_info), sizeof(glp_iter_stat),
+ * sizeof(glp_kernel_stat) (at most max_entries written).  Host only. */
+glp_status glp_struct_sizes(int64_t *out, int32_t max_entries);
 
 const char *glp_last_error(void);  /* thread-local, never NULL */
 const char *glp_version(void);

@@ -42,7 +42,7 @@ class glp_csr(ctypes.Structure):
     _fields_ = [("n_global", ctypes.c_int64), ("v_begin", ctypes.c_int64), ("v_end", ctypes.c_int64),
                 ("nnz_local", ctypes.c_int64), ("row_offsets", ctypes.c_void_p),
                 ("col_idx", ctypes.c_void_p), ("on_device", ctypes.c_int32),
-                ("symmetric", ctypes.c_int32)]
+                ("symmetric", ctypes.c_int32), ("weights", ctypes.c_void_p)]
 
 
 class glp_dist(ctypes.Structure):
@@ -78,7 +78,8 @@ class glp_kernel_stat(ctypes.Structure):
 
 EXPORTS = ["glp_nccl_unique_id", "glp_partition", "glp_graph_create", "glp_run", "glp_labels_get",
            "glp_iter_stats", "glp_kernel_stats", "glp_graph_info", "glp_graph_destroy",
-           "glp_local_group_create", "glp_local_group_destroy", "glp_last_error", "glp_version"]
+           "glp_local_group_create", "glp_local_group_destroy", "glp_struct_sizes", "glp_last_error",
+           "glp_version"]
 
 _lib = None
 
@@ -106,6 +107,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "glp_graph_destroy": [P],
         "glp_local_group_create": [I32, P],
         "glp_local_group_destroy": [P],
+        "glp_struct_sizes": [P, I32],
     }
     for name, args in sig.items():
         fn = getattr(lib, name)
@@ -164,9 +166,11 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
                      v_begin: int = 0, v_end: int | None = None, symmetric: bool = False,
                      rank: int = 0, nranks: int = 1, device: int | None = None,
                      nccl_unique_id: bytes | None = None, stream: torch.cuda.Stream | None = None,
-                     validate: bool = True, local_group=None, host_arcs: bool = False):
+                     validate: bool = True, local_group=None, host_arcs: bool = False, weights=None):
     """Create a device graph.  CUDA tensors are borrowed (keep them alive);
-    CPU tensors are copied.  Returns an opaque handle (ctypes.c_void_p)."""
+    CPU tensors are copied.  weights: optional per-arc integer weights in
+    [1, 2^31) on the same device as col_idx (weighted LP).  Returns an opaque
+    handle (ctypes.c_void_p)."""
     lib = load_library()
     if v_end is None:
         v_end = n_global
@@ -185,6 +189,12 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
     c.col_idx = col_idx.data_ptr() if col_idx.numel() else None
     c.on_device = int(on_device)
     c.symmetric = int(bool(symmetric))
+    if weights is not None:
+        if not torch.is_tensor(weights) or weights.dtype not in (torch.int32, torch.int64) \
+                or weights.numel() != col_idx.numel() or weights.is_cuda != on_device:
+            raise TypeError("weights: an int32/int64 tensor with one entry per arc, on col_idx's device")
+        weights = weights.to(torch.int32).contiguous()  # uint32 bit pattern (values < 2^31)
+        c.weights = weights.data_ptr() if weights.numel() else None
     d = None
     uid_buf = None
     if nranks > 1 or device is not None or stream is not None or local_group is not None:
@@ -290,6 +300,13 @@ def glp_graph_destroy(handle) -> None:
         _check(load_library().glp_graph_destroy(handle))
 
 
+def glp_struct_sizes() -> list:
+    import numpy as np
+    out = np.zeros(6, dtype=np.int64)
+    _check(load_library().glp_struct_sizes(out.ctypes.data, 6))
+    return out.tolist()
+
+
 def glp_version() -> str:
     return load_library().glp_version().decode()
 
@@ -318,7 +335,7 @@ class Graph:
     """
 
     def __init__(self, csr=None, *, n=None, row_offsets=None, col_idx=None, symmetric=None,
-                 validate=True, **dist):
+                 validate=True, weights=None, **dist):
         # symmetric: None = the CSR's own flag (glp_inputs.CSR.symmetric), else
         # False -- the frontier push is exact only on symmetric graphs, so it
         # is never assumed (the C ABI's zero default)
@@ -330,9 +347,12 @@ class Graph:
         self.n = int(n)
         self._off = row_offsets
         self._col = col_idx
+        if weights is not None and torch.is_tensor(weights) and weights.is_cuda:
+            weights = weights.to(torch.int32).contiguous()
+        self._w = weights
         self.device = row_offsets.device if row_offsets.is_cuda else torch.device("cuda", torch.cuda.current_device())
         self.handle = glp_graph_create(self.n, row_offsets, col_idx, symmetric=symmetric,
-                                       validate=validate, **dist)
+                                       validate=validate, weights=self._w, **dist)
 
     def run(self, variant="classic", max_iters: int = 20, seeds=None, **kw) -> RunInfo:
         v = VARIANTS[variant] if isinstance(variant, str) else int(variant)

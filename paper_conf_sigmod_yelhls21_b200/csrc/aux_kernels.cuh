@@ -141,6 +141,39 @@ __global__ void k_relayout(const int64_t* __restrict__ off, const int32_t* __res
   }
 }
 
+// Weighted LP: the arc weights beside the relayouted arcs (same positions).
+__global__ void k_relayout_w(const int64_t* __restrict__ off, const uint32_t* __restrict__ w,
+                             const int64_t* __restrict__ ioff, const int32_t* __restrict__ pos, int64_t nl, int64_t vb,
+                             uint32_t* __restrict__ w2) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t v = gw; v < nl; v += nw) {
+    const int64_t s = off[v], d = off[v + 1] - s, o = ioff[pos[vb + v] - vb];
+    for (int64_t j = lane; j < d; j += 32) w2[o + j] = w[s + j];
+  }
+}
+// weights in [1, 2^31) and every row's total < 2^31 (exact 32-bit sums)
+__global__ void k_validate_w(const int64_t* __restrict__ off, const uint32_t* __restrict__ w, int64_t nl,
+                             int* __restrict__ bad) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t v = gw; v < nl; v += nw) {
+    unsigned long long sum = 0;
+    bool zero = false;
+    for (int64_t e = off[v] + lane; e < off[v + 1]; e += 32) {
+      const uint32_t x = w[e];
+      sum += x;
+      zero |= x == 0u || x >= 0x80000000u;
+    }
+    for (int s = 16; s > 0; s >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, s);
+    if (__any_sync(0xffffffffu, zero) || sum >= 0x80000000ull) {
+      if (lane == 0) atomicOr(bad, 16);
+    }
+  }
+}
+
 // Predicted distinct labels of each row at t = 1 (performance hint only).
 __global__ void k_init_pred(const BinItem* __restrict__ rows, int32_t n_rows, unsigned* __restrict__ pred0,
                             unsigned* __restrict__ pred1, unsigned* __restrict__ pred2, unsigned seed_cap) {

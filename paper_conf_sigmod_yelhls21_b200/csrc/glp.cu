@@ -29,6 +29,7 @@
 #include "glp_internal.cuh"
 #include "layout.cuh"
 #include "mfl_kernels.cuh"
+#include "mfl_weighted.cuh"
 
 using namespace glp;
 
@@ -328,11 +329,12 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
   }
   g->nnz2 = rows_base + padded_total;
   if (g->nnz2 >= ((int64_t)1 << 48)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
-  g->n_gt256 = g->n_gt2048 = g->n_ge8k = 0;
+  g->n_gt256 = g->n_gt2048 = g->n_ge8k = g->n_gt512 = 0;
   for (const BinItem& it : row_i) {
     g->n_gt256 += it.d > 256;
     g->n_gt2048 += it.d > 2048;
     g->n_ge8k += it.d >= 8192;
+    g->n_gt512 += it.d > kWtWarpMax;
   }
   for (int k = 0; k < 3; ++k) g->pred[k] = dalloc<unsigned>(g, std::max<int64_t>(n_rows, 1));
   g->redo_m = dalloc<int32_t>(g, std::max<int64_t>(n_rows, 1));
@@ -577,6 +579,34 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     else if (nranks > 1 || (dist && dist->nccl_unique_id)) g->comm = new NcclComm(g, dist->nccl_unique_id);
     if (g->comm) g->comm->setup(g);
     build_layout(g, off_d, col_d);
+    if (csr->weights) {
+      // weighted LP: validate and place the weights beside the arcs
+      const uint32_t* w_d = csr->weights;
+      if (!csr->on_device) {
+        void* pw = nullptr;
+        if (g->nnz && pool_malloc(&pw, g->nnz * sizeof(uint32_t), g->stream) != cudaSuccess) {
+          cudaGetLastError();
+          fail(GLP_ERR_OUT_OF_MEMORY, "staging the weights on the device failed");
+        }
+        if (pw) {
+          temps.push_back(pw);
+          CK(cudaMemcpyAsync(pw, csr->weights, g->nnz * sizeof(uint32_t), cudaMemcpyHostToDevice, g->stream));
+        }
+        w_d = (const uint32_t*)pw;
+      }
+      g->w2 = dalloc<uint32_t>(g, std::max<int64_t>(g->nnz2, 1));
+      CK(cudaMemsetAsync(g->w2, 0, std::max<int64_t>(g->nnz2, 1) * sizeof(uint32_t), g->stream));
+      if (g->nl && g->nnz) {
+        k_validate_w<<<g->sms * 4, 256, 0, g->stream>>>(off_d, w_d, g->nl, dbad);
+        k_relayout_w<<<g->sms * 8, 256, 0, g->stream>>>(off_d, w_d, g->ioff, g->pos, g->nl, g->vb, g->w2);
+        CK(cudaGetLastError());
+      }
+      int bad = 0;
+      CK(cudaMemcpyAsync(&bad, dbad, sizeof(int), cudaMemcpyDeviceToHost, g->stream));
+      CK(cudaStreamSynchronize(g->stream));
+      if (bad & 16) fail(GLP_ERR_INVALID_GRAPH, "weights must be in [1, 2^31) with every row total < 2^31");
+      g->weighted = true;
+    }
     if (g->registered) {  // the caller's arcs are not read after the relayout
       CK(cudaStreamSynchronize(g->stream));
       cudaHostUnregister(g->registered);
@@ -622,6 +652,13 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     g->grid_w = grid_for(sms, (const void*)mfl_warp<V_LLP>, kWBlock, ws_);
     g->grid_m = grid_for(sms, (const void*)GLP_M_KERNEL(V_LLP), kMBlock, ms_);
     g->grid_mono = grid_for(sms, (const void*)mfl_mono<V_LLP>, kMonoBlock, 0);
+    const int wtw_ = (kWtBlock / 32) * kWtWarpSlots * 8, wtb_ = kWtSlots * 8;
+    CK(cudaFuncSetAttribute(mfl_wt_warp<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, wtw_));
+    CK(cudaFuncSetAttribute(mfl_wt_warp<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, wtw_));
+    CK(cudaFuncSetAttribute(mfl_wt_block<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, wtb_));
+    CK(cudaFuncSetAttribute(mfl_wt_block<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, wtb_));
+    g->grid_wtw = grid_for(sms, (const void*)mfl_wt_warp<V_CLASSIC>, kWtBlock, wtw_);
+    g->grid_wtb = grid_for(sms, (const void*)mfl_wt_block<V_CLASSIC>, kWtBlock, wtb_);
     g->grid_l = grid_for(sms, (const void*)GLP_L_KERNEL(V_LLP), kLBlock, ls_);
     const int gs_ = GLP_GIANT_SMEM ? kGSlots * 8 : 0;
     CK(cudaFuncSetAttribute(mfl_giant_count<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
@@ -668,8 +705,10 @@ cudaEvent_t pool_event(glp_graph* g, size_t& used) {
 }
 
 const char* kKernelNames[] = {"mfl_low", "mfl_warp", "mfl_block_m", "mfl_block_l", "push", "llp_hist", "exchange",
-                              "mfl_giant", "mfl_mono"};
-constexpr int kNumKernelNames = 9;
+                              "mfl_giant", "mfl_mono", "mfl_wt_warp", "mfl_wt_block"};
+constexpr int kNumKernelNames = 11;
+// counter slot of each MFL kernel id (glp_internal.cuh kNumCounters)
+inline int counter_of(int kid) { return kid == 7 ? 4 : kid == 8 ? 5 : kid == 9 ? 1 : kid == 10 ? 3 : kid; }
 
 template <class F>
 void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t& used, cudaStream_t st, F f) {
@@ -806,6 +845,34 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   return n;
 }
 
+// weighted LP (§8(f)3): long rows block-per-row, the rest warp-per-vertex
+template <int VAR>
+int launch_wt(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, size_t& used) {
+  Counters* c = g->d_cnt;
+  Sched* sc = g->d_sched;
+  cudaStream_t s0 = g->stream;
+  a.w2 = g->w2; a.ioff = g->ioff; a.ideg = g->ideg;
+  int n = 0;
+  if (g->n_gt512) {
+    MflArgs b = a;
+    b.items = g->rows; b.n_items = g->n_gt512; b.cnt = c + 3; b.work = &sc->work_l;
+    const int grid = std::min(g->grid_wtb, g->n_gt512);
+    timed(g, prof, 10, pend, used, s0,
+          [&] { mfl_wt_block<VAR><<<grid, kWtBlock, kWtSlots * 8, s0>>>(b); });
+    ++n;
+  }
+  const int64_t lo = g->n_gt512, hi = (int64_t)g->n_rows + g->n_low;
+  if (hi > lo) {
+    MflArgs b = a;
+    b.wt_lo = lo; b.wt_hi = hi; b.cnt = c + 1;
+    const int grid = (int)std::min<int64_t>(g->grid_wtw, (hi - lo + kWtBlock - 1) / kWtBlock);
+    timed(g, prof, 9, pend, used, s0,
+          [&] { mfl_wt_warp<VAR><<<grid, kWtBlock, (kWtBlock / 32) * kWtWarpSlots * 8, s0>>>(b); });
+    ++n;
+  }
+  return n;
+}
+
 void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_t* seeds, int64_t n_seeds,
               const glp_params* prm, glp_run_info* info) {
   if (!g) fail(GLP_ERR_INVALID_ARGUMENT, "graph is NULL");
@@ -815,6 +882,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   if (variant == GLP_VARIANT_LLP) {
     if (!std::isfinite(p.gamma) || p.gamma < 0) fail(GLP_ERR_INVALID_ARGUMENT, "gamma must be finite and >= 0");
     if (p.frontier == 1) fail(GLP_ERR_INVALID_ARGUMENT, "the frontier is not exact for LLP (frontier=1 rejected)");
+    if (g->weighted) fail(GLP_ERR_UNSUPPORTED, "weighted LP supports CLASSIC and SEEDED (not LLP)");
   }
   if (variant != GLP_VARIANT_SEEDED && (seeds != nullptr || n_seeds != 0))
     fail(GLP_ERR_INVALID_ARGUMENT, "seeds are only valid for GLP_VARIANT_SEEDED");
@@ -912,7 +980,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       ks.ms += kms;
       if (with_counters && (pe.kid < 4 || pe.kid >= 7) && pe.t == cur_t && !credited[pe.kid]) {
         credited[pe.kid] = true;
-        const Counters& c = g->h_cnt[pe.kid == 7 ? 4 : pe.kid == 8 ? 5 : pe.kid];
+        const Counters& c = g->h_cnt[counter_of(pe.kid)];
         ks.arcs += (double)c.arcs;
         // 4 B/arc (col_idx) + 8 B/active vertex (row offsets) + 4 B/changed label
         ks.bytes += 4.0 * (double)c.arcs + 8.0 * (double)c.verts + 4.0 * (double)c.changed;
@@ -952,7 +1020,10 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     // t = 1: every row is a sorted-row candidate (unique labels); they go to
     // the table-free mono kernel (SEEDED never takes the sorted path)
     a.mono_kernel = (t == 1 && variant != GLP_VARIANT_SEEDED && g->use_mono) ? 1 : 0;
-    switch (variant) {
+    if (g->weighted) {
+      launches += variant == GLP_VARIANT_SEEDED ? launch_wt<V_SEEDED>(g, a, prof, pend, used)
+                                                : launch_wt<V_CLASSIC>(g, a, prof, pend, used);
+    } else switch (variant) {
       case GLP_VARIANT_CLASSIC: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
       default: launches += launch_mfl<V_LLP>(g, a, prof, pend, used); break;
@@ -1185,6 +1256,16 @@ glp_status glp_nccl_unique_id(uint8_t out[128]) {
 
 glp_status glp_graph_destroy(glp_graph* g) {
   return guard([&] { free_graph(g); });
+}
+
+glp_status glp_struct_sizes(int64_t* out, int32_t max_entries) {
+  return guard([&] {
+    if (!out && max_entries > 0) fail(GLP_ERR_INVALID_ARGUMENT, "out is NULL");
+    const int64_t v[6] = {(int64_t)sizeof(glp_csr),      (int64_t)sizeof(glp_dist),
+                          (int64_t)sizeof(glp_params),   (int64_t)sizeof(glp_run_info),
+                          (int64_t)sizeof(glp_iter_stat), (int64_t)sizeof(glp_kernel_stat)};
+    for (int i = 0; i < max_entries && i < 6; ++i) out[i] = v[i];
+  });
 }
 
 const char* glp_last_error(void) { return g_last_error.c_str(); }

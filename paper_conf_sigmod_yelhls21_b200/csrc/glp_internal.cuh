@@ -201,6 +201,11 @@ struct MflArgs {
   int32_t v_ones;                       // LLP: V[l] == 1 for every l (L_{t-1} is PickLabel's permutation)
   int32_t lv_labels;                    // LLP sharded: neighbour labels are read from LV (R holds owned rows only)
   int32_t mono_kernel;                  // sorted-row candidates go to mfl_mono (launched this iteration)
+  // weighted LP (mfl_weighted.cuh)
+  const uint32_t* __restrict__ w2;      // arc weights beside col2
+  const int64_t* __restrict__ ioff;     // [nl] row start in col2
+  const int32_t* __restrict__ ideg;     // [nl] degree
+  int64_t wt_lo, wt_hi;                 // local vertices of the warp kernel
 };
 
 // Internal error: thrown inside the library, converted to glp_status at the ABI.
@@ -233,6 +238,9 @@ struct glp_graph {
   const int32_t* col = nullptr;
   bool own_csr = false;
   bool host_arcs = false;       // hybrid mode: col2 in pinned mapped host memory
+  bool weighted = false;        // weighted LP: w2 holds the arc weights
+  uint32_t* w2 = nullptr;       // [nnz2] weights beside col2 (padding 0)
+  int32_t n_gt512 = 0;          // prefix of rows with deg > kWtWarpMax
   void* col2_host = nullptr;    // its host allocation
   void* registered = nullptr;   // caller's host arcs registered during create
   int symmetric = 1;
@@ -290,6 +298,7 @@ struct glp_graph {
 
   // launch geometry
   int grid_low = 0, grid_w = 0, grid_m = 0, grid_l = 0, grid_g = 0, grid_aux = 0, grid_mono = 0;
+  int grid_wtw = 0, grid_wtb = 0;
 
   int cur = 0;  // index of L holding the result of the last run
   int cur_t = 0;  // iteration being launched (profiling)

@@ -62,7 +62,7 @@ class LocalGroup:
     exchange, counter reduction, frontier-mark merge, sharded LLP histogram)
     where only one GPU is available.  Argument marshalling only."""
 
-    def __init__(self, csr, nranks: int, edge_balanced: bool = False, bounds=None, device=None):
+    def __init__(self, csr, nranks: int, edge_balanced: bool = False, bounds=None, device=None, weights=None):
         self.nranks = int(nranks)
         self.n = csr.n
         self.bounds = list(bounds) if bounds is not None else \
@@ -72,13 +72,19 @@ class LocalGroup:
         off = csr.row_offsets.to(dev)
         col = csr.col_idx.to(dev)
         self._parts = [local_rows(off, col, self.bounds[r], self.bounds[r + 1]) for r in range(self.nranks)]
+        self._w = [None] * self.nranks
+        if weights is not None:
+            w = weights.to(dev).to(torch.int32)
+            offc = off.cpu()
+            self._w = [w[int(offc[self.bounds[r]]):int(offc[self.bounds[r + 1]])].contiguous()
+                       for r in range(self.nranks)]
         torch.cuda.synchronize(dev)
 
         def make(r):
             o, c = self._parts[r]
             return Graph(n=csr.n, row_offsets=o, col_idx=c, symmetric=csr.symmetric, rank=r, nranks=self.nranks,
                          v_begin=self.bounds[r], v_end=self.bounds[r + 1], device=dev.index,
-                         local_group=self.handle)
+                         local_group=self.handle, weights=self._w[r])
         self.graphs = self._all(make)
 
     def _all(self, fn):

@@ -33,11 +33,11 @@ def test_library_builds_and_exports_all_symbols():
 
 
 def test_struct_layout_matches_header():
-    # sizes the C side checks (glp_params.struct_size) and the ctypes mirror
-    assert ctypes.sizeof(glp.glp_params) == 64
-    assert ctypes.sizeof(glp.glp_csr) == 56
-    assert ctypes.sizeof(glp.glp_run_info) == 40
-    assert ctypes.sizeof(glp.glp_iter_stat) == 48
+    # the ctypes mirror against the compiled header's sizeof (glp_struct_sizes)
+    mine = [ctypes.sizeof(t) for t in (glp.glp_csr, glp.glp_dist, glp.glp_params, glp.glp_run_info,
+                                        glp.glp_iter_stat, glp.glp_kernel_stat)]
+    assert mine == glp.glp_struct_sizes()
+    assert ctypes.sizeof(glp.glp_params) == 64  # glp_params.struct_size is checked by glp_run
 
 
 def test_version_and_partition_host_only():
