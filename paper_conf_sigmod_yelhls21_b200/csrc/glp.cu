@@ -856,6 +856,7 @@ int launch_wt(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, si
   if (g->n_gt512) {
     MflArgs b = a;
     b.items = g->rows; b.n_items = g->n_gt512; b.cnt = c + 3; b.work = &sc->work_l;
+    b.pred = g->pred[g->pb]; b.pred_next = g->pred[(g->pb + 1) % 3];
     const int grid = std::min(g->grid_wtb, g->n_gt512);
     timed(g, prof, 10, pend, used, s0,
           [&] { mfl_wt_block<VAR><<<grid, kWtBlock, kWtSlots * 8, s0>>>(b); });

@@ -13,11 +13,13 @@
 // weights w2 sit beside the arcs of col2):
 //   mfl_wt_warp   vertices with 1 <= deg <= kWtWarpMax: one warp per vertex,
 //                 per-warp shared table of pow2 >= 2 deg slots (never full)
-//   mfl_wt_block  longer rows: one block per row, 8192-slot shared table; a
-//                 row with more labels than half the table is counted in
-//                 label-hash partitions (every pass re-reads the row and
-//                 counts only its part's labels), doubling the parts when a
-//                 part overflows -- exact by construction
+//   mfl_wt_block  longer rows: one block per row.  A row whose labels are
+//                 strictly increasing (t = 1) needs no table; otherwise an
+//                 8192-slot shared table, and a row with more labels than half
+//                 the table (predicted from its last distinct count) is
+//                 counted in label-hash partitions (every pass re-reads the
+//                 row and counts only its part's labels), doubling the parts
+//                 when a part overflows -- exact by construction
 #pragma once
 #include "mfl_kernels.cuh"
 
@@ -88,7 +90,7 @@ __global__ void __launch_bounds__(kWtBlock) mfl_wt_warp(MflArgs a) {
 template <int VAR>
 __global__ void __launch_bounds__(kWtBlock) mfl_wt_block(MflArgs a) {
   extern __shared__ __align__(16) unsigned long long wtb_tab[];  // kWtSlots
-  __shared__ int s_k, s_over;
+  __shared__ int s_k, s_over, s_distinct;
   Tally ty;
   for (;;) {
     if (threadIdx.x == 0) s_k = (int)atomicAdd(a.work, 1ull);
@@ -96,43 +98,77 @@ __global__ void __launch_bounds__(kWtBlock) mfl_wt_block(MflArgs a) {
     const int k = s_k;
     if (k >= a.n_items) break;
     const BinItem it = a.items[k];
+    const unsigned raw = a.pred[k];
     if (!a.dense && !a.flag[a.vb + it.v]) {
+      if (threadIdx.x == 0) a.pred_next[k] = raw;  // inactive: carry the count forward
       __syncthreads();  // s_k is rewritten by the next ticket
       continue;
     }
     const int d = it.d;
-    unsigned nparts = max(1u, (2u * (unsigned)d + kWtSlots - 1) / kWtSlots);
     Best<VAR> b;
-    for (;;) {
-      b = Best<VAR>();
-      bool over = false;
-      for (unsigned p = 0; p < nparts && !over; ++p) {
-        const Table tab{wtb_tab, (unsigned)kWtSlots};
-        tab.clear(threadIdx.x, kWtBlock);
-        if (threadIdx.x == 0) s_over = 0;
-        __syncthreads();
-        // one part: a full probe when the whole row fits at half load
-        const unsigned probe = nparts == 1u ? (unsigned)kWtSlots : (unsigned)kLProbe;
-        unsigned fresh = 0;
-        for (int e = threadIdx.x; e < d; e += kWtBlock) {
-          const int l = gather(a, a.col[it.start + e]);
-          if (l < 0 || (nparts > 1u && label_part((unsigned)l, nparts) != p)) continue;
-          const unsigned c = ht_add(tab, (unsigned)l, a.w2[it.start + e], probe, &fresh);
-          if (c == 0u) {
-            s_over = 1;
-            break;
-          }
-          b.observe(c, (unsigned)l, a);
-        }
-        __syncthreads();
-        over = s_over != 0;
-        __syncthreads();  // the next part clears the table
+    unsigned distinct = 0;
+    bool done = false;
+    // Sorted-row fast path (t = 1's unique labels on sorted rows, checked on
+    // the data): labels strictly increasing along the row occur once each, so
+    // a label's weight sum is its arc's weight -- no table, one pass.
+    if (mono_cand<VAR>(raw, a.pred_cap, d)) {
+      bool inc = true;
+      for (int e = threadIdx.x; e < d; e += kWtBlock) {
+        const int l = gather(a, a.col[it.start + e]);
+        const int lp = e > 0 ? gather(a, a.col[it.start + e - 1]) : -1;
+        inc = inc && l >= 0 && lp < l;
+        if (inc) b.observe(a.w2[it.start + e], (unsigned)l, a);
       }
-      if (!over) break;
-      nparts *= 2u;  // a part overflowed: finer partitions, recount (exact)
+      done = __syncthreads_and(inc ? 1 : 0) != 0;
+      if (done) distinct = (unsigned)d;
+      else b = Best<VAR>();
+    }
+    if (!done) {
+      // table passes: parts sized from the last distinct count (a row that
+      // took the sorted path last time: 40 % of it -- labels collapse
+      // [P:130]); an overflowing part doubles the parts (exact recount)
+      const unsigned pr = raw & kPredMask;
+      const unsigned est = (raw & kMonoTried) ? max(1u, (unsigned)(((unsigned long long)pr * 40ull) / 100ull)) : max(pr, 1u);
+      unsigned nparts = max(1u, (2u * min(est, (unsigned)d) + kWtSlots - 1) / kWtSlots);
+      if (2u * (unsigned)d <= (unsigned)kWtSlots) nparts = 1u;
+      for (;;) {
+        b = Best<VAR>();
+        if (threadIdx.x == 0) s_distinct = 0;
+        bool over = false;
+        for (unsigned p = 0; p < nparts && !over; ++p) {
+          const Table tab{wtb_tab, (unsigned)kWtSlots};
+          tab.clear(threadIdx.x, kWtBlock);
+          if (threadIdx.x == 0) s_over = 0;
+          __syncthreads();
+          // the whole row at half load: a full probe never fails
+          const unsigned probe = 2u * (unsigned)d <= (unsigned)kWtSlots ? (unsigned)kWtSlots : (unsigned)kLProbe;
+          unsigned fresh = 0;
+          for (int e = threadIdx.x; e < d; e += kWtBlock) {
+            const int l = gather(a, a.col[it.start + e]);
+            if (l < 0 || (nparts > 1u && label_part((unsigned)l, nparts) != p)) continue;
+            const unsigned c = ht_add(tab, (unsigned)l, a.w2[it.start + e], probe, &fresh);
+            if (c == 0u) {
+              s_over = 1;
+              break;
+            }
+            b.observe(c, (unsigned)l, a);
+          }
+          fresh = __reduce_add_sync(kFull, fresh);
+          if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(&s_distinct, (int)fresh);
+          __syncthreads();
+          over = s_over != 0;
+          __syncthreads();  // the next part clears the table
+        }
+        if (!over) break;
+        nparts *= 2u;
+      }
+      distinct = (unsigned)s_distinct;
     }
     b = block_best<VAR, kWtBlock>(b);
-    if (threadIdx.x == 0) update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty, d);
+    if (threadIdx.x == 0) {
+      a.pred_next[k] = max(distinct, 1u) | (done ? kMonoTried : 0u);
+      update_vertex<VAR>(a, it.v, d, b.have(), b.label(), ty, d);
+    }
     __syncthreads();
   }
   tally_flush(ty, a.cnt);
