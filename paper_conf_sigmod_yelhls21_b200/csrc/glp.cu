@@ -510,12 +510,13 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
         void* dp = nullptr;
         // already pinned (cudaHostAlloc / registered by the caller): mapped
         // under UVA as it is; otherwise register it for the create
-        if (cudaHostGetDevicePointer(&dp, hp, 0) != cudaSuccess) {
-          cudaGetLastError();
+        cudaPointerAttributes pa;
+        CK(cudaPointerGetAttributes(&pa, hp));
+        if (pa.type != cudaMemoryTypeHost) {
           CK(cudaHostRegister(hp, g->nnz * sizeof(int32_t), cudaHostRegisterMapped | cudaHostRegisterReadOnly));
           g->registered = hp;
-          CK(cudaHostGetDevicePointer(&dp, hp, 0));
         }
+        CK(cudaHostGetDevicePointer(&dp, hp, 0));
         col_d = (const int32_t*)dp;
       }
     } else {

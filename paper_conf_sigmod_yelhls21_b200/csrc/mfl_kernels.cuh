@@ -217,6 +217,17 @@ __device__ __forceinline__ bool strict_majority(const Best<VAR>& b, int d) {
   return __any_sync(kFull, 2ull * k > (unsigned long long)d);
 }
 
+// Monotone shared flags (overflow, strict majority) are polled by other warps
+// while they are being set; both sides use atomics, so the polling is a
+// synchronised read (compute-sanitizer racecheck clean) and a stale 0 only
+// delays an exit by one round.  One lane reads and broadcasts.
+__device__ __forceinline__ void flag_set(volatile int* f) { atomicExch((int*)f, 1); }
+__device__ __forceinline__ bool warp_flag(volatile int* f) {
+  int v = 0;
+  if ((threadIdx.x & 31) == 0) v = atomicOr((int*)f, 0);
+  return __shfl_sync(kFull, v, 0) != 0;
+}
+
 __device__ __forceinline__ unsigned slot_hash(unsigned lab, unsigned tsz) {
   return __umulhi(lab * 0x9E3779B1u, tsz);
 }
@@ -361,7 +372,7 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
     const unsigned tot = __reduce_add_sync(kFull, hc);
     if (lane == 0 && tot) {
       const unsigned cnt = ht_add(t, (unsigned)hot, tot, max_probe, &nfresh);
-      if (cnt == 0u) *overflow = 1;
+      if (cnt == 0u) flag_set(overflow);
       else if (obs) b.observe(cnt, (unsigned)hot, a, hotv);
     }
   }
@@ -389,7 +400,7 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
   for (int j = 0; j < N; ++j) {
     if (lab[j] >= 0 && cnt[j] == 0u) {
       cnt[j] = ht_probe_from(t, (unsigned)lab[j], mc[j], h[j], max_probe, &nfresh);
-      if (cnt[j] == 0u) *overflow = 1;
+      if (cnt[j] == 0u) flag_set(overflow);
     }
   }
   if (obs) {
@@ -834,7 +845,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v, hot);
         }
         __syncwarp();
-        over = s_over[wid] != 0;
+        over = warp_flag(&s_over[wid]);
         if (GLP_MAJORITY && VAR != V_LLP && !over && off + kWRound < d) major = strict_majority(b, d);
       }
       if ((over || major) && !next_loaded) load_round(a.col, nstart, 0, nd, x0, x1);
@@ -1026,10 +1037,10 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
     if (GLP_MAJORITY && VAR != V_LLP && major != nullptr && base + STEP < d) {
       // a strict-majority observation ends the row for every warp (they poll the flag)
       const bool m = strict_majority(b, d);
-      if (m && (threadIdx.x & 31) == 0) *major = 1;
-      if (m || __any_sync(kFull, *major != 0)) break;
+      if (m && (threadIdx.x & 31) == 0) flag_set(major);
+      if (m || warp_flag(major)) break;
     }
-    if (__any_sync(kFull, *overflow != 0)) break;  // warp-uniform exit
+    if (warp_flag(overflow)) break;  // warp-uniform exit
   }
   fresh = __reduce_add_sync(kFull, fresh);
   if ((threadIdx.x & 31) == 0) {
@@ -1134,7 +1145,7 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
     }
     const int nov[4] = {-1, -1, -1, -1};
     fresh += warp_insert_n<VAR, 4>(a, tab, max_probe, lab, b, overflow, nov, false, GLP_HOT_DIV == 0);
-    if (__any_sync(kFull, *overflow != 0)) break;
+    if (warp_flag(overflow)) break;
   }
   fresh = __reduce_add_sync(kFull, fresh);
   if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
