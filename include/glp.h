@@ -155,7 +155,17 @@ typedef struct {
                                   device.  Needs a host CSR (on_device = 0),
                                   whose col_idx is registered (pinned) during
                                   create.  Results are identical.  Default 0 */
-  int32_t reserved[4];
+  int32_t tail_cms;            /* 1: L rows (long, many labels) count with the
+                                  paper's HT + Count-Min Sketch single scan
+                                  [P:132-182 §4.1]; the HT's best is taken
+                                  only when it beats every sketch estimate
+                                  strictly, else the row is recounted exactly
+                                  (results never change).  Default 0 */
+  int32_t cms_ht_slots;        /* tail_cms: HT capacity h (power of two <=
+                                  8192; 0 = 8192).  Testing / analysis        */
+  int32_t cms_depth;           /* tail_cms: sketch rows d (1..8, width =
+                                  8192 / d; 0 = 4)                             */
+  int32_t reserved[1];
 } glp_params;
 
 typedef struct {
@@ -176,6 +186,9 @@ typedef struct {
   int32_t dense;               /* 1 if the iteration was a full sweep           */
   int32_t pad;
   double ms;                   /* device time of the iteration                  */
+  int64_t cms_rows;            /* tail_cms: L rows whose scan used the sketch   */
+  int64_t cms_rescans;         /* ... of those, rows rescanned for estimates    */
+  int64_t cms_fallbacks;       /* ... of those, rows recounted exactly          */
 } glp_iter_stat;
 
 /* Per-kernel totals of the last run with params.profile = 1. */

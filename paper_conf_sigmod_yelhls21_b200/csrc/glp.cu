@@ -642,9 +642,11 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaFuncSetAttribute(GLP_M_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, ms_));
     CK(cudaFuncSetAttribute(GLP_M_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, ms_));
     CK(cudaFuncSetAttribute(GLP_M_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, ms_));
-    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, ls_));
-    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, ls_));
-    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, ls_));
+    // (+ the CMS counters of the §8(f)2 HT + CMS mode)
+    const int lsc_ = ls_ + (int)kCmsCounters * 4;
+    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_CLASSIC), cudaFuncAttributeMaxDynamicSharedMemorySize, lsc_));
+    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_SEEDED), cudaFuncAttributeMaxDynamicSharedMemorySize, lsc_));
+    CK(cudaFuncSetAttribute(GLP_L_KERNEL(V_LLP), cudaFuncAttributeMaxDynamicSharedMemorySize, lsc_));
     g->grid_low = grid_for(sms, (const void*)mfl_low<V_LLP>, kLowBlock, 0);
     const int ws_ = (kWBlock / 32) * kWSlots * 8;
     CK(cudaFuncSetAttribute(mfl_warp<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
@@ -748,7 +750,7 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   Counters* c = g->d_cnt;
   Sched* sc = g->d_sched;
   int n = 0;
-  const size_t ms_ = kMSlots * 8, ls_ = kLSlots * 8;
+  const size_t ms_ = kMSlots * 8, ls_ = kLSlots * 8 + (a.cms ? kCmsCounters * 4 : 0);
   MflArgs r = a;
   r.items = g->rows; r.big_prefix = g->n_ge8k; r.pred = g->pred[g->pb]; r.pred_prev = g->pred[(g->pb + 2) % 3];
   r.pred_next = g->pred[(g->pb + 1) % 3];
@@ -1022,6 +1024,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     // t = 1: every row is a sorted-row candidate (unique labels); they go to
     // the table-free mono kernel (SEEDED never takes the sorted path)
     a.mono_kernel = (t == 1 && variant != GLP_VARIANT_SEEDED && g->use_mono) ? 1 : 0;
+    a.cms = p.tail_cms ? 1 : 0;
+    a.cms_ht = p.cms_ht_slots > 0 ? (unsigned)p.cms_ht_slots : 0u;
+    a.cms_depth = p.cms_depth > 0 ? (unsigned)p.cms_depth : 4u;
     if (g->weighted) {
       launches += variant == GLP_VARIANT_SEEDED ? launch_wt<V_SEEDED>(g, a, prof, pend, used)
                                                 : launch_wt<V_CLASSIC>(g, a, prof, pend, used);
@@ -1043,6 +1048,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     for (int b = 0; b < kNumCounters; ++b) {
       tot.changed += g->h_cnt[b].changed; tot.d2 += g->h_cnt[b].d2; tot.chdeg += g->h_cnt[b].chdeg;
       tot.arcs += g->h_cnt[b].arcs; tot.verts += g->h_cnt[b].verts;
+      tot.pad0 += g->h_cnt[b].pad0; tot.pad[0] += g->h_cnt[b].pad[0]; tot.pad[1] += g->h_cnt[b].pad[1];
     }
     glp_iter_stat st;
     memset(&st, 0, sizeof(st));
@@ -1051,6 +1057,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     st.active_vertices = (int64_t)tot.verts;
     st.active_arcs = (int64_t)tot.arcs;
     st.dense = dense ? 1 : 0;
+    st.cms_rows = (int64_t)tot.pad0;
+    st.cms_rescans = (int64_t)tot.pad[0];
+    st.cms_fallbacks = (int64_t)tot.pad[1];
     float ms = 0;
     CK(cudaEventElapsedTime(&ms, e0, e1));
     st.ms = ms;

@@ -149,8 +149,8 @@ struct Counters {
   unsigned long long chdeg;     // sum of deg over changed vertices
   unsigned long long arcs;      // arcs scanned
   unsigned long long verts;     // vertices scanned
-  unsigned long long pad0;
-  unsigned long long pad[2];
+  unsigned long long pad0;    // L rows that used the CMS (§8(f)2)
+  unsigned long long pad[2];  // [0] of those, rows rescanned for estimates; [1] rows recounted (fallback)
 };
 
 // per-kernel iteration counters: low, W, M, L, giant, mono
@@ -206,6 +206,10 @@ struct MflArgs {
   const int64_t* __restrict__ ioff;     // [nl] row start in col2
   const int32_t* __restrict__ ideg;     // [nl] degree
   int64_t wt_lo, wt_hi;                 // local vertices of the warp kernel
+  // §8(f)2 HT + CMS for L rows (mfl_kernels.cuh cms_count)
+  int32_t cms;                          // 1: L rows count with HT + CMS
+  unsigned cms_ht;                      // HT slots (0 = the whole L table)
+  unsigned cms_depth;                   // sketch rows d (width = 8192 / d)
 };
 
 // Internal error: thrown inside the library, converted to glp_status at the ABI.

@@ -326,6 +326,35 @@ __device__ __forceinline__ unsigned ht_add(const Table& t, unsigned lab, unsigne
 // match) with predicated atomics; only labels whose home slot holds another
 // label fall back to the probing loop.  Returns this lane's count of newly
 // claimed slots.
+// ---------------------------------------------------------------------------
+// Count-Min Sketch beside the hash table (§8(f)2, PAPER §4.1 Procedure
+// SharedMemBigNodes [P:132-182]): a label whose insertion into the shared HT
+// fails (its probe chain is full) is counted in a CMS of `depth` rows x
+// `width` u32 counters in shared memory instead, and flags `used`.  A label is
+// wholly in HT or wholly in the CMS (HT slots are never freed, so once a
+// label's chain is full it stays full), so HT counts are exact.
+constexpr unsigned kCmsCounters = 8192;  // u32 sketch counters per block (32 KB)
+struct Cms {
+  unsigned* c;      // depth * width counters (shared memory)
+  unsigned depth, width;
+  volatile int* used;
+  __device__ __forceinline__ unsigned slot(unsigned l, unsigned i) const {
+    // row i: an independent multiplicative hash (odd multipliers)
+    return __umulhi((l ^ (0x9E3779B9u * (i + 1u))) * (0x85EBCA6Bu + 2u * i * 0x27D4EB2Du), width);
+  }
+  __device__ __forceinline__ void add(unsigned l, unsigned k) const {
+    for (unsigned i = 0; i < depth; ++i) atomicAdd(c + i * width + slot(l, i), k);
+    flag_set(used);
+  }
+  // estimate g(l) = min over rows (read after a barrier: an upper bound of
+  // l's count, exact for every label that went to the sketch [P:134, Lemma 2])
+  __device__ __forceinline__ unsigned estimate(unsigned l) const {
+    unsigned g = 0xffffffffu;
+    for (unsigned i = 0; i < depth; ++i) g = min(g, c[i * width + slot(l, i)]);
+    return g;
+  }
+};
+
 // Rows predicted to hold more than d / GLP_HOT_DIV distinct labels (few
 // repeats per label: t = 2..3) skip the hot-label pass, whose single-lane
 // insert costs more than it saves there (0 = always take it).
@@ -344,7 +373,8 @@ __device__ __forceinline__ bool hot_pass(unsigned pred, int d) {
 template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
                                                   const int (&labin)[N], Best<VAR>& b, volatile int* overflow,
-                                                  const int (&vin)[N], bool use_v, bool hot_ok = true) {
+                                                  const int (&vin)[N], bool use_v, bool hot_ok = true,
+                                                  const Cms* cms = nullptr) {
   // use_v (LLP with a.LV): labels carry their V, so LLP observes at insert
   // like CLASSIC; otherwise LLP scores from the final table (table_scan)
   const bool obs = VAR != V_LLP || use_v;
@@ -372,8 +402,12 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
     const unsigned tot = __reduce_add_sync(kFull, hc);
     if (lane == 0 && tot) {
       const unsigned cnt = ht_add(t, (unsigned)hot, tot, max_probe, &nfresh);
-      if (cnt == 0u) flag_set(overflow);
-      else if (obs) b.observe(cnt, (unsigned)hot, a, hotv);
+      if (cnt == 0u) {
+        if (cms) cms->add((unsigned)hot, tot);  // HT full: the sketch counts it
+        else flag_set(overflow);
+      } else if (obs) {
+        b.observe(cnt, (unsigned)hot, a, hotv);
+      }
     }
   }
   unsigned mc[N];  // occurrences this lane inserts for slot j
@@ -400,7 +434,10 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
   for (int j = 0; j < N; ++j) {
     if (lab[j] >= 0 && cnt[j] == 0u) {
       cnt[j] = ht_probe_from(t, (unsigned)lab[j], mc[j], h[j], max_probe, &nfresh);
-      if (cnt[j] == 0u) flag_set(overflow);
+      if (cnt[j] == 0u) {
+        if (cms) cms->add((unsigned)lab[j], mc[j]);
+        else flag_set(overflow);
+      }
     }
   }
   if (obs) {
@@ -1004,7 +1041,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
                                             volatile int* overflow, int* distinct, Best<VAR>& b,
                                             volatile int* major, unsigned fparts = 1u, int* scanned = nullptr,
-                                            bool hot = true) {
+                                            bool hot = true, const Cms* cms = nullptr) {
   constexpr int STEP = BLOCK * 4 * UNROLL;
   unsigned fresh = 0;
   int base = 0;
@@ -1033,7 +1070,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
     }
-    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot);
+    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot, cms);
     if (GLP_MAJORITY && VAR != V_LLP && major != nullptr && base + STEP < d) {
       // a strict-majority observation ends the row for every warp (they poll the flag)
       const bool m = strict_majority(b, d);
@@ -1149,6 +1186,110 @@ __device__ __forceinline__ void count_staged(const MflArgs& a, const int32_t* st
   }
   fresh = __reduce_add_sync(kFull, fresh);
   if ((threadIdx.x & 31) == 0 && fresh) atomicAdd(distinct, (int)fresh);
+}
+
+// Linear-probe lookup (post-count, read only): is l in the HT?
+__device__ __forceinline__ bool ht_has(const Table& t, unsigned l, unsigned max_probe) {
+  unsigned h = slot_hash(l, t.tsz);
+  for (unsigned p = 0; p < max_probe; ++p) {
+    const unsigned k = t.key[h];
+    if (k == l) return true;
+    if (k == kFree) return false;
+    h = (h + 1) & (t.tsz - 1);
+  }
+  return false;
+}
+
+// Block-wide max of a u64 key (every thread gets it).
+template <int BLOCK>
+__device__ __forceinline__ unsigned long long block_max_u64(unsigned long long x) {
+  __shared__ unsigned long long red[BLOCK / 32];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+  for (int s = 16; s > 0; s >>= 1) x = max(x, __shfl_xor_sync(kFull, x, s));
+  __syncthreads();
+  if (lane == 0) red[wid] = x;
+  __syncthreads();
+  unsigned long long y = 0;
+  for (int w = 0; w < BLOCK / 32; ++w) y = max(y, red[w]);
+  return y;
+}
+
+// HT + CMS count of one L row (§8(f)2).  The shared table region holds the HT
+// (a.cms_ht slots, default all SLOTS) and, after it, the sketch counters.
+// Returns true when the HT's best is the row's MFL (b then holds it in the
+// usual running-max form); false when the row must be recounted exactly.
+// Decision, all post-barrier (R15):
+//   1. no label reached the sketch: the HT holds every label (exact);
+//   2. a strict majority was observed in the HT: it is the MFL;
+//   3. s(HT) > bound, bound = min over rows of the row's largest counter (an
+//      upper bound of every sketch label's count) -- no rescan;
+//   4. s(HT) > s(CMS) = max over sketch labels of their estimate g(l) =
+//      min_i C[i][h_i(l)] (Lemma 2's quantity), found by rescanning the row
+//      for labels not in the HT;
+//   else fallback.  Scores compare strictly: a sketch label tying the HT's
+//   best could be smaller (min-label ties, R4).  Stats go to cnt->pad0
+//   (rows that used the sketch), pad[0] (rescans), pad[1] (fallbacks).
+template <int VAR, int BLOCK, int SLOTS, int UNROLL>
+__device__ __forceinline__ bool cms_count(const MflArgs& a, int64_t start, int d, int4 (&cur)[UNROLL], Best<VAR>& b,
+                                          volatile int* s_over, int* s_distinct, volatile int* s_major, int* s_scan,
+                                          bool hot) {
+  extern __shared__ __align__(16) unsigned long long smem_tab[];
+  __shared__ int s_used;
+  const unsigned hs = a.cms_ht ? min((unsigned)SLOTS, 1u << (31 - __clz(max(a.cms_ht, 2u)))) : (unsigned)SLOTS;
+  const Table tab{smem_tab, hs};
+  const unsigned depth = min(max(a.cms_depth, 1u), 8u);
+  const unsigned width = kCmsCounters / depth;
+  unsigned* ctr = (unsigned*)(smem_tab + SLOTS);
+  const Cms cm{ctr, depth, width, &s_used};
+  tab.clear(threadIdx.x, BLOCK);
+  for (unsigned j = threadIdx.x; j < kCmsCounters / 4; j += BLOCK) ((uint4*)ctr)[j] = make_uint4(0u, 0u, 0u, 0u);
+  if (threadIdx.x == 0) s_used = 0;
+  __syncthreads();
+  // the probe limit marks an HT insertion as failed (chain full); with a tiny
+  // HT (a.cms_ht) it is "the HT is full" of the paper
+  block_count<VAR, BLOCK, UNROLL, GLP_L_IPF>(a, start, d, tab, kLProbe, cur, nullptr, s_over, s_distinct, b, s_major,
+                                             1u, s_scan, hot, &cm);
+  __syncthreads();
+  if (a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);  // LLP without carried V
+  if (s_used == 0) return true;
+  Counters* st = a.cnt;
+  if (threadIdx.x == 0) atomicAdd(&st->pad0, 1ull);
+  if (*s_major) return true;  // (never set for LLP)
+  // s(HT) as an order-preserving key: CLASSIC/SEEDED count<<32 | ~label,
+  // LLP dkey(score)
+  Best<VAR> hb = b;
+  hb.warp_reduce();
+  const unsigned long long hkey = block_max_u64<BLOCK>(hb.key);
+  // 3. cheap bound
+  unsigned long long rowmin = ~0ull;
+  for (unsigned i = 0; i < depth; ++i) {
+    unsigned m = 0;
+    for (unsigned j = threadIdx.x; j < width; j += BLOCK) m = max(m, ctr[i * width + j]);
+    rowmin = min(rowmin, block_max_u64<BLOCK>(m));
+  }
+  auto score_key = [&](unsigned g, int v) -> unsigned long long {
+    // the best key a sketch label with count <= g and histogram v could reach
+    if (VAR == V_LLP) return dkey(llp_score(g, v, a.gamma));
+    return ((unsigned long long)g << 32) | 0xffffffffull;  // (label 0: the strongest tie-break)
+  };
+  const unsigned long long hcmp = VAR == V_LLP ? hkey : (hkey | 0xffffffffull);  // compare counts only
+  // LLP: V[l] >= 1 for a present label, and the score falls with V
+  if (hcmp > score_key((unsigned)rowmin, 1)) return true;
+  // 4. per-label estimates of the sketch labels (rescan of the row)
+  if (threadIdx.x == 0) atomicAdd(&st->pad[0], 1ull);
+  unsigned long long ckey = 0ull;
+  for (int e = threadIdx.x; e < d; e += BLOCK) {
+    const int l = gather(a, a.col[start + e]);
+    if (l < 0 || ht_has(tab, (unsigned)l, kLProbe)) continue;
+    const unsigned g = cm.estimate((unsigned)l);
+    const int v = VAR == V_LLP ? (a.v_ones ? 1 : (a.LV ? __ldg(&a.LV[a.col[start + e]].y) : ld_label(a.V + l))) : 0;
+    ckey = max(ckey, score_key(g, v));
+  }
+  ckey = block_max_u64<BLOCK>(ckey);
+  if (hcmp > ckey) return true;
+  if (threadIdx.x == 0) atomicAdd(&st->pad[1], 1ull);
+  return false;
 }
 
 // mfl_block: one block per row of class CLS (M or L).  mode 0 scans the
@@ -1273,7 +1414,17 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
     unsigned nparts = PART ? max(1u, (min(est, (unsigned)d) + SLOTS / 2 - 1) / (SLOTS / 2)) : 1u;
     bool staged = false;  // stageA holds the row's gathered labels
     bool over = false;
-    if (nparts == 1u) {
+    if (PART && a.cms) {
+      // §8(f)2 SharedMemBigNodes [P:132-182]: one scan, HT + CMS; the HT's
+      // best is the MFL when it beats every sketch estimate strictly (R15),
+      // else the row is recounted exactly in partitions (the paper's global
+      // table fallback [P:166])
+      over = !cms_count<VAR, BLOCK, SLOTS, UNROLL>(a, it.start, d, cur, b, &s_over, &s_distinct, &s_major, &s_scan,
+                                                  hot_pass(est, d));
+      if (over) nparts = min(max(2u, ((unsigned)d + SLOTS / 2 - 1) / (SLOTS / 2)), 255u);
+      if (over) b = Best<VAR>();
+      __syncthreads();
+    } else if (nparts == 1u) {
       // single pass: gather + count.  Nothing is staged: an overflow stops the
       // count early, so the partition passes below gather the row again
       // (GLP_L_STAGE1 = 1 restores the old, never-read staging writes), and a

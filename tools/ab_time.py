@@ -21,6 +21,7 @@ import paper_conf_sigmod_yelhls21_b200 as glp  # noqa: E402
 wl = sys.argv[1] if len(sys.argv) > 1 else "rmat24"
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 10
 spec, variant, max_iters, gamma = bench.WORKLOADS[wl]
+kw = json.loads(os.environ.get("GLP_AB_KW", "{}"))  # extra glp_run params (A/B of run modes)
 csr, seeds = bench.make_graph(spec, "cuda")
 torch.cuda.synchronize()
 torch.cuda.empty_cache()
@@ -28,11 +29,11 @@ g = glp.Graph(csr)
 flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device="cuda")
 stream = torch.cuda.current_stream()
 for _ in range(3):
-    g.run(variant, max_iters, seeds, gamma=gamma)
+    g.run(variant, max_iters, seeds, gamma=gamma, **kw)
 ms, its, shas = [], [], set()
 for _ in range(reps):
     flush.fill_(1)
-    info = g.run(variant, max_iters, seeds, gamma=gamma)
+    info = g.run(variant, max_iters, seeds, gamma=gamma, **kw)
     ms.append(info.elapsed_ms)
     its.append([round(s["ms"], 3) for s in g.iter_stats()])
     shas.add(hashlib.sha1(g.labels("cpu").numpy().tobytes()).hexdigest()[:12])
@@ -41,7 +42,7 @@ w = (torch.arange(csr.col_idx.numel(), device="cuda", dtype=torch.int64) % 10000
 graph_sum = int((csr.col_idx.to(torch.int64) * w).sum()) ^ int(csr.row_offsets.sum())
 med = statistics.median(ms)
 i = ms.index(sorted(ms)[len(ms) // 2])
-print(json.dumps({"lib": os.environ.get("GLP_LIB", "in-tree"), "workload": wl, "median_ms": round(med, 3),
+print(json.dumps({"lib": os.environ.get("GLP_LIB", "in-tree"), "kw": kw, "workload": wl, "median_ms": round(med, 3),
                   "min_ms": round(min(ms), 3), "iterations": info.iterations, "iter_ms": its[i],
                   "labels_sha": hashlib.sha1(lab.tobytes()).hexdigest()[:12], "distinct_runs": len(shas),
                   "graph_sum": graph_sum}), flush=True)
