@@ -165,7 +165,11 @@ typedef struct {
                                   8192; 0 = 8192).  Testing / analysis        */
   int32_t cms_depth;           /* tail_cms: sketch rows d (1..8, width =
                                   8192 / d; 0 = 4)                             */
-  int32_t reserved[1];
+  int32_t sparse_exchange;     /* nranks > 1, CLASSIC / SEEDED (§8(f)1): replace
+                                  the label all-gather by an exchange of the
+                                  changed vertices' (id, label) pairs of t-1
+                                  and t.  -1 auto (default: when changed at
+                                  t-1 < n / (4 nranks)), 0 never, 1 always     */
 } glp_params;
 
 typedef struct {
@@ -184,7 +188,8 @@ typedef struct {
   int64_t active_vertices;     /* vertices scanned (superset of the frontier)   */
   int64_t active_arcs;         /* arcs scanned                                  */
   int32_t dense;               /* 1 if the iteration was a full sweep           */
-  int32_t pad;
+  int32_t exchange;            /* nranks > 1: 1 label all-gather, 2 sparse
+                                  (changed pairs), 3 (label, V) all-gather     */
   double ms;                   /* device time of the iteration                  */
   int64_t cms_rows;            /* tail_cms: L rows whose scan used the sketch   */
   int64_t cms_rescans;         /* ... of those, rows rescanned for estimates    */

@@ -57,7 +57,7 @@ class glp_params(ctypes.Structure):
                 ("validate", ctypes.c_int32), ("profile", ctypes.c_int32),
                 ("dense_divisor", ctypes.c_int32), ("debug_pred_cap", ctypes.c_int32),
                 ("llp_hist", ctypes.c_int32), ("host_arcs", ctypes.c_int32), ("tail_cms", ctypes.c_int32),
-                ("cms_ht_slots", ctypes.c_int32), ("cms_depth", ctypes.c_int32), ("reserved", ctypes.c_int32 * 1)]
+                ("cms_ht_slots", ctypes.c_int32), ("cms_depth", ctypes.c_int32), ("sparse_exchange", ctypes.c_int32)]
 
 
 class glp_run_info(ctypes.Structure):
@@ -69,7 +69,7 @@ class glp_run_info(ctypes.Structure):
 class glp_iter_stat(ctypes.Structure):
     _fields_ = [("changed", ctypes.c_int64), ("d2", ctypes.c_int64),
                 ("active_vertices", ctypes.c_int64), ("active_arcs", ctypes.c_int64),
-                ("dense", ctypes.c_int32), ("pad", ctypes.c_int32), ("ms", ctypes.c_double),
+                ("dense", ctypes.c_int32), ("exchange", ctypes.c_int32), ("ms", ctypes.c_double),
                 ("cms_rows", ctypes.c_int64), ("cms_rescans", ctypes.c_int64), ("cms_fallbacks", ctypes.c_int64)]
 
 
@@ -131,7 +131,7 @@ def _check(st: int):
 def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = True,
                 validate: bool = True, profile: bool = False, dense_divisor: int = 0,
                 debug_pred_cap: int = 0, llp_hist: int = 0, host_arcs: bool = False, tail_cms: bool = False,
-                cms_ht_slots: int = 0, cms_depth: int = 0) -> glp_params:
+                cms_ht_slots: int = 0, cms_depth: int = 0, sparse_exchange: int = -1) -> glp_params:
     p = glp_params()
     p.struct_size = ctypes.sizeof(glp_params)
     p.gamma = float(gamma)
@@ -146,6 +146,7 @@ def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = T
     p.tail_cms = int(bool(tail_cms))
     p.cms_ht_slots = int(cms_ht_slots)
     p.cms_depth = int(cms_depth)
+    p.sparse_exchange = int(sparse_exchange)
     return p
 
 
@@ -235,7 +236,7 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
 def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, gamma: float = 0.0,
             frontier: int = -1, stop_on_2cycle: bool = True, profile: bool = False,
             dense_divisor: int = 0, debug_pred_cap: int = 0, llp_hist: int = 0, tail_cms: bool = False,
-            cms_ht_slots: int = 0, cms_depth: int = 0) -> dict:
+            cms_ht_slots: int = 0, cms_depth: int = 0, sparse_exchange: int = -1) -> dict:
     import numpy as np
     lib = load_library()
     sd = None
@@ -246,7 +247,8 @@ def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, 
     info = glp_run_info()
     prm = make_params(gamma=gamma, frontier=frontier, stop_on_2cycle=stop_on_2cycle, profile=profile,
                       dense_divisor=dense_divisor, debug_pred_cap=debug_pred_cap, llp_hist=llp_hist,
-                      tail_cms=tail_cms, cms_ht_slots=cms_ht_slots, cms_depth=cms_depth)
+                      tail_cms=tail_cms, cms_ht_slots=cms_ht_slots, cms_depth=cms_depth,
+                      sparse_exchange=sparse_exchange)
     _check(lib.glp_run(handle, int(variant), int(max_iters), None if sd is None else sd.ctypes.data, ns,
                        ctypes.byref(prm), ctypes.byref(info)))
     return dict(iterations=info.iterations, stop_reason=info.stop_reason,
@@ -269,7 +271,7 @@ def glp_iter_stats(handle) -> list:
     arr = (glp_iter_stat * max(n.value, 1))()
     _check(lib.glp_iter_stats(handle, ctypes.cast(arr, ctypes.c_void_p), n.value, ctypes.byref(n)))
     return [dict(changed=s.changed, d2=s.d2, active_vertices=s.active_vertices, active_arcs=s.active_arcs,
-                 dense=bool(s.dense), ms=s.ms, cms_rows=s.cms_rows, cms_rescans=s.cms_rescans,
+                 dense=bool(s.dense), exchange=s.exchange, ms=s.ms, cms_rows=s.cms_rows, cms_rescans=s.cms_rescans,
                  cms_fallbacks=s.cms_fallbacks) for s in arr[:n.value]]
 
 

@@ -13,6 +13,12 @@
 //   allreduce_i32(s, r, k)    r = sum over ranks of s (LLP sharded histogram)
 //   merge_flags(flag)         owned slice of the frontier marks = max over the
 //                             ranks' marks (each rank's push marks global ids)
+//   exchange_changes(W, ...)  §8(f)1 sparse exchange: instead of the label
+//                             slices, every rank's (id, label) pairs of the
+//                             vertices it changed at t-1 and at t (W holds
+//                             L_{t-2} outside the owned rows; applying both
+//                             lists in order yields L_t) -- volume 8 B per
+//                             change instead of 4 B per vertex
 //
 // Two implementations:
 //   NcclComm   one process per GPU: ncclAllGather (grouped ncclBroadcast when
@@ -55,6 +61,12 @@ struct Comm {
   virtual void allreduce_u64(glp_graph* g, unsigned long long* p, size_t k) = 0;
   virtual void allreduce_i32(glp_graph* g, const int32_t* send, int32_t* recv, size_t k) = 0;
   virtual void merge_flags(glp_graph* g, uint8_t* flag) = 0;
+  // sparse replacement of allgather(L_t) (§8(f)1): W holds L_{t-2} outside
+  // this rank's rows; applying every other rank's changes of t-1 (lists[0],
+  // counts[0]) and then of t (lists[1], counts[1]) turns it into L_t.
+  // Lists and counts are device memory.
+  virtual void exchange_changes(glp_graph* g, int32_t* W, const int2* const lists[2],
+                                const unsigned* const counts[2]) = 0;
   // a rank failed: release the others (local group) instead of letting them wait
   virtual void abort(const std::string&) {}
 };
@@ -76,6 +88,47 @@ inline void set_bounds(glp_graph* g, const std::vector<int64_t>& all) {
   if (g->bounds[0] != 0 || g->bounds[g->nranks] != g->n)
     throw Err{GLP_ERR_INVALID_ARGUMENT, "rank row ranges do not cover [0, n_global)"};
 }
+
+constexpr int kMaxLocalRanks = 16;
+
+// ---- sparse exchange (§8(f)1): only (vertex, label) pairs of changed vertices
+// This rank's owned vertices changed at t (so.x == t): (global internal id,
+// new label), compacted with one atomic per warp.
+__global__ void k_collect_changes(const int2* __restrict__ so, const int32_t* __restrict__ W, int64_t nl, int64_t vb,
+                                  int32_t t, int2* __restrict__ out, unsigned* __restrict__ n_out) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < nl;
+       base += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t v = base + lane;
+    const bool ch = v < nl && so[v].x == t;
+    const unsigned m = __ballot_sync(0xffffffffu, ch);
+    unsigned at = 0;
+    if (lane == 0 && m) at = atomicAdd(n_out, (unsigned)__popc(m));
+    at = __shfl_sync(0xffffffffu, at, 0);
+    if (ch) out[at + __popc(m & ((1u << lane) - 1u))] = make_int2((int)(vb + v), W[vb + v]);
+  }
+}
+// W[q] = label for every pair of the given lists (other ranks' changes)
+struct ChgLists {
+  const int2* p[kMaxLocalRanks];
+  const unsigned* n[kMaxLocalRanks];
+  int nranks, skip;  // skip = this rank (its own changes are already in W)
+};
+__global__ void k_apply_changes(ChgLists L, int32_t* __restrict__ W) {
+  for (int r = 0; r < L.nranks; ++r) {
+    if (r == L.skip) continue;
+    const unsigned cnt = *L.n[r];
+    for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
+      const int2 x = L.p[r][i];
+      W[x.x] = x.y;
+    }
+  }
+}
+__global__ void k_apply_pairs(const int2* __restrict__ p, int64_t cnt, int32_t* __restrict__ W) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cnt; i += (int64_t)gridDim.x * blockDim.x)
+    W[p[i].x] = p[i].y;
+}
+
 
 // ------------------------------------------------------------------ NCCL
 struct NcclComm : Comm {
@@ -129,6 +182,41 @@ struct NcclComm : Comm {
   void allreduce_i32(glp_graph* g, const int32_t* send, int32_t* recv, size_t k) override {
     NCK(nccl_api().AllReduce(send, recv, k, ncclInt32, ncclSum, c, g->stream));
   }
+  // counts all-gathered (one host sync), then each rank's lists broadcast
+  // into one receive buffer per list (grouped), then applied in order
+  void exchange_changes(glp_graph* g, int32_t* W, const int2* const lists[2], const unsigned* const counts[2]) override {
+    NcclApi& A = nccl_api();
+    const int P = g->nranks;
+    unsigned* d = nullptr;
+    cuda_ok(cudaMallocAsync((void**)&d, sizeof(unsigned) * 2 * P, g->stream), "cudaMallocAsync");
+    cuda_ok(cudaMemcpyAsync(d + 2 * g->rank, counts[0], sizeof(unsigned), cudaMemcpyDeviceToDevice, g->stream), "copy");
+    cuda_ok(cudaMemcpyAsync(d + 2 * g->rank + 1, counts[1], sizeof(unsigned), cudaMemcpyDeviceToDevice, g->stream),
+            "copy");
+    NCK(A.AllGather(d + 2 * g->rank, d, 2, ncclUint32, c, g->stream));
+    std::vector<unsigned> all(2 * P);
+    cuda_ok(cudaMemcpyAsync(all.data(), d, sizeof(unsigned) * 2 * P, cudaMemcpyDeviceToHost, g->stream), "copy");
+    cuda_ok(cudaStreamSynchronize(g->stream), "sync");
+    cudaFreeAsync(d, g->stream);
+    for (int j = 0; j < 2; ++j) {
+      int64_t tot = 0;
+      for (int r = 0; r < P; ++r) tot += all[2 * r + j];
+      if (tot == 0) continue;
+      int2* recv = nullptr;
+      cuda_ok(cudaMallocAsync((void**)&recv, sizeof(int2) * tot, g->stream), "cudaMallocAsync");
+      NCK(A.GroupStart());
+      int64_t at = 0;
+      for (int r = 0; r < P; ++r) {
+        const unsigned k = all[2 * r + j];
+        if (k) NCK(A.Broadcast(r == g->rank ? (const void*)lists[j] : (const void*)(recv + at), recv + at,
+                               (size_t)k * 2, ncclInt32, r, c, g->stream));
+        at += k;
+      }
+      NCK(A.GroupEnd());
+      k_apply_pairs<<<g->sms * 2, 256, 0, g->stream>>>(recv, tot, W);  // own pairs rewrite own values: harmless
+      cuda_ok(cudaGetLastError(), "k_apply_pairs");
+      cudaFreeAsync(recv, g->stream);
+    }
+  }
   void merge_flags(glp_graph* g, uint8_t* flag) override {
     NcclApi& A = nccl_api();
     if (g->equal_slices) {
@@ -141,7 +229,6 @@ struct NcclComm : Comm {
 };
 
 // ------------------------------------------------------------------ local group
-constexpr int kMaxLocalRanks = 16;
 struct Peers {
   const void* p[kMaxLocalRanks];
   int nranks;
@@ -229,6 +316,11 @@ struct LocalComm : Comm {
   cudaEvent_t ready = nullptr, done = nullptr;
   unsigned long long* stage = nullptr;  // allreduce_u64 send copy
   size_t stage_k = 0;
+  struct Desc {
+    const int2* p[2];
+    const unsigned* n[2];
+  };
+  Desc host_desc;  // this rank's change lists (device pointers), read by the peers' host threads
 
   LocalComm(glp_graph* g, glp_local_group* grp_) : grp(grp_), rank(g->rank) {
     if (grp->nranks != g->nranks) throw Err{GLP_ERR_INVALID_ARGUMENT, "local group size != nranks"};
@@ -310,6 +402,27 @@ struct LocalComm : Comm {
   void allreduce_i32(glp_graph* g, const int32_t* send, int32_t* recv, size_t k) override {
     collective(g, send, [&](const Peers& pe) {
       k_sum_i32<<<g->sms * 4, 256, 0, g->stream>>>(pe, recv, (int64_t)k);
+    });
+  }
+  // peers' lists read in place: publish a device descriptor of this rank's
+  // two lists, then apply every other rank's t-1 lists, then their t lists
+  void exchange_changes(glp_graph* g, int32_t* W, const int2* const lists[2], const unsigned* const counts[2]) override {
+    Desc h;
+    h.p[0] = lists[0]; h.p[1] = lists[1]; h.n[0] = counts[0]; h.n[1] = counts[1];
+    host_desc = h;  // peers read the host copy (pointers are process-wide)
+    collective(g, &host_desc, [&](const Peers& pe) {
+      for (int j = 0; j < 2; ++j) {
+        ChgLists L;
+        memset(&L, 0, sizeof(L));
+        L.nranks = g->nranks;
+        L.skip = rank;
+        for (int r = 0; r < g->nranks; ++r) {
+          const Desc* dr = (const Desc*)pe.p[r];
+          L.p[r] = dr->p[j];
+          L.n[r] = dr->n[j];
+        }
+        k_apply_changes<<<g->sms * 2, 256, 0, g->stream>>>(L, W);
+      }
     });
   }
   void merge_flags(glp_graph* g, uint8_t* flag) override {

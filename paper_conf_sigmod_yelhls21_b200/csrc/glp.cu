@@ -150,6 +150,7 @@ glp_params default_params() {
   p.validate = 1;
   p.profile = 0;
   p.dense_divisor = 4;
+  p.sparse_exchange = -1;
   return p;
 }
 
@@ -945,6 +946,16 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     CK(cudaGetLastError());
     g->init_launches += 1;
   }
+  // change lists of t-1 and t for the sparse exchange (CLASSIC / SEEDED, P > 1)
+  const bool track_changes = g->comm && variant != GLP_VARIANT_LLP && p.sparse_exchange != 0;
+  if (track_changes) {
+    if (!g->chg[0]) {
+      g->chg[0] = dalloc<int2>(g, std::max<int64_t>(g->nl, 1));
+      g->chg[1] = dalloc<int2>(g, std::max<int64_t>(g->nl, 1));
+      g->chg_n = dalloc<unsigned>(g, 2);
+    }
+    CK(cudaMemsetAsync(g->chg_n, 0, 2 * sizeof(unsigned), s));  // nothing changed at t = 0 (seeds are in L0 and L1)
+  }
   int rb = 0;  // R = L[rb], W = L[1-rb]
   int fb = 0;  // flags read this iteration
   bool dense = true;
@@ -1035,9 +1046,32 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
       default: launches += launch_mfl<V_LLP>(g, a, prof, pend, used); break;
     }
+    int exch = 0;
     if (g->comm) {
-      // sharded LLP replicates (label, V) pairs after the histogram instead
-      if (!llp_shard) timed(g, prof, 6, pend, used, s, [&] { g->comm->allgather(g, g->L[1 - rb], sizeof(int32_t)); });
+      // sharded LLP replicates (label, V) pairs after the histogram instead;
+      // CLASSIC / SEEDED may exchange only the changed vertices (§8(f)1)
+      if (track_changes) {
+        const int ct = t & 1;
+        CK(cudaMemsetAsync(g->chg_n + ct, 0, sizeof(unsigned), s));
+        if (g->nl) k_collect_changes<<<ga, 256, 0, s>>>(g->so, g->L[1 - rb], g->nl, g->vb, t, g->chg[ct], g->chg_n + ct);
+        CK(cudaGetLastError());
+        launches += 1;
+      }
+      const bool sparse = track_changes && (p.sparse_exchange == 1 ||
+                                            (p.sparse_exchange < 0 && t >= 2 &&
+                                             (double)changed_last * 4.0 * g->nranks < (double)g->n));
+      if (sparse) {
+        const int ct = t & 1;
+        const int2* lists[2] = {g->chg[1 - ct], g->chg[ct]};
+        const unsigned* counts[2] = {g->chg_n + (1 - ct), g->chg_n + ct};
+        timed(g, prof, 6, pend, used, s, [&] { g->comm->exchange_changes(g, g->L[1 - rb], lists, counts); });
+        exch = 2;
+      } else if (!llp_shard) {
+        timed(g, prof, 6, pend, used, s, [&] { g->comm->allgather(g, g->L[1 - rb], sizeof(int32_t)); });
+        exch = 1;
+      } else {
+        exch = 3;
+      }
       g->comm->allreduce_u64(g, (unsigned long long*)g->d_cnt, kNumCounters * sizeof(Counters) / sizeof(unsigned long long));
     }
     CK(cudaMemcpyAsync(g->h_cnt, g->d_cnt, kNumCounters * sizeof(Counters), cudaMemcpyDeviceToHost, s));
@@ -1057,6 +1091,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     st.active_vertices = (int64_t)tot.verts;
     st.active_arcs = (int64_t)tot.arcs;
     st.dense = dense ? 1 : 0;
+    st.exchange = exch;
     st.cms_rows = (int64_t)tot.pad0;
     st.cms_rescans = (int64_t)tot.pad[0];
     st.cms_fallbacks = (int64_t)tot.pad[1];

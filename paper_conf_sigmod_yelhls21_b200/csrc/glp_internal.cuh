@@ -277,6 +277,8 @@ struct glp_graph {
   int32_t* redo_m = nullptr;                         // [n_rows]
   int32_t* redo_l = nullptr;                         // [n_rows]
   int32_t* push_big = nullptr;                       // [nl] changed rows of >= kPushBig arcs (push)
+  int2* chg[2] = {nullptr, nullptr};                 // sparse exchange: (id, label) of owned changes, t-1 / t
+  unsigned* chg_n = nullptr;                         // [2] their counts
   unsigned* push_nbig = nullptr;
   glp::Sched* d_sched = nullptr;
   int64_t bin_verts[glp::NBINS] = {0}, bin_arcs[glp::NBINS] = {0};

@@ -137,3 +137,21 @@ def test_failed_rank_releases_group():
             grp._all(body)
     finally:
         grp.close()
+
+
+@pytest.mark.parametrize("mode", [1, -1])
+@pytest.mark.parametrize("P", [2, 3])
+def test_sparse_exchange(mode, P):
+    """§8(f)1: only the changed vertices' (id, label) pairs of t-1 and t are
+    exchanged (forced every iteration, or automatically once few vertices
+    change); labels and iteration counts stay bit-exact."""
+    for csr, variant, seeds, mi in [(graphs.rmat(14, seed=8), "classic", None, 20),
+                                    (graphs.sbm(n=20_010, k=30, m=200_000, mu=0.1, seed=2), "classic", None, 30),
+                                    (graphs.taobao(users=40_000, items=10_000, pairs=200_000, rings=40, seed=5)[0],
+                                     "seeded", np.array([3, 500, 40_000, 45_000], dtype=np.int32), 30)]:
+        ref, labs, infos, st, ks, b = check(csr, P, variant, mi, seeds=seeds, sparse_exchange=mode)
+        ex = [s["exchange"] for s in st[0]]
+        if mode == 1:
+            assert set(ex) == {2}
+        else:
+            assert 2 in ex and 1 in ex  # dense early, sparse once changes are few

@@ -324,6 +324,12 @@ def test_nccl_exchange_path_single_rank():
             lab = g.labels("cpu").numpy()
         ref = oracle.run(csr, glp.VARIANTS[variant], 12, gamma=gamma, threads=8)
         assert info.iterations == ref.iterations and (lab == ref.labels).all()
+        if variant == "classic":  # the NCCL sparse exchange calls (§8(f)1), one rank
+            with glp.Graph(c, rank=0, nranks=1, nccl_unique_id=glp.glp_nccl_unique_id(), device=0) as g:
+                info = g.run(variant, 12, seeds, sparse_exchange=1)
+                lab = g.labels("cpu").numpy()
+                assert {s["exchange"] for s in g.iter_stats()} == {2}
+            assert info.iterations == ref.iterations and (lab == ref.labels).all()
     csr, seeds = graphs.taobao(users=40_000, items=10_000, pairs=200_000, rings=40, seed=5)
     uid = glp.glp_nccl_unique_id()
     with glp.Graph(csr.to("cuda"), rank=0, nranks=1, nccl_unique_id=uid, device=0) as g:
