@@ -626,6 +626,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaMemsetAsync(g->flag[0], 0, std::max<int64_t>(npad, 1), g->stream));
     CK(cudaMemsetAsync(g->flag[1], 0, std::max<int64_t>(npad, 1), g->stream));
     g->d_cnt = dalloc<Counters>(g, kNumCounters);
+    g->push_big = dalloc<int32_t>(g, std::max<int64_t>(g->nl, 1));  // frontier push: long changed rows
+    g->push_nbig = dalloc<unsigned>(g, 1);
     CK(cudaMallocHost(&g->h_cnt, kNumCounters * sizeof(Counters)));
     CK(cudaEventCreate(&g->ev_a));
     CK(cudaEventCreate(&g->ev_b));
@@ -735,10 +737,6 @@ void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t&
 // frontier push of the vertices changed at t (k_push + its long-row pass)
 void push(glp_graph* g, int32_t t, uint8_t* flag) {
   cudaStream_t s = g->stream;
-  if (!g->push_big) {
-    g->push_big = dalloc<int32_t>(g, std::max<int64_t>(g->nl, 1));
-    g->push_nbig = dalloc<unsigned>(g, 1);
-  }
   CK(cudaMemsetAsync(g->push_nbig, 0, sizeof(unsigned), s));
   k_push<<<g->grid_aux, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, flag, g->push_big,
                                      g->push_nbig);

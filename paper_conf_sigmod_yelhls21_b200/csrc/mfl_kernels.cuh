@@ -728,6 +728,92 @@ __device__ __forceinline__ bool warp_quads_increasing(const int (&x)[4], int bas
 }
 
 // ---------------------------------------------------------------------------
+// Sort-and-count of one short row held by a warp (<= 128 arcs, 4 per lane:
+// element i = 4 * lane + j, the load_round layout).  For rows whose labels are
+// mostly distinct (t = 2..3) this replaces ~25 instructions of hash insert
+// per label by a bitonic sort in registers (28 compare-exchange stages, 15 of
+// them across lanes) plus a run-length scan: the per-row count the paper's
+// segmented-sort baseline computes [P:126], kept in registers instead of a
+// global neighbour-label array.  Invalid arcs (-1 label, padding) sort last as
+// INT_MAX and never vote.  Observes every run (count, label) into b, returns
+// this lane's number of runs (distinct labels).
+#ifndef GLP_W_SORT
+#define GLP_W_SORT 1
+#endif
+#ifndef GLP_W_SORT_MAX
+#define GLP_W_SORT_MAX 64  // rows up to this many arcs (<= kWRound) take the sort path
+                          // A/B (sort 64 / 128 / off): SBM 5.33 / 5.35 / 5.60 ms, R24 17.99 / 17.97 / 18.0-18.4,
+                          // R24 LLP 194.7 / 196.7 / 194.1 ms per run
+#endif
+template <int VAR, int K>
+__device__ __forceinline__ unsigned warp_sort_count(int (&v)[K], const MflArgs& a, Best<VAR>& b) {
+  constexpr int N = 32 * K;
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int j = 0; j < K; ++j) v[j] = v[j] < 0 ? INT_MAX : v[j];
+  // bitonic sort of N keys, ascending in i = K * lane + j
+#pragma unroll
+  for (int k = 2; k <= N; k <<= 1) {
+#pragma unroll
+    for (int st = k >> 1; st > 0; st >>= 1) {
+      if (st >= K) {
+        const int ls = st / K;  // partner lane = lane ^ ls, same j
+#pragma unroll
+        for (int j = 0; j < K; ++j) {
+          const int o = __shfl_xor_sync(kFull, v[j], ls);
+          const int i = K * lane + j;
+          const bool up = (i & k) == 0;
+          const bool low = (lane & ls) == 0;  // this element has the smaller index of the pair
+          v[j] = (low == up) ? min(v[j], o) : max(v[j], o);
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < K; ++j) {
+          const int pj = j ^ st;
+          if (pj > j) {
+            const int i = K * lane + j;
+            const bool up = (i & k) == 0;
+            const int x = v[j], y = v[pj];
+            v[j] = up ? min(x, y) : max(x, y);
+            v[pj] = up ? max(x, y) : min(x, y);
+          }
+        }
+      }
+    }
+  }
+  // run starts: element differs from its predecessor
+  const int prev_last = __shfl_up_sync(kFull, v[K - 1], 1);
+  bool start[K];
+  start[0] = v[0] != INT_MAX && (lane == 0 || prev_last != v[0]);
+#pragma unroll
+  for (int j = 1; j < K; ++j) start[j] = v[j] != INT_MAX && v[j] != v[j - 1];
+  // end of each run = position of the next start (or of the first INT_MAX)
+  int nvalid = 0;
+#pragma unroll
+  for (int j = 0; j < K; ++j) nvalid += __popc(__ballot_sync(kFull, v[j] != INT_MAX));
+  int first_start = K;
+#pragma unroll
+  for (int j = K - 1; j >= 0; --j) first_start = start[j] ? j : first_start;
+  const unsigned lanes_with = __ballot_sync(kFull, first_start < K);
+  const unsigned after = lane < 31 ? (lanes_with >> (lane + 1)) : 0u;
+  const int nl = after ? lane + __ffs(after) : 32;             // next lane holding a start
+  const int nfs = __shfl_sync(kFull, first_start, nl & 31);  // its first start
+  const int next_lane_pos = nl < 32 ? K * nl + nfs : nvalid;
+  unsigned distinct = 0;
+  int nxt = next_lane_pos;
+#pragma unroll
+  for (int j = K - 1; j >= 0; --j) {
+    if (start[j]) {
+      const unsigned cnt = (unsigned)(nxt - (K * lane + j));
+      b.observe(cnt, (unsigned)v[j], a);  // LLP: V[l] gathered once per distinct label
+      ++distinct;
+      nxt = K * lane + j;
+    }
+  }
+  return distinct;  // this lane's runs (the caller reduces over the warp)
+}
+
+// ---------------------------------------------------------------------------
 // mfl_warp: one warp per row of class W (few distinct labels): per-warp shared
 // table of pow2 >= 4*pred slots (<= 512), one 128-bit load per lane per
 // round (128 arcs per warp; 256-arc rounds measured 2 % slower: most W rows
@@ -812,7 +898,9 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       const unsigned tsz =
           min(max(64u, 1u << (32 - __clz(GLP_W_LOAD * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
       const Table tab{wtabs + (size_t)wid * kWSlots, tsz};
-      tab.clear(lane, 32);
+      // rows of <= 128 arcs predicted mostly distinct: sort-and-count, no table
+      const bool wsort = GLP_W_SORT && d <= GLP_W_SORT_MAX && !(pred & kMonoTried) && 4u * (pred & kPredMask) > (unsigned)d;
+      if (!wsort) tab.clear(lane, 32);
       if (lane == 0) s_over[wid] = 0;
       __syncwarp();
       Best<VAR> b;
@@ -874,6 +962,20 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
             fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v, hot);
           }
         }
+        if (wsort) {  // the whole row is this round (d <= kWRound)
+          if (d <= 64) {
+            // 2 per lane: lane L takes arcs 2L, 2L+1 from lane L/2's quad
+            const int src = lane >> 1;
+            const int q0 = __shfl_sync(kFull, l[0], src), q1 = __shfl_sync(kFull, l[1], src);
+            const int q2 = __shfl_sync(kFull, l[2], src), q3 = __shfl_sync(kFull, l[3], src);
+            int l2[2] = {(lane & 1) ? q2 : q0, (lane & 1) ? q3 : q1};
+            fresh = warp_sort_count<VAR, 2>(l2, a, b);
+          } else {
+            int l4[4] = {l[0], l[1], l[2], l[3]};
+            fresh = warp_sort_count<VAR, 4>(l4, a, b);
+          }
+          break;
+        }
         if (kWRound == 256 && d - off > 128) {  // warp-uniform
           fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v, hot);
         } else {
@@ -889,7 +991,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       if (over) {
         if (lane == 0) a.redo_out[atomicAdd(a.redo_out_n, 1u)] = base + jl * nwarps + gw;
       } else {
-        if (a.LV == nullptr) table_scan<VAR>(tab, lane, 32, a, b);  // LLP (s_over's __syncwarp ended the count)
+        if (a.LV == nullptr && !wsort) table_scan<VAR>(tab, lane, 32, a, b);  // LLP (s_over's __syncwarp ended the count)
         b.warp_reduce();
         fresh = __reduce_add_sync(kFull, fresh);
         if (lane == jl) {
