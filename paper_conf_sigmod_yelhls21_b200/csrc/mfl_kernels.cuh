@@ -455,10 +455,20 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
 #ifndef GLP_PRED_EXTRAP
 #define GLP_PRED_EXTRAP 1
 #endif
+// LLP does not converge: with gamma > 0 the labels oscillate with period 2
+// (the distinct counts alternate spread / collapsed), so the count of t-2 is
+// the prediction (GLP_PRED_LLP 1), or the larger of t-1 and t-2 (2); 0 =
+// the converging extrapolation above.
+#ifndef GLP_PRED_LLP
+#define GLP_PRED_LLP 2  // A/B (0 / 1 / 2): R24 LLP 194.6 / 185.0 / 175.2 ms, R28 LLP 4103 / - / 3860 ms per run
+#endif
+template <int VAR>
 __device__ __forceinline__ unsigned pred_est(unsigned raw, unsigned rawprev, unsigned cap) {
   unsigned p = raw & kPredMask;
   const unsigned q = rawprev & kPredMask;
-  if (GLP_PRED_EXTRAP && q > p) p = (unsigned)(((unsigned long long)p * p) / q);
+  if (VAR == V_LLP && GLP_PRED_LLP == 1) p = q > 0 ? q : p;
+  else if (VAR == V_LLP && GLP_PRED_LLP == 2) p = max(p, q);
+  else if (GLP_PRED_EXTRAP && q > p) p = (unsigned)(((unsigned long long)p * p) / q);
   if (cap) p = min(p, cap);
   return max(p, 1u);
 }
@@ -862,7 +872,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       const unsigned raw = a.pred[il];
       // in this kernel bit 31 of mpred marks a sorted-row candidate
       const bool cand = mono_cand<VAR>(raw, a.pred_cap, mine.d);
-      mpred = pred_est(raw, a.pred_prev[il], a.pred_cap) | (cand ? kMonoTried : 0u);
+      mpred = pred_est<VAR>(raw, a.pred_prev[il], a.pred_cap) | (cand ? kMonoTried : 0u);
       ok = row_class(mpred & kPredMask, mine.d, cand, a.mono_kernel) == CLS_W;
       if (ok && !a.dense && !a.flag[a.vb + mine.v]) {
         ok = false;
@@ -1455,7 +1465,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
         ik = a.mode ? a.redo_in[k] : k;
         itk = a.items[ik];
         raw = a.pred[ik];
-        pe = pred_est(raw, a.pred_prev[ik], a.pred_cap);
+        pe = pred_est<VAR>(raw, a.pred_prev[ik], a.pred_cap);
         cnd = mono_cand<VAR>(raw, a.pred_cap, itk.d);
         if (!a.mode) {
           ok = row_class(pe, itk.d, cnd, a.mono_kernel) == CLS;

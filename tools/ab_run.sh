@@ -4,6 +4,6 @@
 wls=$1; reps=$2; shift 2
 for wl in $wls; do
   for v in "$@"; do
-    GLP_LIB=build/$v.so timeout 300 python tools/ab_time.py $wl $reps 2>&1 | grep '^{' || echo "{\"lib\": \"$v\", \"failed\": true}"
+    GLP_LIB=build/$v.so timeout 900 python tools/ab_time.py $wl $reps 2>&1 | grep '^{' || echo "{\"lib\": \"$v\", \"failed\": true}"
   done
 done
