@@ -638,6 +638,16 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       g->use_vl = !(novl && novl[0] == '1');
       const char* nomono = getenv("GLP_NO_MONO");
       g->use_mono = !(nomono && nomono[0] == '1');
+      const char* l2w = getenv("GLP_L2_WINDOW");
+      if (l2w && l2w[0] == '1') {
+        // persisting L2 set-aside up to the device maximum
+        int maxp = 0, maxw = 0;
+        CK(cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev));
+        CK(cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev));
+        CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp));
+        g->l2_window = maxp > 0 && maxw > 0;
+        g->l2_window_max = (size_t)maxw;
+      }
     }
 
     const int sms = g->sms;
@@ -769,6 +779,22 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
   if (cc) {
     CK(cudaEventRecord(g->xev[0], s0));
     for (auto x : g->xs) CK(cudaStreamWaitEvent(x, g->xev[0], 0));
+  }
+  if (g->l2_window) {
+    // A/B (GLP_L2_WINDOW=1): an L2 persisting access-policy window on the
+    // array every arc gathers from (L_{t-1}, or LV for LLP), on every stream
+    // that runs an MFL kernel of this iteration
+    cudaStreamAttrValue av;
+    memset(&av, 0, sizeof(av));
+    const void* base = a.LV ? (const void*)a.LV : (const void*)a.R;
+    const size_t bytes = (size_t)g->npad * (a.LV ? sizeof(int2) : sizeof(int32_t));
+    av.accessPolicyWindow.base_ptr = const_cast<void*>(base);
+    av.accessPolicyWindow.num_bytes = std::min(bytes, g->l2_window_max);
+    av.accessPolicyWindow.hitRatio = 1.0f;
+    av.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    av.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    CK(cudaStreamSetAttribute(s0, cudaStreamAttributeAccessPolicyWindow, &av));
+    for (auto x : g->xs) CK(cudaStreamSetAttribute(x, cudaStreamAttributeAccessPolicyWindow, &av));
   }
   if (g->n_giant) {  // giant rows: all blocks count segments into per-row global tables
     MflArgs b = r;

@@ -317,7 +317,9 @@ struct glp_graph {
   // xs[0] giant, xs[1] L, xs[2] M, xs[3] low; W and the redo chain on `stream`
   bool concurrent = true;
   bool use_vl = true;  // LLP gathers (label, V[label]) pairs from LV (GLP_NO_VL=1 disables)
-  bool use_mono = true;  // t = 1 sorted-row candidates in mfl_mono (GLP_NO_MONO=1: in the W kernel)
+  bool use_mono = true;
+  bool l2_window = false;     // A/B: persisting L2 window on the gathered array (GLP_L2_WINDOW=1)
+  size_t l2_window_max = 0;  // t = 1 sorted-row candidates in mfl_mono (GLP_NO_MONO=1: in the W kernel)
   int* col_bad = nullptr;  // create: col_idx range check flag (side stream)
   cudaStream_t xs[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaEvent_t xev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
