@@ -49,6 +49,9 @@ def _load():
         lib.glp_oracle_run_w.restype = ctypes.c_int
         lib.glp_oracle_run_w.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, ctypes.c_int32, P,
                                          ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, P, P, P, P]
+        lib.glp_oracle_slp.restype = ctypes.c_int
+        lib.glp_oracle_slp.argtypes = [ctypes.c_int64, P, P, ctypes.c_int32, ctypes.c_double, ctypes.c_int32,
+                                       ctypes.c_int32, P, P, P]
         lib.glp_oracle_modularity.restype = ctypes.c_double
         lib.glp_oracle_modularity.argtypes = [ctypes.c_int64, P, P, P]
         _lib = lib
@@ -130,6 +133,21 @@ def run_weighted(csr, weights, variant: int = CLASSIC, max_iters: int = 20, seed
     it = int(info[0])
     return OracleResult(labels[:n].copy(), changed[:it].copy(), it, int(info[1]),
                         None if tr is None else tr[:it, :n].copy())
+
+
+def run_slp(csr, K: int = 5, r: float = 0.0, max_iters: int = 20, threads: int = 1):
+    """Speaker-listener LP (see glp_oracle.c): returns (mem_labels [n, K],
+    mem_counts [n, K], speakers [n])."""
+    lib = _load()
+    n, off, col = _csr_np(csr)
+    ml = np.empty((max(n, 1), K), dtype=np.int32)
+    mc = np.empty((max(n, 1), K), dtype=np.int32)
+    sp = np.empty(max(n, 1), dtype=np.int32)
+    rc = lib.glp_oracle_slp(n, _ptr(off), _ptr(col), int(K), float(r), int(max_iters), int(threads), _ptr(ml),
+                            _ptr(mc), _ptr(sp))
+    if rc != 0:
+        raise ValueError(f"glp_oracle_slp failed rc={rc}")
+    return ml[:n].copy(), mc[:n].copy(), sp[:n].copy()
 
 
 def step(csr, variant: int, labels_prev, v_begin: int = 0, v_end=None, V=None, is_seed=None,
