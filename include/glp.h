@@ -58,7 +58,14 @@ typedef enum {
 typedef enum {
   GLP_VARIANT_CLASSIC = 0,
   GLP_VARIANT_SEEDED = 1,
-  GLP_VARIANT_LLP = 2
+  GLP_VARIANT_LLP = 2,
+  GLP_VARIANT_SLP = 3  /* speaker-listener LP [P:120]: each vertex keeps up to
+                          slp_max_labels candidate labels; per iteration its
+                          speaker label (the most frequent candidate) is what
+                          the neighbours count, and the MFL heard joins the
+                          candidates (R19).  Runs exactly max_iters iterations;
+                          glp_labels_get returns the speaker labels,
+                          glp_slp_memory_get the candidates                   */
 } glp_variant;
 
 typedef enum {
@@ -165,6 +172,11 @@ typedef struct {
                                   8192; 0 = 8192).  Testing / analysis        */
   int32_t cms_depth;           /* tail_cms: sketch rows d (1..8, width =
                                   8192 / d; 0 = 4)                             */
+  int32_t slp_max_labels;      /* SLP: candidate labels per vertex K, 1..16
+                                  (0 = 5 [P:270])                              */
+  double slp_threshold;        /* SLP: after iteration t a candidate whose count
+                                  is < slp_threshold * (t + 1) is dropped
+                                  (never the most frequent one); >= 0, default 0 */
   int32_t sparse_exchange;     /* nranks > 1, CLASSIC / SEEDED (§8(f)1): replace
                                   the label all-gather by an exchange of the
                                   changed vertices' (id, label) pairs of t-1
@@ -235,6 +247,13 @@ glp_status glp_graph_create(const glp_csr *csr, const glp_dist *dist, const glp_
  * info may be NULL.  Labels stay on the device (glp_labels_get). */
 glp_status glp_run(glp_graph *g, glp_variant variant, int32_t max_iters, const int32_t *seeds,
                    int64_t n_seeds, const glp_params *params, glp_run_info *info);
+
+/* SLP candidates of the last SLP run, in original vertex order, for this
+ * rank's rows [v_begin, v_end): labels_out / counts_out hold K entries per
+ * vertex (K = the run's slp_max_labels; -1 / 0 = empty slot), out_len >=
+ * (v_end - v_begin) * K; out_on_device as for glp_labels_get. */
+glp_status glp_slp_memory_get(const glp_graph *g, int32_t *labels_out, int32_t *counts_out, int64_t out_len,
+                              int32_t out_on_device);
 
 /* Copy all n_global labels of the last run into out (out_on_device = 0: host
  * buffer, 1: device buffer), out_len >= n_global. */

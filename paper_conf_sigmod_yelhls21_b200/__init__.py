@@ -22,8 +22,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 # GLP_LIB: load another in-tree build of the same library (kernel A/B experiments)
 LIB_PATH = os.environ.get("GLP_LIB") or _build.LIB
 
-CLASSIC, SEEDED, LLP = 0, 1, 2
-VARIANTS = {"classic": CLASSIC, "seeded": SEEDED, "llp": LLP}
+CLASSIC, SEEDED, LLP, SLP = 0, 1, 2, 3
+VARIANTS = {"classic": CLASSIC, "seeded": SEEDED, "llp": LLP, "slp": SLP}
 STOP_MAX_ITERS, STOP_FIXED_POINT, STOP_TWO_CYCLE = 0, 1, 2
 STOP_NAMES = {0: "max_iters", 1: "fixed_point", 2: "two_cycle"}
 STATUS = {0: "GLP_OK", 1: "GLP_ERR_INVALID_ARGUMENT", 2: "GLP_ERR_INVALID_GRAPH",
@@ -57,7 +57,9 @@ class glp_params(ctypes.Structure):
                 ("validate", ctypes.c_int32), ("profile", ctypes.c_int32),
                 ("dense_divisor", ctypes.c_int32), ("debug_pred_cap", ctypes.c_int32),
                 ("llp_hist", ctypes.c_int32), ("host_arcs", ctypes.c_int32), ("tail_cms", ctypes.c_int32),
-                ("cms_ht_slots", ctypes.c_int32), ("cms_depth", ctypes.c_int32), ("sparse_exchange", ctypes.c_int32)]
+                ("cms_ht_slots", ctypes.c_int32), ("cms_depth", ctypes.c_int32),
+                ("slp_max_labels", ctypes.c_int32), ("slp_threshold", ctypes.c_double),
+                ("sparse_exchange", ctypes.c_int32)]
 
 
 class glp_run_info(ctypes.Structure):
@@ -80,8 +82,8 @@ class glp_kernel_stat(ctypes.Structure):
 
 EXPORTS = ["glp_nccl_unique_id", "glp_partition", "glp_graph_create", "glp_run", "glp_labels_get",
            "glp_iter_stats", "glp_kernel_stats", "glp_graph_info", "glp_graph_destroy",
-           "glp_local_group_create", "glp_local_group_destroy", "glp_struct_sizes", "glp_last_error",
-           "glp_version"]
+           "glp_local_group_create", "glp_local_group_destroy", "glp_struct_sizes", "glp_slp_memory_get",
+           "glp_last_error", "glp_version"]
 
 _lib = None
 
@@ -110,6 +112,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "glp_local_group_create": [I32, P],
         "glp_local_group_destroy": [P],
         "glp_struct_sizes": [P, I32],
+        "glp_slp_memory_get": [P, P, P, I64, I32],
     }
     for name, args in sig.items():
         fn = getattr(lib, name)
@@ -131,7 +134,8 @@ def _check(st: int):
 def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = True,
                 validate: bool = True, profile: bool = False, dense_divisor: int = 0,
                 debug_pred_cap: int = 0, llp_hist: int = 0, host_arcs: bool = False, tail_cms: bool = False,
-                cms_ht_slots: int = 0, cms_depth: int = 0, sparse_exchange: int = -1) -> glp_params:
+                cms_ht_slots: int = 0, cms_depth: int = 0, sparse_exchange: int = -1, slp_max_labels: int = 0,
+                slp_threshold: float = 0.0) -> glp_params:
     p = glp_params()
     p.struct_size = ctypes.sizeof(glp_params)
     p.gamma = float(gamma)
@@ -147,6 +151,8 @@ def make_params(gamma: float = 0.0, frontier: int = -1, stop_on_2cycle: bool = T
     p.cms_ht_slots = int(cms_ht_slots)
     p.cms_depth = int(cms_depth)
     p.sparse_exchange = int(sparse_exchange)
+    p.slp_max_labels = int(slp_max_labels)
+    p.slp_threshold = float(slp_threshold)
     return p
 
 
@@ -236,7 +242,8 @@ def glp_graph_create(n_global: int, row_offsets: torch.Tensor, col_idx: torch.Te
 def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, gamma: float = 0.0,
             frontier: int = -1, stop_on_2cycle: bool = True, profile: bool = False,
             dense_divisor: int = 0, debug_pred_cap: int = 0, llp_hist: int = 0, tail_cms: bool = False,
-            cms_ht_slots: int = 0, cms_depth: int = 0, sparse_exchange: int = -1) -> dict:
+            cms_ht_slots: int = 0, cms_depth: int = 0, sparse_exchange: int = -1, slp_max_labels: int = 0,
+            slp_threshold: float = 0.0) -> dict:
     import numpy as np
     lib = load_library()
     sd = None
@@ -248,7 +255,7 @@ def glp_run(handle, variant: int = CLASSIC, max_iters: int = 20, seeds=None, *, 
     prm = make_params(gamma=gamma, frontier=frontier, stop_on_2cycle=stop_on_2cycle, profile=profile,
                       dense_divisor=dense_divisor, debug_pred_cap=debug_pred_cap, llp_hist=llp_hist,
                       tail_cms=tail_cms, cms_ht_slots=cms_ht_slots, cms_depth=cms_depth,
-                      sparse_exchange=sparse_exchange)
+                      sparse_exchange=sparse_exchange, slp_max_labels=slp_max_labels, slp_threshold=slp_threshold)
     _check(lib.glp_run(handle, int(variant), int(max_iters), None if sd is None else sd.ctypes.data, ns,
                        ctypes.byref(prm), ctypes.byref(info)))
     return dict(iterations=info.iterations, stop_reason=info.stop_reason,
@@ -292,6 +299,15 @@ def glp_graph_info(handle) -> dict:
     names = ["isolated", "low", "mid", "high", "huge"]
     bins = {nm: dict(vertices=int(out[2 + 2 * i]), arcs=int(out[3 + 2 * i])) for i, nm in enumerate(names)}
     return dict(n=int(out[0]), nnz=int(out[1]), bins=bins, max_degree=int(out[12]), low_chunks=int(out[13]))
+
+
+def glp_slp_memory_get(handle, n_rows: int, K: int):
+    """SLP candidates of this rank's rows: (labels [n_rows, K], counts [n_rows, K]) int32 CPU tensors."""
+    lab = torch.empty((n_rows, K), dtype=torch.int32)
+    cnt = torch.empty((n_rows, K), dtype=torch.int32)
+    _check(load_library().glp_slp_memory_get(handle, lab.data_ptr() if lab.numel() else None,
+                                             cnt.data_ptr() if cnt.numel() else None, lab.numel(), 0))
+    return lab, cnt
 
 
 def glp_local_group_create(nranks: int):
@@ -378,6 +394,10 @@ class Graph:
 
     def iter_stats(self):
         return glp_iter_stats(self.handle)
+
+    def slp_memory(self, K: int = 5, n_rows=None):
+        """Candidates of the last SLP run (K = the run's slp_max_labels)."""
+        return glp_slp_memory_get(self.handle, self.n if n_rows is None else n_rows, K)
 
     def kernel_stats(self):
         return glp_kernel_stats(self.handle)

@@ -211,6 +211,64 @@ __global__ void k_hist(const int32_t* __restrict__ L, int64_t n, int32_t* __rest
   }
 }
 
+// ---- SLP (§8(f)3, speaker-listener LP [P:120]; readings R19).  Memory of
+// owned vertex q (local internal id): K slots (label, count), label -1 = empty.
+__device__ __forceinline__ int slp_argmax(const int32_t* l, const int32_t* c, int K) {
+  int b = -1;
+  for (int k = 0; k < K; ++k) {
+    if (l[k] < 0) continue;
+    if (b < 0 || c[k] > c[b] || (c[k] == c[b] && l[k] < l[b])) b = k;
+  }
+  return b;
+}
+__global__ void k_slp_init(int32_t* __restrict__ ml, int32_t* __restrict__ mc, const int32_t* __restrict__ orig,
+                           int64_t nl, int64_t vb, int K) {
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nl; q += (int64_t)gridDim.x * blockDim.x)
+    for (int k = 0; k < K; ++k) {
+      ml[q * K + k] = k == 0 ? orig[vb + q] : -1;
+      mc[q * K + k] = k == 0 ? 1 : 0;
+    }
+}
+// listener: the MFL heard (W, written by the classic MFL kernels from the
+// speakers) joins the candidates of every owned vertex with neighbours; then
+// the threshold; then the speaker of t+1 (the most frequent candidate, min
+// label on ties) is written to W for every owned vertex
+__global__ void k_slp_listen_speak(int32_t* __restrict__ ml, int32_t* __restrict__ mc, int32_t* __restrict__ W,
+                                   const int32_t* __restrict__ ideg, int64_t nl, int64_t vb, int K, double thr) {
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nl; q += (int64_t)gridDim.x * blockDim.x) {
+    int32_t* l = ml + q * K;
+    int32_t* c = mc + q * K;
+    if (ideg[q] > 0) {
+      const int32_t m = W[vb + q];
+      int hit = -1, empty = -1, low = -1;
+      for (int k = 0; k < K; ++k) {
+        if (l[k] == m) hit = k;
+        if (l[k] < 0 && empty < 0) empty = k;
+        if (l[k] >= 0 && (low < 0 || c[k] < c[low] || (c[k] == c[low] && l[k] > l[low]))) low = k;
+      }
+      if (hit >= 0) c[hit] += 1;
+      else if (empty >= 0) { l[empty] = m; c[empty] = 1; }
+      else { l[low] = m; c[low] = 1; }
+    }
+    const int keep = slp_argmax(l, c, K);
+    for (int k = 0; k < K; ++k)
+      if (k != keep && l[k] >= 0 && (double)c[k] < thr) { l[k] = -1; c[k] = 0; }
+    W[vb + q] = l[keep];
+  }
+}
+// glp_slp_memory_get: original order, owned rows [vb, ve)
+__global__ void k_slp_unpermute(const int32_t* __restrict__ ml, const int32_t* __restrict__ mc,
+                                const int32_t* __restrict__ pos, int64_t vb, int64_t ve, int K,
+                                int32_t* __restrict__ ol, int32_t* __restrict__ oc) {
+  for (int64_t v = vb + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ve; v += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t q = pos[v] - vb;
+    for (int k = 0; k < K; ++k) {
+      ol[(v - vb) * K + k] = ml[q * K + k];
+      oc[(v - vb) * K + k] = mc[q * K + k];
+    }
+  }
+}
+
 // L2 flush helper for benchmarks (writes a buffer larger than L2).
 __global__ void k_fill(uint4* __restrict__ p, int64_t n16, unsigned x) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n16; i += (int64_t)gridDim.x * blockDim.x)

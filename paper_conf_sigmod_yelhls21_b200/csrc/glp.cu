@@ -906,7 +906,15 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
               const glp_params* prm, glp_run_info* info) {
   if (!g) fail(GLP_ERR_INVALID_ARGUMENT, "graph is NULL");
   glp_params p = get_params(prm);
-  if (variant < GLP_VARIANT_CLASSIC || variant > GLP_VARIANT_LLP) fail(GLP_ERR_INVALID_ARGUMENT, "unknown variant");
+  if (variant < GLP_VARIANT_CLASSIC || variant > GLP_VARIANT_SLP) fail(GLP_ERR_INVALID_ARGUMENT, "unknown variant");
+  const bool slp = variant == GLP_VARIANT_SLP;
+  const int slp_k = p.slp_max_labels > 0 ? p.slp_max_labels : 5;
+  if (slp) {
+    if (slp_k > 16) fail(GLP_ERR_INVALID_ARGUMENT, "slp_max_labels must be in [1, 16]");
+    if (!(p.slp_threshold >= 0.0) || !std::isfinite(p.slp_threshold))
+      fail(GLP_ERR_INVALID_ARGUMENT, "slp_threshold must be finite and >= 0");
+    if (g->weighted) fail(GLP_ERR_UNSUPPORTED, "SLP on a weighted graph is not supported");
+  }
   if (max_iters < 0) fail(GLP_ERR_INVALID_ARGUMENT, "max_iters < 0");
   if (variant == GLP_VARIANT_LLP) {
     if (!std::isfinite(p.gamma) || p.gamma < 0) fail(GLP_ERR_INVALID_ARGUMENT, "gamma must be finite and >= 0");
@@ -920,7 +928,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     if (seeds[i] < 0 || seeds[i] >= g->n) fail(GLP_ERR_INVALID_ARGUMENT, "seed id out of range");
   if (p.frontier == 1 && !g->symmetric)
     fail(GLP_ERR_INVALID_ARGUMENT, "frontier=1 needs a symmetric graph (glp_csr.symmetric)");
-  const bool use_frontier = variant != GLP_VARIANT_LLP && g->symmetric && p.frontier != 0;
+  // SLP: the speakers change by the memory rule, not by the neighbours alone:
+  // full sweeps (R19)
+  const bool use_frontier = variant != GLP_VARIANT_LLP && !slp && g->symmetric && p.frontier != 0;
   const bool prof = p.profile != 0;
 
   CK(cudaSetDevice(g->device));
@@ -971,7 +981,20 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     g->init_launches += 1;
   }
   // change lists of t-1 and t for the sparse exchange (CLASSIC / SEEDED, P > 1)
-  const bool track_changes = g->comm && variant != GLP_VARIANT_LLP && p.sparse_exchange != 0;
+  const bool track_changes = g->comm && variant != GLP_VARIANT_LLP && !slp && p.sparse_exchange != 0;
+  if (slp) {
+    // memory M^0: slot 0 = (own label, 1); the speakers of t = 1 are L_0
+    if (g->slp_cap < slp_k) {
+      g->slp_l = dalloc<int32_t>(g, std::max<int64_t>(g->nl * slp_k, 1));
+      g->slp_c = dalloc<int32_t>(g, std::max<int64_t>(g->nl * slp_k, 1));
+      g->slp_cap = slp_k;
+    }
+    g->slp_k = slp_k;
+    if (g->nl) k_slp_init<<<ga, 256, 0, s>>>(g->slp_l, g->slp_c, g->orig, g->nl, g->vb, slp_k);
+    CK(cudaGetLastError());
+    g->init_launches += 1;
+  }
+  g->slp_valid = false;
   if (track_changes) {
     if (!g->chg[0]) {
       g->chg[0] = dalloc<int2>(g, std::max<int64_t>(g->nl, 1));
@@ -1068,7 +1091,17 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     } else switch (variant) {
       case GLP_VARIANT_CLASSIC: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       case GLP_VARIANT_SEEDED: launches += launch_mfl<V_SEEDED>(g, a, prof, pend, used); break;
+      case GLP_VARIANT_SLP: launches += launch_mfl<V_CLASSIC>(g, a, prof, pend, used); break;
       default: launches += launch_mfl<V_LLP>(g, a, prof, pend, used); break;
+    }
+    if (slp) {
+      // listener update + threshold + the speakers of t+1, written to W
+      // before the exchange replicates W
+      if (g->nl)
+        k_slp_listen_speak<<<ga, 256, 0, s>>>(g->slp_l, g->slp_c, g->L[1 - rb], g->ideg, g->nl, g->vb, slp_k,
+                                              p.slp_threshold * (double)(t + 1));
+      CK(cudaGetLastError());
+      launches += 1;
     }
     int exch = 0;
     if (g->comm) {
@@ -1131,7 +1164,9 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     arcs_total += st.active_arcs;
     // stop rule (R8): fixed point, or L_t == L_{t-2} (d2 == 0) with changes
     bool stop = false;
-    if (st.changed == 0) { reason = GLP_STOP_FIXED_POINT; stop = true; }
+    // (SLP runs max_iters iterations: its memories keep changing)
+    if (slp) {
+    } else if (st.changed == 0) { reason = GLP_STOP_FIXED_POINT; stop = true; }
     else if (p.stop_on_2cycle && t >= 2 && st.d2 == 0) { reason = GLP_STOP_TWO_CYCLE; stop = true; }
     // frontier of t+1: dense when the changed vertices touch > nnz/divisor arcs
     const int nf = 1 - fb;
@@ -1200,6 +1235,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   CK(cudaEventElapsedTime(&run_ms, ev_run0, ev_run1));
   g->cur = rb;
   g->has_run = true;
+  g->slp_valid = slp;
   if (info) {
     info->iterations = iters;
     info->stop_reason = reason;
@@ -1257,6 +1293,39 @@ glp_status glp_labels_get(const glp_graph* g, int32_t* out, int64_t out_len, int
     if (!out_on_device)
       CK(cudaMemcpyAsync(out, dst, g->n * sizeof(int32_t), cudaMemcpyDeviceToHost, g->stream));
     CK(cudaStreamSynchronize(g->stream));
+  });
+}
+
+glp_status glp_slp_memory_get(const glp_graph* g, int32_t* labels_out, int32_t* counts_out, int64_t out_len,
+                              int32_t out_on_device) {
+  return guard([&] {
+    if (!g) fail(GLP_ERR_INVALID_ARGUMENT, "graph is NULL");
+    if (!g->slp_valid) fail(GLP_ERR_STATE, "the last run was not an SLP run");
+    const int64_t need = g->nl * g->slp_k;
+    if (out_len < need) fail(GLP_ERR_INVALID_ARGUMENT, "out_len < (v_end - v_begin) * slp_max_labels");
+    if (need == 0) return;
+    if (!labels_out || !counts_out) fail(GLP_ERR_INVALID_ARGUMENT, "output is NULL");
+    CK(cudaSetDevice(g->device));
+    int32_t* dl = labels_out;
+    int32_t* dc = counts_out;
+    std::vector<void*> tmp;
+    if (!out_on_device) {
+      void *a = nullptr, *b = nullptr;
+      CK(cudaMalloc(&a, need * sizeof(int32_t)));
+      tmp.push_back(a);
+      CK(cudaMalloc(&b, need * sizeof(int32_t)));
+      tmp.push_back(b);
+      dl = (int32_t*)a;
+      dc = (int32_t*)b;
+    }
+    k_slp_unpermute<<<g->grid_aux, 256, 0, g->stream>>>(g->slp_l, g->slp_c, g->pos, g->vb, g->ve, g->slp_k, dl, dc);
+    CK(cudaGetLastError());
+    if (!out_on_device) {
+      CK(cudaMemcpyAsync(labels_out, dl, need * sizeof(int32_t), cudaMemcpyDeviceToHost, g->stream));
+      CK(cudaMemcpyAsync(counts_out, dc, need * sizeof(int32_t), cudaMemcpyDeviceToHost, g->stream));
+    }
+    CK(cudaStreamSynchronize(g->stream));
+    for (void* p : tmp) cudaFree(p);
   });
 }
 

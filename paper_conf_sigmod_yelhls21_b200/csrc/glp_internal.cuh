@@ -278,6 +278,10 @@ struct glp_graph {
   int32_t* redo_l = nullptr;                         // [n_rows]
   int32_t* push_big = nullptr;                       // [nl] changed rows of >= kPushBig arcs (push)
   int2* chg[2] = {nullptr, nullptr};                 // sparse exchange: (id, label) of owned changes, t-1 / t
+  int32_t* slp_l = nullptr;                          // SLP candidates [nl * slp_k] (labels, counts)
+  int32_t* slp_c = nullptr;
+  int32_t slp_k = 0, slp_cap = 0;                    // K of the last SLP run, allocated K
+  bool slp_valid = false;
   unsigned* chg_n = nullptr;                         // [2] their counts
   unsigned* push_nbig = nullptr;
   glp::Sched* d_sched = nullptr;

@@ -36,8 +36,7 @@ def test_struct_layout_matches_header():
     # the ctypes mirror against the compiled header's sizeof (glp_struct_sizes)
     mine = [ctypes.sizeof(t) for t in (glp.glp_csr, glp.glp_dist, glp.glp_params, glp.glp_run_info,
                                         glp.glp_iter_stat, glp.glp_kernel_stat)]
-    assert mine == glp.glp_struct_sizes()
-    assert ctypes.sizeof(glp.glp_params) == 64  # glp_params.struct_size is checked by glp_run
+    assert mine == glp.glp_struct_sizes()  # (glp_params.struct_size is also checked by glp_run)
 
 
 def test_version_and_partition_host_only():
