@@ -60,6 +60,8 @@ HOST_ARCS = {"rmat24_hostarcs"}
 # §8(f)3 weighted LP: RMAT-24 with symmetric integer arc weights in [1, 8]
 WORKLOADS["rmat24_weighted"] = (dict(kind="rmat", scale=24, edge_factor=16, seed=1), "classic", 20, 0.0)
 WEIGHTED = {"rmat24_weighted"}
+# §8(f)3 SLP: 5 candidate labels, 20 iterations [P:270]
+WORKLOADS["rmat24_slp"] = (dict(kind="rmat", scale=24, edge_factor=16, seed=1), "slp", 20, 0.0)
 
 
 def host_link_gbs(dev) -> float:
@@ -160,12 +162,18 @@ def cpu_reference(csr_cpu, variant, seeds, gamma, iters_per_sample, reps, warmup
     `iters_per_sample` LP iterations from PickLabel."""
     import oracle
     threads = os.cpu_count() or 1
-    vid = {"classic": oracle.CLASSIC, "seeded": oracle.SEEDED, "llp": oracle.LLP}[variant]
+    vid = {"classic": oracle.CLASSIC, "seeded": oracle.SEEDED, "llp": oracle.LLP, "slp": None}[variant]
     times = []
     for r in range(warmup + reps):
         t0 = time.perf_counter()
         sd = None if seeds is None else seeds.cpu().numpy()
-        if weights is not None:
+        if variant == "slp":
+            oracle.run_slp(csr_cpu, K=5, r=0.0, max_iters=iters_per_sample, threads=threads)
+
+            class _R:
+                iterations = iters_per_sample
+            res = _R()
+        elif weights is not None:
             res = oracle.run_weighted(csr_cpu, weights.cpu().numpy().astype("uint32"), vid, iters_per_sample,
                                       seeds=sd, threads=threads)
         else:
@@ -465,8 +473,8 @@ def bench_gpu(args):
                                "sample": f"{args.workload}: first {its} LP iteration(s) from PickLabel, "
                                          f"oracle/glp_oracle.c OpenMP over {cores} threads, {sec:.1f} s "
                                          "(the oracle scans every arc each iteration)",
-                               "sequential": cpu_sequential(csr_cpu, variant, seeds, gamma) if wts is None
-                               else None}
+                               "sequential": cpu_sequential(csr_cpu, variant, seeds, gamma)
+                               if wts is None and variant != "slp" else None}
     if rank == 0:
         print(json.dumps(out), flush=True)
     g.close()
