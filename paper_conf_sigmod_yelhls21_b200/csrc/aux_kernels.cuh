@@ -76,9 +76,15 @@ constexpr int kPushBig = 8192;
 __device__ __forceinline__ void mark(uint8_t* flag, int32_t x) {
   if (!GLP_PUSH_CHECK || !flag[x]) flag[x] = 1;
 }
+// ctl (device-driven loop): {stopped, dense of t+1}; the push is skipped when
+// the run stopped or t+1 is a full sweep, and marks its flags dirty.
+__device__ __forceinline__ bool push_off(const int* ctl) { return ctl && (ctl[0] || ctl[1]); }
 __global__ void k_push(const int64_t* __restrict__ ioff, const int32_t* __restrict__ ideg,
                        const int32_t* __restrict__ col2, const int2* __restrict__ so, int64_t nl, int64_t vb,
-                       int32_t t, uint8_t* __restrict__ flag, int32_t* __restrict__ big, unsigned* __restrict__ n_big) {
+                       int32_t t, uint8_t* __restrict__ flag, int32_t* __restrict__ big, unsigned* __restrict__ n_big,
+                       const int* __restrict__ ctl = nullptr, int* __restrict__ dirty = nullptr) {
+  if (push_off(ctl)) return;
+  if (dirty && blockIdx.x == 0 && threadIdx.x == 0) *dirty = 1;
   const int lane = threadIdx.x & 31;
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -102,7 +108,9 @@ __global__ void k_push(const int64_t* __restrict__ ioff, const int32_t* __restri
 // the listed long rows: every thread of the grid takes a stride of each row
 __global__ void k_push_big(const int64_t* __restrict__ ioff, const int32_t* __restrict__ ideg,
                            const int32_t* __restrict__ col2, const int32_t* __restrict__ big,
-                           const unsigned* __restrict__ n_big, uint8_t* __restrict__ flag) {
+                           const unsigned* __restrict__ n_big, uint8_t* __restrict__ flag,
+                           const int* __restrict__ ctl = nullptr) {
+  if (push_off(ctl)) return;
   const unsigned nb = *n_big;
   const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   const int64_t nth = (int64_t)gridDim.x * blockDim.x;
@@ -116,7 +124,9 @@ __global__ void k_push_big(const int64_t* __restrict__ ioff, const int32_t* __re
 
 // Sparse iterations: a low-degree chunk is active if any of its vertices is.
 __global__ void k_chunk_flags(const LowChunk* __restrict__ chunks, int32_t n_chunks, int64_t low_base,
-                              const uint8_t* __restrict__ flag, int64_t vb, uint8_t* __restrict__ cflag) {
+                              const uint8_t* __restrict__ flag, int64_t vb, uint8_t* __restrict__ cflag,
+                              const int* __restrict__ ctl = nullptr) {
+  if (push_off(ctl)) return;
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n_chunks; c += (int64_t)gridDim.x * blockDim.x) {
     const LowChunk ch = chunks[c];
     const int nv = __popc(ch.segmask);
@@ -196,6 +206,61 @@ __global__ void k_vl(const int32_t* __restrict__ L, const int32_t* __restrict__ 
     const int32_t l = L[q];
     LV[q] = make_int2(l, l >= 0 ? V[l] : 0);
   }
+}
+
+// device-driven loop: clear a mark buffer after the iteration that read it,
+// if a push wrote it
+__global__ void k_clear_flags(uint8_t* __restrict__ flag, int64_t n, int* __restrict__ dirty) {
+  if (!*dirty) return;
+  uint4* f4 = (uint4*)flag;
+  const int64_t n16 = n / 16;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n16; i += (int64_t)gridDim.x * blockDim.x)
+    f4[i] = make_uint4(0u, 0u, 0u, 0u);
+  for (int64_t i = n16 * 16 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    flag[i] = 0;
+}
+__global__ void k_reset_dirty(int* dirty) { *dirty = 0; }
+
+// One iteration's record of the device-driven loop (glp_iter_stat fields).
+struct IterRec {
+  unsigned long long changed, d2, chdeg, arcs, verts, cms0, cms1, cms2;
+  int dense, pad;
+};
+// End of iteration t (device-driven loop; one thread): totals of the per-kernel
+// counters -> rec[t-1]; the stop rule R8 (fixed point / two-cycle); the
+// frontier decision for t+1 (dense when the changed vertices touch more than
+// nnz / dense_div arcs); the counters and tickets are zeroed for t+1, and the
+// stop flag is mirrored to mapped host memory for the host's look-ahead.
+// ctl = {stopped, dense, reason, iters}.
+__global__ void k_decide(Counters* __restrict__ cnt, int ncnt, unsigned long long* __restrict__ sched, int nsched,
+                         int* __restrict__ ctl, IterRec* __restrict__ rec, volatile int* __restrict__ h_stop, int t,
+                         long long nnz_global, int dense_div, int stop_2c, int use_frontier, int never_stop) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  if (ctl[0]) return;
+  Counters tot;
+  memset(&tot, 0, sizeof(tot));
+  for (int b = 0; b < ncnt; ++b) {
+    tot.changed += cnt[b].changed; tot.d2 += cnt[b].d2; tot.chdeg += cnt[b].chdeg;
+    tot.arcs += cnt[b].arcs; tot.verts += cnt[b].verts;
+    tot.pad0 += cnt[b].pad0; tot.pad[0] += cnt[b].pad[0]; tot.pad[1] += cnt[b].pad[1];
+  }
+  IterRec r;
+  r.changed = tot.changed; r.d2 = tot.d2; r.chdeg = tot.chdeg; r.arcs = tot.arcs; r.verts = tot.verts;
+  r.cms0 = tot.pad0; r.cms1 = tot.pad[0]; r.cms2 = tot.pad[1];
+  r.dense = ctl[1]; r.pad = 0;
+  rec[t - 1] = r;
+  int reason = 0;
+  if (!never_stop) {
+    if (tot.changed == 0) reason = 1;
+    else if (stop_2c && t >= 2 && tot.d2 == 0) reason = 2;
+  }
+  ctl[3] = t;
+  if (reason) { ctl[0] = 1; ctl[2] = reason; }
+  ctl[1] = (!use_frontier || (double)tot.chdeg * (double)dense_div > (double)nnz_global) ? 1 : 0;
+  for (int b = 0; b < ncnt; ++b) memset(&cnt[b], 0, sizeof(Counters));
+  for (int i = 0; i < nsched; ++i) sched[i] = 0ull;
+  *h_stop = ctl[0];
+  __threadfence_system();
 }
 
 // LLP at t = 0: L_0 is a permutation, so V[L_0[q]] = 1 for every q.

@@ -189,6 +189,7 @@ void free_graph(glp_graph* g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   g->allocs.clear();
   if (g->h_cnt) cudaFreeHost(g->h_cnt);
+  if (g->h_stop) cudaFreeHost((void*)g->h_stop);
   if (g->col2_host) cudaFreeHost(g->col2_host);
   if (g->registered) cudaHostUnregister(g->registered);
   if (g->ev_a) cudaEventDestroy(g->ev_a);
@@ -638,6 +639,13 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       g->use_vl = !(novl && novl[0] == '1');
       const char* nomono = getenv("GLP_NO_MONO");
       g->use_mono = !(nomono && nomono[0] == '1');
+      // device-driven loop: opt-in (GLP_DEVICE_LOOP=1).  A/B, median ms/run:
+      // karate 0.47 -> 0.59, SBM 5.38 -> 5.44, R24 18.19 -> 17.98, TaoBao
+      // 109.1 -> 108.5, R24 LLP 177.7 -> 178.1: the kernels it must enqueue
+      // unconditionally (push, mark clearing, decide) cost about what the
+      // host round trip saved
+      const char* dl = getenv("GLP_DEVICE_LOOP");
+      g->dev_loop = dl && dl[0] == '1';
       const char* l2w = getenv("GLP_L2_WINDOW");
       if (l2w && l2w[0] == '1') {
         // persisting L2 set-aside up to the device maximum
@@ -745,12 +753,13 @@ void timed(glp_graph* g, bool prof, int kid, std::vector<Pending>& pend, size_t&
 
 // ---------------------------------------------------------------- run
 // frontier push of the vertices changed at t (k_push + its long-row pass)
-void push(glp_graph* g, int32_t t, uint8_t* flag) {
+void push(glp_graph* g, int32_t t, uint8_t* flag, const int* ctl = nullptr, int* dirty = nullptr) {
   cudaStream_t s = g->stream;
   CK(cudaMemsetAsync(g->push_nbig, 0, sizeof(unsigned), s));
   k_push<<<g->grid_aux, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->so, g->nl, g->vb, t, flag, g->push_big,
-                                     g->push_nbig);
-  if (g->max_deg >= kPushBig) k_push_big<<<g->sms * 4, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->push_big, g->push_nbig, flag);
+                                     g->push_nbig, ctl, dirty);
+  if (g->max_deg >= kPushBig)
+    k_push_big<<<g->sms * 4, 256, 0, s>>>(g->ioff, g->ideg, g->col2, g->push_big, g->push_nbig, flag, ctl);
   CK(cudaGetLastError());
 }
 
@@ -1055,6 +1064,160 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   int reason = GLP_STOP_MAX_ITERS;
   int64_t changed_last = 0, arcs_total = 0;
   int64_t launches = 0;  // kernels of this run (excluding memsets/copies)
+
+  // ---- device-driven loop (one rank, not profiled): the stop rule and the
+  // frontier decision run on the device (k_decide), so the host never waits
+  // for an iteration to finish before enqueueing the next; it looks two
+  // iterations back through a mapped stop flag, and iterations enqueued past
+  // the stop return at once (every kernel checks ctl).  Opt-in
+  // (GLP_DEVICE_LOOP=1); the host-driven loop below is the default.
+  if (!prof && !g->comm && g->dev_loop && max_iters > 0) {
+    if (g->rec_cap < max_iters) {
+      g->d_rec = dalloc<IterRec>(g, max_iters);
+      g->rec_cap = max_iters;
+    }
+    if (!g->d_ctl) {
+      g->d_ctl = dalloc<int>(g, 8);  // {stopped, dense, reason, iters}, dirty[2]
+      CK(cudaHostAlloc((void**)&g->h_stop, sizeof(int), cudaHostAllocMapped));
+      CK(cudaHostGetDevicePointer((void**)&g->d_hstop, (void*)g->h_stop, 0));
+    }
+    *g->h_stop = 0;
+    const int ctl0[8] = {0, dense ? 1 : 0, 0, 0, use_frontier ? 1 : 0, 0, 0, 0};  // dirty[fb = 0]: seeded push
+    g->h_ctl_init[0] = ctl0[0];
+    for (int i = 0; i < 8; ++i) g->h_ctl_init[i] = ctl0[i];
+    CK(cudaMemcpyAsync(g->d_ctl, g->h_ctl_init, 8 * sizeof(int), cudaMemcpyHostToDevice, s));
+    CK(cudaMemsetAsync(g->d_cnt, 0, kNumCounters * sizeof(Counters), s));
+    CK(cudaMemsetAsync(g->d_sched, 0, sizeof(Sched), s));
+    int* dirty = g->d_ctl + 4;
+    std::vector<cudaEvent_t> e0v, e1v;
+    std::vector<int64_t> lv;  // launches per enqueued iteration
+    int32_t enq = 0;
+    for (int32_t t = 1; t <= max_iters; ++t) {
+      if (t >= 3) {  // look-ahead of two iterations
+        CK(cudaEventSynchronize(e1v[t - 3]));
+        if (*(volatile int*)g->h_stop) break;
+      }
+      int64_t lt = 0;
+      cudaEvent_t e0 = pool_event(g, used), e1 = pool_event(g, used);
+      e0v.push_back(e0);
+      e1v.push_back(e1);
+      CK(cudaEventRecord(e0, s));
+      g->cur_t = t;
+      if (g->n_giant) {
+        if (++g->gepoch >= (1ull << kGEpochBits)) {
+          CK(cudaMemsetAsync(g->gtab, 0, g->gtab_slots * sizeof(unsigned long long), s));
+          g->gepoch = 1;
+        }
+      }
+      MflArgs a;
+      memset(&a, 0, sizeof(a));
+      a.col = g->col2; a.R = g->L[rb]; a.W = g->L[1 - rb]; a.so = g->so;
+      a.V = g->V; a.is_seed = g->is_seed; a.flag = g->flag[fb];
+      a.vb = g->vb; a.gamma = p.gamma; a.t = t; a.dense = 1;
+      a.ctl = g->d_ctl;
+      a.pred_cap = p.debug_pred_cap > 0 ? (unsigned)p.debug_pred_cap : 0u;
+      a.v_ones = (variant == GLP_VARIANT_LLP && t == 1) ? 1 : 0;
+      a.LV = (variant == GLP_VARIANT_LLP && g->use_vl) ? g->LV : nullptr;
+      a.mono_kernel = (t == 1 && variant != GLP_VARIANT_SEEDED && g->use_mono) ? 1 : 0;
+      a.cms = p.tail_cms ? 1 : 0;
+      a.cms_ht = p.cms_ht_slots > 0 ? (unsigned)p.cms_ht_slots : 0u;
+      a.cms_depth = p.cms_depth > 0 ? (unsigned)p.cms_depth : 4u;
+      if (g->weighted) {
+        lt += variant == GLP_VARIANT_SEEDED ? launch_wt<V_SEEDED>(g, a, false, pend, used)
+                                            : launch_wt<V_CLASSIC>(g, a, false, pend, used);
+      } else switch (variant) {
+        case GLP_VARIANT_CLASSIC: lt += launch_mfl<V_CLASSIC>(g, a, false, pend, used); break;
+        case GLP_VARIANT_SEEDED: lt += launch_mfl<V_SEEDED>(g, a, false, pend, used); break;
+        case GLP_VARIANT_SLP: lt += launch_mfl<V_CLASSIC>(g, a, false, pend, used); break;
+        default: lt += launch_mfl<V_LLP>(g, a, false, pend, used); break;
+      }
+      if (slp && g->nl) {
+        k_slp_listen_speak<<<ga, 256, 0, s>>>(g->slp_l, g->slp_c, g->L[1 - rb], g->ideg, g->nl, g->vb, slp_k,
+                                              p.slp_threshold * (double)(t + 1));
+        lt += 1;
+      }
+      k_decide<<<1, 32, 0, s>>>(g->d_cnt, kNumCounters, (unsigned long long*)g->d_sched,
+                                (int)(sizeof(Sched) / sizeof(unsigned long long)), g->d_ctl, g->d_rec, g->d_hstop,
+                                t, (long long)g->nnz_global, p.dense_divisor, p.stop_on_2cycle, use_frontier ? 1 : 0,
+                                slp ? 1 : 0);
+      CK(cudaGetLastError());
+      lt += 1;
+      CK(cudaEventRecord(e1, s));
+      const int nf = 1 - fb;
+      if (use_frontier && t < max_iters) {
+        // the marks of t+1 (skipped on the device when t+1 is dense or the
+        // run stopped); the marks just read are cleared if a push wrote them
+        CK(cudaMemsetAsync(dirty + nf, 0, sizeof(int), s));
+        push(g, t, g->flag[nf], g->d_ctl, dirty + nf);
+        lt += g->max_deg >= kPushBig ? 2 : 1;
+        if (g->n_chunks) {
+          k_chunk_flags<<<ga, 256, 0, s>>>(g->chunks, g->n_chunks, g->low_base, g->flag[nf], g->vb, g->cflag, g->d_ctl);
+          lt += 1;
+        }
+      }
+      if (use_frontier) {
+        k_clear_flags<<<ga, 256, 0, s>>>(g->flag[fb], g->npad, dirty + fb);
+        k_reset_dirty<<<1, 1, 0, s>>>(dirty + fb);
+        lt += 2;
+      }
+      if (t < max_iters && variant == GLP_VARIANT_LLP) {
+        CK(cudaMemsetAsync(g->V, 0, std::max<int64_t>(g->n, 1) * sizeof(int32_t), s));
+        k_hist<<<ga, 256, 0, s>>>(g->L[1 - rb], g->n, g->V);
+        if (g->use_vl) k_vl<<<ga, 256, 0, s>>>(g->L[1 - rb], g->V, g->n, g->LV);
+        lt += g->use_vl ? 2 : 1;
+      }
+      CK(cudaGetLastError());
+      lv.push_back(lt);
+      g->pb = (g->pb + 1) % 3;
+      rb = 1 - rb;
+      fb = nf;
+      enq = t;
+    }
+    CK(cudaStreamSynchronize(s));
+    int ctl_h[8];
+    CK(cudaMemcpy(ctl_h, g->d_ctl, sizeof(ctl_h), cudaMemcpyDeviceToHost));
+    iters = ctl_h[3];
+    reason = ctl_h[0] ? ctl_h[2] : GLP_STOP_MAX_ITERS;
+    std::vector<IterRec> rec(std::max(iters, 1));
+    if (iters > 0) CK(cudaMemcpy(rec.data(), g->d_rec, iters * sizeof(IterRec), cudaMemcpyDeviceToHost));
+    for (int32_t t = 1; t <= iters; ++t) {
+      const IterRec& r = rec[t - 1];
+      glp_iter_stat st;
+      memset(&st, 0, sizeof(st));
+      st.changed = (int64_t)r.changed; st.d2 = (int64_t)r.d2;
+      st.active_vertices = (int64_t)r.verts; st.active_arcs = (int64_t)r.arcs;
+      st.dense = r.dense;
+      st.cms_rows = (int64_t)r.cms0; st.cms_rescans = (int64_t)r.cms1; st.cms_fallbacks = (int64_t)r.cms2;
+      float ms = 0;
+      CK(cudaEventElapsedTime(&ms, e0v[t - 1], e1v[t - 1]));
+      st.ms = ms;
+      g->iter_stats.push_back(st);
+      changed_last = st.changed;
+      arcs_total += st.active_arcs;
+      launches += lv[t - 1];
+    }
+    (void)enq;
+    // stale flags of a buffer a skipped iteration would have cleared
+    g->flag_clean[0] = g->flag_clean[1] = false;
+    cudaEvent_t ev_run1 = pool_event(g, used);
+    CK(cudaEventRecord(ev_run1, s));
+    CK(cudaStreamSynchronize(s));
+    float run_ms = 0;
+    CK(cudaEventElapsedTime(&run_ms, ev_run0, ev_run1));
+    g->cur = iters & 1;
+    g->has_run = true;
+    g->slp_valid = slp;
+    if (info) {
+      info->iterations = iters;
+      info->stop_reason = reason;
+      info->changed_last = changed_last;
+      info->arcs_processed = arcs_total;
+      info->elapsed_ms = run_ms;
+      info->kernel_launches = launches + g->init_launches;
+    }
+    return;
+  }
+
   for (int32_t t = 1; t <= max_iters; ++t) {
     cudaEvent_t e0 = pool_event(g, used), e1 = pool_event(g, used);
     CK(cudaEventRecord(e0, s));

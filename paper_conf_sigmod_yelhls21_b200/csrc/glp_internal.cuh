@@ -23,7 +23,8 @@
 
 namespace glp {
 
-struct Comm;  // comm.cuh: the exchange of the 1-D partition (NCCL or in-process)
+struct Comm;     // comm.cuh: the exchange of the 1-D partition (NCCL or in-process)
+struct IterRec;  // aux_kernels.cuh: one iteration's record of the device-driven loop
 
 // Degree bin of the packed-warp kernel (PAPER §4.2): deg <= 32.
 constexpr int kLowMax = 32;
@@ -196,7 +197,8 @@ struct MflArgs {
   int64_t vb;                           // global id of local row 0
   double gamma;
   int32_t t;                            // iteration number (1-based)
-  int32_t dense;                        // 1: process every listed vertex
+  int32_t dense;                        // 1: process every listed vertex (host-driven loop)
+  const int* __restrict__ ctl;          // device-driven loop: {stopped, dense} (glp.cu k_decide), or null
   const int2* __restrict__ LV;          // LLP: (L_{t-1}[u], V[L_{t-1}[u]]) interleaved, or null
   int32_t v_ones;                       // LLP: V[l] == 1 for every l (L_{t-1} is PickLabel's permutation)
   int32_t lv_labels;                    // LLP sharded: neighbour labels are read from LV (R holds owned rows only)
@@ -322,6 +324,13 @@ struct glp_graph {
   bool concurrent = true;
   bool use_vl = true;  // LLP gathers (label, V[label]) pairs from LV (GLP_NO_VL=1 disables)
   bool use_mono = true;
+  bool dev_loop = false;      // device-driven iteration loop (GLP_DEVICE_LOOP=1)
+  int* d_ctl = nullptr;       // {stopped, dense, reason, iters, dirty[2]}
+  volatile int* h_stop = nullptr;  // mapped host mirror of the stop flag
+  int* d_hstop = nullptr;
+  int h_ctl_init[8] = {0};
+  glp::IterRec* d_rec = nullptr;
+  int32_t rec_cap = 0;
   bool l2_window = false;     // A/B: persisting L2 window on the gathered array (GLP_L2_WINDOW=1)
   size_t l2_window_max = 0;  // t = 1 sorted-row candidates in mfl_mono (GLP_NO_MONO=1: in the W kernel)
   int* col_bad = nullptr;  // create: col_idx range check flag (side stream)

@@ -150,6 +150,16 @@ __device__ __forceinline__ int gather_lv(const MflArgs& a, int u, bool use_v, in
   return ld_label(a.R + u);
 }
 
+// Device-driven iteration loop: a.ctl = {stopped, dense} written by k_decide
+// at the end of the previous iteration (null: host-driven, a.dense).  An
+// iteration enqueued after the stop rule fired does nothing.
+#define GLP_CTL_PROLOGUE(a)                 \
+  int dense_ = (a).dense;                   \
+  if ((a).ctl) {                            \
+    if ((a).ctl[0]) return;                 \
+    dense_ = (a).ctl[1];                    \
+  }
+
 // LLP score val = k - gamma * (v - k) [P:119], double, no contraction (R11).
 __device__ __forceinline__ double llp_score(unsigned k, int v, double gamma) {
   double kd = (double)k;
@@ -571,6 +581,7 @@ __device__ __forceinline__ void update_vertex_pre(const MflArgs& a, int v, int d
 
 template <int VAR>
 __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
+  GLP_CTL_PROLOGUE(a)
   const int lane = threadIdx.x & 31;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -584,7 +595,7 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
     bool act = cl < a.n_chunks;
     if (act) {
       mine = a.chunks[cl];
-      if (!a.dense) act = a.cflag[cl] != 0;
+      if (!dense_) act = a.cflag[cl] != 0;
     }
     unsigned todo = __ballot_sync(kFull, act);
     if (!todo) continue;
@@ -855,6 +866,7 @@ template <int VAR>
 #define GLP_W_MINB 4
 #endif
 __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
+  GLP_CTL_PROLOGUE(a)
   extern __shared__ __align__(16) unsigned long long wtabs[];  // [kWBlock / 32][kWSlots] (dynamic)
   __shared__ int s_over[kWBlock / 32];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -874,7 +886,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       const bool cand = mono_cand<VAR>(raw, a.pred_cap, mine.d);
       mpred = pred_est<VAR>(raw, a.pred_prev[il], a.pred_cap) | (cand ? kMonoTried : 0u);
       ok = row_class(mpred & kPredMask, mine.d, cand, a.mono_kernel) == CLS_W;
-      if (ok && !a.dense && !a.flag[a.vb + mine.v]) {
+      if (ok && !dense_ && !a.flag[a.vb + mine.v]) {
         ok = false;
         a.pred_next[il] = raw;  // inactive: carry the prediction forward
       }
@@ -1046,6 +1058,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
 constexpr int kMonoBlock = 256;
 template <int VAR>
 __global__ void __launch_bounds__(kMonoBlock, GLP_MONO_MINB) mfl_mono(MflArgs a) {
+  GLP_CTL_PROLOGUE(a)
   const int lane = threadIdx.x & 31;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -1060,7 +1073,7 @@ __global__ void __launch_bounds__(kMonoBlock, GLP_MONO_MINB) mfl_mono(MflArgs a)
       const unsigned raw = a.pred[il];
       ok = mono_cand<VAR>(raw, a.pred_cap, mine.d) &&
            row_class(raw & kPredMask, mine.d, true, true) == CLS_MONO;
-      if (ok && !a.dense && !a.flag[a.vb + mine.v]) {
+      if (ok && !dense_ && !a.flag[a.vb + mine.v]) {
         ok = false;
         a.pred_next[il] = raw;
       }
@@ -1426,6 +1439,7 @@ template <int VAR, int BLOCK, int SLOTS, bool PART, int UNROLL, int CLS>
 #define GLP_L_MINB 2
 #endif
 __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_block(MflArgs a) {
+  GLP_CTL_PROLOGUE(a)
   extern __shared__ __align__(16) unsigned long long smem_tab[];  // SLOTS
   __shared__ int s_over, s_distinct, s_major, s_scan;
   __shared__ int s_hist[PART ? 256 : 1], s_cur[PART ? 256 : 1];
@@ -1469,7 +1483,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
         cnd = mono_cand<VAR>(raw, a.pred_cap, itk.d);
         if (!a.mode) {
           ok = row_class(pe, itk.d, cnd, a.mono_kernel) == CLS;
-          if (ok && !a.dense && !a.flag[a.vb + itk.v]) {
+          if (ok && !dense_ && !a.flag[a.vb + itk.v]) {
             ok = false;
             a.pred_next[ik] = raw;  // inactive: carry the prediction forward
           }
@@ -1745,6 +1759,7 @@ __device__ __forceinline__ unsigned giant_add(unsigned long long* tab, unsigned 
 constexpr int kGSlots = 8192;  // shared pre-aggregation table (64 KB)
 template <int VAR>
 __global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
+  GLP_CTL_PROLOGUE(a)
   extern __shared__ __align__(16) unsigned long long gsm[];  // kGSlots (GLP_GIANT_SMEM)
   __shared__ int s_k;
   const int lane = threadIdx.x & 31;
@@ -1756,7 +1771,7 @@ __global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
     if (k >= a.n_gsegs) break;
     const GiantSeg sg = a.gsegs[k];
     const BinItem it = a.items[sg.row];
-    if (!a.dense && !a.flag[a.vb + it.v]) continue;  // block-uniform
+    if (!dense_ && !a.flag[a.vb + it.v]) continue;  // block-uniform
     unsigned long long* tab = a.gtab + a.gtab_off[sg.row];
     const unsigned long long tsz = (unsigned long long)(a.gtab_off[sg.row + 1] - a.gtab_off[sg.row]);
     const int end = min(sg.begin + kGiantSeg, it.d);
@@ -1864,10 +1879,11 @@ __global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
 // over all observations is exact, see the header) and updates the vertex.
 template <int VAR>
 __global__ void __launch_bounds__(256) mfl_giant_finish(MflArgs a, const int32_t* __restrict__ seg_first) {
+  GLP_CTL_PROLOGUE(a)
   Tally ty;
   const int i = blockIdx.x;
   const BinItem it = a.items[i];
-  const bool active = a.dense || a.flag[a.vb + it.v];
+  const bool active = dense_ || a.flag[a.vb + it.v];
   if (active) {
     Best<VAR> b;
     for (int k = seg_first[i] + (int)threadIdx.x; k < seg_first[i + 1]; k += 256) b.merge(a.gcand_key[k], a.gcand_lab[k]);

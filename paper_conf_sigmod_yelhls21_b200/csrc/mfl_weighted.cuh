@@ -32,6 +32,7 @@ constexpr int kWtSlots = 8192;
 
 template <int VAR>
 __global__ void __launch_bounds__(kWtBlock) mfl_wt_warp(MflArgs a) {
+  GLP_CTL_PROLOGUE(a)
   extern __shared__ __align__(16) unsigned long long wts_tab[];  // [8][kWtWarpSlots]
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -43,7 +44,7 @@ __global__ void __launch_bounds__(kWtBlock) mfl_wt_warp(MflArgs a) {
     bool ok = v < a.wt_hi;
     if (ok) {
       deg = a.ideg[v];
-      ok = deg >= 1 && deg <= kWtWarpMax && (a.dense || a.flag[a.vb + v]);
+      ok = deg >= 1 && deg <= kWtWarpMax && (dense_ || a.flag[a.vb + v]);
     }
     unsigned todo = __ballot_sync(kFull, ok);
     bool rdone = false;
@@ -89,6 +90,7 @@ __global__ void __launch_bounds__(kWtBlock) mfl_wt_warp(MflArgs a) {
 
 template <int VAR>
 __global__ void __launch_bounds__(kWtBlock) mfl_wt_block(MflArgs a) {
+  GLP_CTL_PROLOGUE(a)
   extern __shared__ __align__(16) unsigned long long wtb_tab[];  // kWtSlots
   __shared__ int s_k, s_over, s_distinct;
   Tally ty;
@@ -99,7 +101,7 @@ __global__ void __launch_bounds__(kWtBlock) mfl_wt_block(MflArgs a) {
     if (k >= a.n_items) break;
     const BinItem it = a.items[k];
     const unsigned raw = a.pred[k];
-    if (!a.dense && !a.flag[a.vb + it.v]) {
+    if (!dense_ && !a.flag[a.vb + it.v]) {
       if (threadIdx.x == 0) a.pred_next[k] = raw;  // inactive: carry the count forward
       __syncthreads();  // s_k is rewritten by the next ticket
       continue;

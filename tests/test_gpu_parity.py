@@ -339,7 +339,8 @@ def test_nccl_exchange_path_single_rank():
     assert info.iterations == ref.iterations and (lab == ref.labels).all()
 
 
-@pytest.mark.parametrize("env", [{"GLP_NO_VL": "1"}, {"GLP_SERIAL": "1"}])
+@pytest.mark.parametrize("env", [{"GLP_NO_VL": "1"}, {"GLP_SERIAL": "1"}, {"GLP_DEVICE_LOOP": "1"},
+                                 {"GLP_NO_MONO": "1"}])
 def test_alternate_execution_modes(env, monkeypatch):
     """The A/B switches read at graph create (LLP without the interleaved
     label/V array, serialised class kernels) give the same exact runs."""
@@ -349,6 +350,9 @@ def test_alternate_execution_modes(env, monkeypatch):
     assert_same_run(csr, 0, 20)
     for gamma in (1.0, 0.37):
         assert_same_run(csr, 2, 8, gamma=gamma)
+    tb, seeds = graphs.taobao(users=40_000, items=10_000, pairs=200_000, rings=40, seed=5)
+    assert_same_run(tb, 1, 30, seeds=seeds.numpy())  # sparse frontier iterations
+    assert_same_run(graphs.karate(), 0, 20)
 
 
 def _label_part(lab, nparts):
