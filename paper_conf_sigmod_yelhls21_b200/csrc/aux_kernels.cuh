@@ -139,15 +139,21 @@ __global__ void k_chunk_flags(const LowChunk* __restrict__ chunks, int32_t n_chu
 // Build the bin-major arc copy: row v of the caller's CSR (local original id)
 // -> col2[ioff[pos[vb + v] - vb] ...], each arc renamed to its internal id.
 // Arc order within a row is kept.
+// Rows [v0, v1) only (the create pipelines the relayout with the arcs' host
+// copy chunk by chunk); an out-of-range column (rejected after the relayout
+// by the validation flag) is written as -1 instead of indexing pos with it.
 __global__ void k_relayout(const int64_t* __restrict__ off, const int32_t* __restrict__ col,
-                           const int64_t* __restrict__ ioff, const int32_t* __restrict__ pos, int64_t nl, int64_t vb,
-                           int32_t* __restrict__ col2) {
+                           const int64_t* __restrict__ ioff, const int32_t* __restrict__ pos, int64_t v0, int64_t v1,
+                           int64_t vb, int64_t n, int32_t* __restrict__ col2) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t v = gw; v < nl; v += nw) {
+  for (int64_t v = v0 + gw; v < v1; v += nw) {
     const int64_t s = off[v], d = off[v + 1] - s, o = ioff[pos[vb + v] - vb];
-    for (int64_t j = lane; j < d; j += 32) col2[o + j] = pos[col[s + j]];
+    for (int64_t j = lane; j < d; j += 32) {
+      const int32_t u = col[s + j];
+      col2[o + j] = (u >= 0 && (int64_t)u < n) ? pos[u] : -1;
+    }
   }
 }
 

@@ -17,6 +17,7 @@
 
 #include <algorithm>
 #include <array>
+#include <chrono>
 #include <mutex>
 #include <cmath>
 #include <cstdio>
@@ -36,6 +37,26 @@ using namespace glp;
 namespace {
 
 thread_local std::string g_last_error = "";
+
+// GLP_TRACE_CREATE=1: host timestamps of the create phases on stderr
+struct CreateTrace {
+  bool on = false;
+  std::chrono::steady_clock::time_point t0;
+  CreateTrace() {
+    const char* e = getenv("GLP_TRACE_CREATE");
+    on = e && e[0] == '1';
+    t0 = std::chrono::steady_clock::now();
+  }
+  void mark(const char* what) const {
+    if (on)
+      fprintf(stderr, "[glp create] %-28s %8.2f ms\n", what,
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+  }
+};
+thread_local CreateTrace* g_trace = nullptr;
+void trace(const char* what) {
+  if (g_trace) g_trace->mark(what);
+}
 
 [[noreturn]] void fail(glp_status st, const std::string& m) { throw Err{st, m}; }
 
@@ -196,6 +217,7 @@ void free_graph(glp_graph* g) {
   if (g->ev_b) cudaEventDestroy(g->ev_b);
   for (auto& e : g->ev_pool) cudaEventDestroy(e);
   for (auto& e : g->xev) if (e) cudaEventDestroy(e);
+  for (auto& e : g->arc_chunk_ev) cudaEventDestroy(e);
   delete g->comm;
   g->comm = nullptr;
   if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
@@ -257,6 +279,7 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
   LayoutStats st;
   CK(cudaMemcpyAsync(&st, dst, sizeof(st), cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
+  trace("degree stats");
   for (int b = 0; b < NBINS; ++b) {
     g->bin_verts[b] = (int64_t)st.verts[b];
     g->bin_arcs[b] = (int64_t)st.arcs[b];
@@ -328,6 +351,7 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     CK(cudaMemcpyAsync(row_i.data(), g->rows, n_rows * sizeof(BinItem), cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(&padded_total, pstart + n_rows, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
+    trace("row order + placement");
   }
   g->nnz2 = rows_base + padded_total;
   if (g->nnz2 >= ((int64_t)1 << 48)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
@@ -391,14 +415,8 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     g->comm->allgather(g, g->pos, sizeof(int32_t));
     g->comm->allgather(g, g->orig, sizeof(int32_t));
   }
-  // ---- the arcs themselves (copied and checked on the side stream)
-  CK(cudaStreamWaitEvent(s, g->xev[1], 0));
-  {
-    int bad = 0;
-    CK(cudaMemcpyAsync(&bad, g->col_bad, sizeof(int), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    if (bad & 8) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
-  }
+  // ---- the arcs themselves (copied and checked on the side stream, in
+  // chunks of rows: each chunk is relayouted as soon as its copy landed)
   if (g->host_arcs) {
     // hybrid mode [P:103]: the bin-major arc array lives in pinned, mapped
     // host memory; the MFL kernels stream it over the host link (labels,
@@ -419,13 +437,30 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), s));  // padding = -1
   }
   if (nl > 0 && g->nnz > 0) {
-    k_relayout<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, g->pos, nl, g->vb, g->col2);
-    CK(cudaGetLastError());
+    for (size_t c = 0; c + 1 < g->arc_chunks.size(); ++c) {
+      if (c < g->arc_chunk_ev.size()) CK(cudaStreamWaitEvent(s, g->arc_chunk_ev[c], 0));
+      else CK(cudaStreamWaitEvent(s, g->xev[1], 0));
+      k_relayout<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, g->pos, g->arc_chunks[c], g->arc_chunks[c + 1], g->vb,
+                                    g->n, g->col2);
+      CK(cudaGetLastError());
+    }
   }
-  CK(cudaStreamSynchronize(s));
+  CK(cudaStreamWaitEvent(s, g->xev[1], 0));
+  {
+    int bad = 0;
+    CK(cudaMemcpyAsync(&bad, g->col_bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    trace("arcs copied + checked + relayout");
+    if (bad & 8) fail(GLP_ERR_INVALID_GRAPH, "col_idx entry outside [0, n_global)");
+  }
 }
 
 void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm, glp_graph** out) {
+  CreateTrace tr;
+  g_trace = &tr;
+  struct Reset {
+    ~Reset() { g_trace = nullptr; }
+  } reset_trace;
   if (!out) fail(GLP_ERR_INVALID_ARGUMENT, "out is NULL");
   *out = nullptr;
   if (!csr) fail(GLP_ERR_INVALID_ARGUMENT, "csr is NULL");
@@ -544,10 +579,35 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaMemsetAsync(dbad, 0, 2 * sizeof(int), g->stream));
     CK(cudaEventRecord(g->xev[0], g->stream));
     CK(cudaStreamWaitEvent(g->xs[0], g->xev[0], 0));
-    if (!csr->on_device && !g->host_arcs && g->nnz)
-      CK(cudaMemcpyAsync((void*)col_d, csr->col_idx, g->nnz * sizeof(int32_t), cudaMemcpyHostToDevice, g->xs[0]));
-    if (p.validate && g->nnz) k_validate_col<<<g->sms * 4, 256, 0, g->xs[0]>>>(col_d, g->nnz, g->n, dbad + 1);
-    CK(cudaGetLastError());
+    // row chunks of ~equal arcs (host offsets): copy + check chunk c, then
+    // record its event; the relayout of chunk c waits for that event only
+    g->arc_chunks.assign({0, g->nl});
+    if (!csr->on_device && !g->host_arcs && g->nnz >= ((int64_t)1 << 26)) {
+      const int K = 8;
+      g->arc_chunks.clear();
+      g->arc_chunks.push_back(0);
+      for (int c = 1; c < K; ++c) {
+        const int64_t target = g->nnz * c / K;
+        const int64_t r = std::upper_bound(csr->row_offsets, csr->row_offsets + g->nl + 1, target) - csr->row_offsets - 1;
+        if (r > g->arc_chunks.back() && r < g->nl) g->arc_chunks.push_back(r);
+      }
+      g->arc_chunks.push_back(g->nl);
+    }
+    for (size_t c = 0; c + 1 < g->arc_chunks.size(); ++c) {
+      const int64_t a0 = csr->on_device || g->host_arcs ? 0 : csr->row_offsets[g->arc_chunks[c]];
+      const int64_t a1 = csr->on_device || g->host_arcs ? g->nnz : csr->row_offsets[g->arc_chunks[c + 1]];
+      if (!csr->on_device && !g->host_arcs && a1 > a0)
+        CK(cudaMemcpyAsync((void*)(col_d + a0), csr->col_idx + a0, (a1 - a0) * sizeof(int32_t),
+                           cudaMemcpyHostToDevice, g->xs[0]));
+      if (p.validate && a1 > a0) k_validate_col<<<g->sms * 4, 256, 0, g->xs[0]>>>(col_d + a0, a1 - a0, g->n, dbad + 1);
+      CK(cudaGetLastError());
+      if (g->arc_chunks.size() > 2) {
+        cudaEvent_t e;
+        CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        g->arc_chunk_ev.push_back(e);
+        CK(cudaEventRecord(e, g->xs[0]));
+      }
+    }
     CK(cudaEventRecord(g->xev[1], g->xs[0]));
     struct TempGuard {
       std::vector<void*>& v;
@@ -566,6 +626,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       int bad = 0;
       CK(cudaMemcpyAsync(&bad, dbad, sizeof(int), cudaMemcpyDeviceToHost, g->stream));
       CK(cudaStreamSynchronize(g->stream));
+      trace("offsets checked");
       if (bad & 3) fail(GLP_ERR_INVALID_GRAPH, "row_offsets[0] must be 0 and row_offsets[last] == nnz_local");
       if (bad & 4) fail(GLP_ERR_INVALID_GRAPH, "row_offsets not non-decreasing");
     }
@@ -700,6 +761,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       g->stage = dalloc<int32_t>(g, (size_t)g->stage_stride * 4 * g->grid_l);
     }
     CK(cudaStreamSynchronize(g->stream));
+    trace("done");
   } catch (const Err& e) {
     if (g->comm) g->comm->abort(e.msg);  // release the other ranks of a local group
     free_graph(g);

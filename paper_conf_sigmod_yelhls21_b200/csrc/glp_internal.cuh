@@ -244,6 +244,8 @@ struct glp_graph {
   const int32_t* col = nullptr;
   bool own_csr = false;
   bool host_arcs = false;       // hybrid mode: col2 in pinned mapped host memory
+  std::vector<int64_t> arc_chunks;         // create: row bounds of the arc copy chunks
+  std::vector<cudaEvent_t> arc_chunk_ev;   // create: chunk c copied + checked
   bool weighted = false;        // weighted LP: w2 holds the arc weights
   uint32_t* w2 = nullptr;       // [nnz2] weights beside col2 (padding 0)
   int32_t n_gt512 = 0;          // prefix of rows with deg > kWtWarpMax
