@@ -20,7 +20,7 @@ scale = {'byte': 1, 'Kbyte': 1e3, 'Mbyte': 1e6, 'Gbyte': 1e9}
 def cls(name):
     if 'mfl_block<' in name:  # template args: <VAR, BLOCK, ...>
         return 'mfl_block_m' if name.split('<')[1].split(',')[1].strip() == '128' else 'mfl_block_l'
-    for k in ('mfl_low', 'mfl_warp', 'mfl_giant'):
+    for k in ('mfl_low', 'mfl_warp', 'mfl_giant', 'mfl_mono', 'mfl_wt_warp', 'mfl_wt_block'):
         if k in name:
             return k
     return None
