@@ -368,11 +368,9 @@ def bench_gpu(args):
         t = torch.tensor([csr.nnz], dtype=torch.int64, device=dev)
         arcs_total = csr.nnz  # every rank generated the full graph
     ms_per_step = total_ms / args.steps
+    # (with several ranks the library all-reduces its per-iteration counters,
+    # so every rank's arcs_processed is already the whole job's)
     scanned = sum(i.arcs_processed for i in infos)
-    if world > 1:
-        t = torch.tensor([scanned], dtype=torch.int64, device=dev)
-        dist.all_reduce(t)  # every rank scans its own rows
-        scanned = int(t.item())
     value = scanned / (total_ms / 1e3) / 1e9
     nnz_iters = arcs_total * sum(i.iterations for i in infos) / (total_ms / 1e3) / 1e9
 
