@@ -32,8 +32,19 @@ if which in ("all", "modes"):
     w = graphs.edge_weights(csr)
     with glp.Graph(csr, weights=w) as G:
         print(G.run("classic", 10))
+    with glp.Graph(hubs, weights=graphs.edge_weights(hubs)) as G:  # partitioned weighted rows
+        print(G.run("classic", 4))
     with glp.Graph(csr.to("cpu"), host_arcs=True) as G:
         print(G.run("classic", 10))
+    with glp.Graph(csr) as G:
+        print(G.run("slp", 8, slp_max_labels=5, slp_threshold=0.1))
+    with glp.Graph(hubs) as G:  # HT + CMS, small HT: sketch, rescans, fallbacks
+        print(G.run("classic", 4, tail_cms=True, cms_ht_slots=256))
+    os.environ["GLP_DEVICE_LOOP"] = "1"
+    with glp.Graph(csr) as G:
+        print(G.run("classic", 20)); print(G.run("seeded", 20, [1, 50, 900]))
+    del os.environ["GLP_DEVICE_LOOP"]
     with LocalGroup(csr, 2) as grp:
         print(grp.run("classic", 10)); print(grp.run("llp", 4, gamma=1.0))
+        print(grp.run("classic", 10, sparse_exchange=1)); print(grp.run("seeded", 10, [1, 50, 900]))
 print("sanitize run ok")
