@@ -377,14 +377,103 @@ struct Cms {
 #ifndef GLP_MATCH_INSERT
 #define GLP_MATCH_INSERT 0
 #endif
+// GLP_LEAN: the label columns left after the hot pass are inserted by a
+// persistent per-lane probe loop (warp_insert_n); GLP_LEAN_PEEK: each probe
+// reads the key before the CAS
+#ifndef GLP_LEAN
+#define GLP_LEAN 1
+#endif
+#ifndef GLP_HOTK
+#define GLP_HOTK 1
+#endif
+#ifndef GLP_LEAN_PEEK
+#define GLP_LEAN_PEEK 0  // A/B (R24 ms/run): 0 17.29, 1 17.27, 2 17.72, 3 17.80; LLP 174.5 / 182.6 / 180.4 / 174.5.  0 never, 1 always, 2 rows predicted to repeat labels, 3 = 2 but not LLP
+#endif
+template <int VAR>
+__device__ __forceinline__ bool peek_pass(unsigned pred, int d) {
+  if (GLP_LEAN_PEEK == 0 || (GLP_LEAN_PEEK == 3 && VAR == V_LLP)) return false;
+  return GLP_LEAN_PEEK == 1 || 2ull * pred <= (unsigned long long)d;
+}
 __device__ __forceinline__ bool hot_pass(unsigned pred, int d) {
   return GLP_HOT_DIV == 0 || (unsigned long long)pred * GLP_HOT_DIV <= (unsigned long long)d;
 }
+// Lean insert of four labels per lane (-1 = none), count 1 each.  The lane's
+// valid labels are first compacted to the front of a 4-entry shift register
+// (five compare-swaps); then a persistent probe loop takes one probe per trip
+// for the register's head: one shared CAS claims a free slot or returns its
+// occupant; on a hit the count is added and the register shifts.  A lane
+// whose label probes does not hold up the other lanes' labels: the warp runs
+// max over lanes of the lane's summed probes, not the sum over label columns
+// of the longest chain.  Returns the lane's number of newly claimed slots.
+template <int VAR>
+__device__ __forceinline__ unsigned lean_insert4(const MflArgs& a, const Table& t, unsigned max_probe, int q0, int q1,
+                                                 int q2, int q3, int v0, int v1, int v2, int v3, Best<VAR>& b,
+                                                 volatile int* overflow, bool use_v, bool obs, const Cms* cms,
+                                                 bool peek) {
+  constexpr bool kV = VAR == V_LLP;  // labels carry V (LLP with a.LV)
+  auto cswap = [&](int& x, int& y, int& vx, int& vy) {
+    const bool s = x < 0;
+    const int tx = x, tv = vx;
+    x = s ? y : x;
+    y = s ? tx : y;
+    if (kV) {
+      vx = s ? vy : vx;
+      vy = s ? tv : vy;
+    }
+  };
+  cswap(q0, q1, v0, v1);
+  cswap(q2, q3, v2, v3);
+  cswap(q0, q2, v0, v2);
+  cswap(q1, q3, v1, v3);
+  cswap(q1, q2, v1, v2);
+  unsigned fresh = 0u, np = 0u;
+  unsigned h = slot_hash((unsigned)q0, t.tsz);
+  const unsigned mask = t.tsz - 1u;
+  while (__any_sync(kFull, q0 >= 0)) {
+    if (q0 >= 0) {
+      // peek (rows predicted to repeat labels): read the key first, so a
+      // repeated label (its slot already claimed) costs a shared load instead
+      // of a CAS serialised with its copies; otherwise one CAS per probe
+      unsigned k = peek ? ld_key(t, h) : kFree;
+      bool claimed = false;
+      if (k == kFree) {
+        k = atomicCAS(t.key + h, kFree, (unsigned)q0);
+        claimed = k == kFree;
+        k = claimed ? (unsigned)q0 : k;
+      }
+      bool next = false;
+      if (k == (unsigned)q0) {
+        const unsigned c = atomicAdd(t.cnt + h, 1u) + 1u;
+        fresh += claimed ? 1u : 0u;
+        if (obs) b.observe(c, (unsigned)q0, a, (kV && use_v) ? v0 : -1);
+        next = true;
+      } else if (++np >= max_probe) {
+        if (cms) {
+          cms->add((unsigned)q0, 1u);
+          next = true;
+        } else {
+          flag_set(overflow);
+          q0 = q1 = q2 = q3 = -1;
+        }
+      } else {
+        h = (h + 1u) & mask;
+      }
+      if (next) {
+        q0 = q1; q1 = q2; q2 = q3; q3 = -1;
+        if (kV) { v0 = v1; v1 = v2; v2 = v3; }
+        h = slot_hash((unsigned)q0, t.tsz);
+        np = 0u;
+      }
+    }
+  }
+  return fresh;
+}
+
 template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
                                                   const int (&labin)[N], Best<VAR>& b, volatile int* overflow,
                                                   const int (&vin)[N], bool use_v, bool hot_ok = true,
-                                                  const Cms* cms = nullptr) {
+                                                  const Cms* cms = nullptr, bool peek = false) {
   // use_v (LLP with a.LV): labels carry their V, so LLP observes at insert
   // like CLASSIC; otherwise LLP scores from the final table (table_scan)
   const bool obs = VAR != V_LLP || use_v;
@@ -400,6 +489,42 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
     candv = (cand < 0 && lab[j] >= 0) ? (use_v ? vin[j] : -1) : candv;
     cand = (cand < 0 && lab[j] >= 0) ? lab[j] : cand;
   }
+#if GLP_HOTK > 1
+  // GLP_HOTK hot labels: the candidates of lanes 0..K-1 (duplicates dropped);
+  // every lane counts its copies of each, K warp sums, then lane c inserts
+  // candidate c with its sum -- the K single-lane inserts in one instruction
+  if (hot_ok && GLP_MATCH_INSERT != 2) {
+    int hk[GLP_HOTK];
+    unsigned mytot = 0u;
+    int mine = -1, minev = -1;
+#pragma unroll
+    for (int c = 0; c < GLP_HOTK; ++c) {
+      hk[c] = __shfl_sync(kFull, cand, c);
+      const int hv = __shfl_sync(kFull, candv, c);
+#pragma unroll
+      for (int e = 0; e < c; ++e) hk[c] = hk[c] == hk[e] ? -1 : hk[c];
+      if (hk[c] >= 0) {  // warp-uniform
+        unsigned hc = 0;
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+          hc += lab[j] == hk[c] ? 1u : 0u;
+          lab[j] = lab[j] == hk[c] ? -1 : lab[j];
+        }
+        const unsigned tot = __reduce_add_sync(kFull, hc);
+        if (lane == c) { mytot = tot; mine = hk[c]; minev = hv; }
+      }
+    }
+    if (mytot) {
+      const unsigned cnt = ht_add(t, (unsigned)mine, mytot, max_probe, &nfresh);
+      if (cnt == 0u) {
+        if (cms) cms->add((unsigned)mine, mytot);
+        else flag_set(overflow);
+      } else if (obs) {
+        b.observe(cnt, (unsigned)mine, a, minev);
+      }
+    }
+  }
+#else
   const int hot = (hot_ok && GLP_MATCH_INSERT != 2) ? __shfl_sync(kFull, cand, 0) : -1;
   const int hotv = __shfl_sync(kFull, candv, 0);
   if (hot >= 0) {  // warp-uniform
@@ -420,6 +545,13 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
       }
     }
   }
+#endif
+#if GLP_LEAN && !GLP_MATCH_INSERT
+#pragma unroll
+  for (int j0 = 0; j0 < N; j0 += 4)
+    nfresh += lean_insert4<VAR>(a, t, max_probe, lab[j0], lab[j0 + 1], lab[j0 + 2], lab[j0 + 3], vin[j0], vin[j0 + 1],
+                                vin[j0 + 2], vin[j0 + 3], b, overflow, use_v, obs, cms, peek);
+#else
   unsigned mc[N];  // occurrences this lane inserts for slot j
 #pragma unroll
   for (int j = 0; j < N; ++j) {
@@ -455,6 +587,7 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
     for (int j = 0; j < N; ++j)
       if (cnt[j]) b.observe(cnt[j], (unsigned)lab[j], a, use_v ? vin[j] : -1);
   }
+#endif
   return nfresh;
 }
 
@@ -935,6 +1068,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       bool major = false;        // a strict-majority label was observed: the rest of the row cannot change the MFL
       int scanned = 0;           // arcs gathered so far
       const bool hot = hot_pass(pred & kPredMask, d);
+      const bool pk = peek_pass<VAR>(pred & kPredMask, d);
       for (int off = 0; off < d && !over && !major; off += kWRound) {
         scanned = min(d, off + kWRound);
         int4 p0, p1;
@@ -981,7 +1115,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
             m8[2] = gather_lv(a, v0.z, use_v, mv8[2]); m8[3] = gather_lv(a, v0.w, use_v, mv8[3]);
             m8[4] = gather_lv(a, v1.x, use_v, mv8[4]); m8[5] = gather_lv(a, v1.y, use_v, mv8[5]);
             m8[6] = gather_lv(a, v1.z, use_v, mv8[6]); m8[7] = gather_lv(a, v1.w, use_v, mv8[7]);
-            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v, hot);
+            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v, hot, nullptr, pk);
           }
         }
         if (wsort) {  // the whole row is this round (d <= kWRound)
@@ -999,11 +1133,11 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           break;
         }
         if (kWRound == 256 && d - off > 128) {  // warp-uniform
-          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v, hot);
+          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v, hot, nullptr, pk);
         } else {
           const int l4[4] = {l[0], l[1], l[2], l[3]};
           const int v4[4] = {lv[0], lv[1], lv[2], lv[3]};
-          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v, hot);
+          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v, hot, nullptr, pk);
         }
         __syncwarp();
         over = warp_flag(&s_over[wid]);
@@ -1166,7 +1300,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
                                             volatile int* overflow, int* distinct, Best<VAR>& b,
                                             volatile int* major, unsigned fparts = 1u, int* scanned = nullptr,
-                                            bool hot = true, const Cms* cms = nullptr) {
+                                            bool hot = true, const Cms* cms = nullptr, bool peek = false) {
   constexpr int STEP = BLOCK * 4 * UNROLL;
   unsigned fresh = 0;
   int base = 0;
@@ -1195,7 +1329,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
     }
-    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot, cms);
+    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot, cms, peek);
     if (GLP_MAJORITY && VAR != V_LLP && major != nullptr && base + STEP < d) {
       // a strict-majority observation ends the row for every warp (they poll the flag)
       const bool m = strict_majority(b, d);
@@ -1564,7 +1698,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : (PART ? tsz : kTabProbe), cur,
                                       (GLP_L_STAGE1 && may_over) ? stageA : nullptr, &s_over, &s_distinct, b,
                                       (may_over && !GLP_L_MAJ) ? nullptr : &s_major, 1u, &s_scan,
-                                      hot_pass(est, d));
+                                      hot_pass(est, d), nullptr, peek_pass<VAR>(est, d));
       __syncthreads();
       over = s_over != 0;
       if (!over && a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
