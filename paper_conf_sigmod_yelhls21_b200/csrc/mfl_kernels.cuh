@@ -386,6 +386,12 @@ struct Cms {
 #ifndef GLP_HOTK
 #define GLP_HOTK 1
 #endif
+#ifndef GLP_LEAN2
+#define GLP_LEAN2 0
+#endif
+#ifndef GLP_HINT
+#define GLP_HINT 1
+#endif
 #ifndef GLP_LEAN_PEEK
 #define GLP_LEAN_PEEK 0  // A/B (R24 ms/run): 0 17.29, 1 17.27, 2 17.72, 3 17.80; LLP 174.5 / 182.6 / 180.4 / 174.5.  0 never, 1 always, 2 rows predicted to repeat labels, 3 = 2 but not LLP
 #endif
@@ -426,6 +432,58 @@ __device__ __forceinline__ unsigned lean_insert4(const MflArgs& a, const Table& 
   cswap(q0, q2, v0, v2);
   cswap(q1, q3, v1, v3);
   cswap(q1, q2, v1, v2);
+#if GLP_LEAN2
+  // two heads (q0, q1) probe per trip with independent CAS / add chains (twice
+  // the shared-memory operations in flight per lane); q2, q3 queue behind them
+  unsigned fresh = 0u, npa = 0u, npb = 0u;
+  unsigned ha = slot_hash((unsigned)q0, t.tsz), hb = slot_hash((unsigned)q1, t.tsz);
+  const unsigned mask = t.tsz - 1u;
+  while (__any_sync(kFull, (q0 & q1) >= 0 || q0 >= 0 || q1 >= 0)) {
+    const bool ia = q0 >= 0, ib = q1 >= 0;
+    unsigned ka = 0u, kb = 0u;
+    if (ia) ka = atomicCAS(t.key + ha, kFree, (unsigned)q0);
+    if (ib) kb = atomicCAS(t.key + hb, kFree, (unsigned)q1);
+    const bool hita = ia && (ka == kFree || ka == (unsigned)q0);
+    const bool hitb = ib && (kb == kFree || kb == (unsigned)q1);
+    unsigned ca = 0u, cb = 0u;
+    if (hita) ca = atomicAdd(t.cnt + ha, 1u) + 1u;
+    if (hitb) cb = atomicAdd(t.cnt + hb, 1u) + 1u;
+    fresh += (hita && ka == kFree ? 1u : 0u) + (hitb && kb == kFree ? 1u : 0u);
+    if (obs) {
+      if (hita) b.observe(ca, (unsigned)q0, a, (kV && use_v) ? v0 : -1);
+      if (hitb) b.observe(cb, (unsigned)q1, a, (kV && use_v) ? v1 : -1);
+    }
+    bool fa = hita, fb = hitb;
+    if (ia && !hita) {
+      if (++npa >= max_probe) {
+        if (cms) { cms->add((unsigned)q0, 1u); fa = true; }
+        else { flag_set(overflow); q0 = q1 = q2 = q3 = -1; continue; }
+      } else {
+        ha = (ha + 1u) & mask;
+      }
+    }
+    if (ib && !hitb) {
+      if (++npb >= max_probe) {
+        if (cms) { cms->add((unsigned)q1, 1u); fb = true; }
+        else { flag_set(overflow); q0 = q1 = q2 = q3 = -1; continue; }
+      } else {
+        hb = (hb + 1u) & mask;
+      }
+    }
+    if (fa) {
+      q0 = q2; q2 = q3; q3 = -1;
+      if (kV) { v0 = v2; v2 = v3; }
+      ha = slot_hash((unsigned)q0, t.tsz);
+      npa = 0u;
+    }
+    if (fb) {
+      q1 = q2; q2 = q3; q3 = -1;
+      if (kV) { v1 = v2; v2 = v3; }
+      hb = slot_hash((unsigned)q1, t.tsz);
+      npb = 0u;
+    }
+  }
+#else
   unsigned fresh = 0u, np = 0u;
   unsigned h = slot_hash((unsigned)q0, t.tsz);
   const unsigned mask = t.tsz - 1u;
@@ -466,6 +524,7 @@ __device__ __forceinline__ unsigned lean_insert4(const MflArgs& a, const Table& 
       }
     }
   }
+#endif
   return fresh;
 }
 
@@ -473,7 +532,8 @@ template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
                                                   const int (&labin)[N], Best<VAR>& b, volatile int* overflow,
                                                   const int (&vin)[N], bool use_v, bool hot_ok = true,
-                                                  const Cms* cms = nullptr, bool peek = false) {
+                                                  const Cms* cms = nullptr, bool peek = false, int hint = -1,
+                                                  int hintv = -1) {
   // use_v (LLP with a.LV): labels carry their V, so LLP observes at insert
   // like CLASSIC; otherwise LLP scores from the final table (table_scan)
   const bool obs = VAR != V_LLP || use_v;
@@ -482,8 +542,11 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
 #pragma unroll
   for (int j = 0; j < N; ++j) lab[j] = labin[j];
   unsigned nfresh = 0;
-  int cand = b.have() ? (int)b.label() : -1;
-  int candv = b.have() ? b.bv : -1;
+  // hot candidate: the lane's best so far, else the hint (the vertex's own
+  // label L_{t-1}[v], the row's MFL of the last iteration: GLP_HINT), else
+  // the lane's first label of this batch
+  int cand = b.have() ? (int)b.label() : (GLP_HINT ? hint : -1);
+  int candv = b.have() ? b.bv : (GLP_HINT ? hintv : -1);
 #pragma unroll
   for (int j = N - 1; j >= 0; --j) {
     candv = (cand < 0 && lab[j] >= 0) ? (use_v ? vin[j] : -1) : candv;
@@ -617,10 +680,13 @@ __device__ __forceinline__ unsigned pred_est(unsigned raw, unsigned rawprev, uns
 }
 // Sorted-row candidate: all labels were distinct last time and the fast path
 // has not been tried on them (every row at t = 1); never for SEEDED (R12).
+// Only at t = 1: sorted labels come from PickLabel's identity labelling
+// [P:68] on sorted rows; a row whose labels were all distinct at t >= 2 is not
+// sorted (retrying it cost SBM 0.3 ms at t = 3).
 template <int VAR>
-__device__ __forceinline__ bool mono_cand(unsigned raw, unsigned cap, int d) {
+__device__ __forceinline__ bool mono_cand(unsigned raw, unsigned cap, int d, int t) {
   const unsigned p = cap ? min(raw & kPredMask, cap) : (raw & kPredMask);
-  return VAR != V_SEEDED && !(raw & kMonoTried) && p >= (unsigned)d;
+  return VAR != V_SEEDED && t <= 1 && !(raw & kMonoTried) && p >= (unsigned)d;
 }
 
 // Per-thread iteration statistics, block-reduced once at kernel exit.
@@ -894,6 +960,9 @@ __device__ __forceinline__ bool warp_quads_increasing(const int (&x)[4], int bas
 #ifndef GLP_W_SORT
 #define GLP_W_SORT 1
 #endif
+#ifndef GLP_W_PAIR
+#define GLP_W_PAIR 1  // rows of <= 64 arcs: two per warp, sort-and-count per half (half_sort_count)
+#endif
 #ifndef GLP_W_SORT_MAX
 #define GLP_W_SORT_MAX 64  // rows up to this many arcs (<= kWRound) take the sort path
                           // A/B (sort 64 / 128 / off): SBM 5.33 / 5.35 / 5.60 ms, R24 17.99 / 17.97 / 18.0-18.4,
@@ -967,6 +1036,77 @@ __device__ __forceinline__ unsigned warp_sort_count(int (&v)[K], const MflArgs& 
   return distinct;  // this lane's runs (the caller reduces over the warp)
 }
 
+// Two short rows per warp (GLP_W_PAIR): each half-warp sorts and counts one
+// row of <= 64 arcs, 4 per lane (element i = 4 * (lane & 15) + j, the int4
+// load layout), with one 64-key bitonic network whose cross-lane stages stay
+// inside the half (partner lane ^ st / 4 <= 8): every instruction serves both
+// rows ("one-warp-multi-vertices" [P:227-234] for rows past the low bin).
+// Invalid arcs (-1, padding) sort last as INT_MAX.  Observes every run
+// (count, label) into b (the lane's half), returns the lane's runs.
+template <int VAR>
+__device__ __forceinline__ unsigned half_sort_count(int (&v)[4], const MflArgs& a, Best<VAR>& b) {
+  const int lane = threadIdx.x & 31, hl = lane & 15;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) v[j] = v[j] < 0 ? INT_MAX : v[j];
+#pragma unroll
+  for (int k = 2; k <= 64; k <<= 1) {
+#pragma unroll
+    for (int st = k >> 1; st > 0; st >>= 1) {
+      if (st >= 4) {
+        const int ls = st / 4;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int o = __shfl_xor_sync(kFull, v[j], ls);
+          const int i = 4 * hl + j;
+          const bool up = (i & k) == 0;
+          const bool low = (hl & ls) == 0;
+          v[j] = (low == up) ? min(v[j], o) : max(v[j], o);
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int pj = j ^ st;
+          if (pj > j) {
+            const int i = 4 * hl + j;
+            const bool up = (i & k) == 0;
+            const int x = v[j], y = v[pj];
+            v[j] = up ? min(x, y) : max(x, y);
+            v[pj] = up ? max(x, y) : min(x, y);
+          }
+        }
+      }
+    }
+  }
+  const unsigned half = lane < 16 ? 0x0000ffffu : 0xffff0000u;
+  const int prev_last = __shfl_up_sync(kFull, v[3], 1);
+  bool start[4];
+  start[0] = v[0] != INT_MAX && (hl == 0 || prev_last != v[0]);
+#pragma unroll
+  for (int j = 1; j < 4; ++j) start[j] = v[j] != INT_MAX && v[j] != v[j - 1];
+  int nvalid = 0;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) nvalid += __popc(__ballot_sync(kFull, v[j] != INT_MAX) & half);
+  int first_start = 4;
+#pragma unroll
+  for (int j = 3; j >= 0; --j) first_start = start[j] ? j : first_start;
+  const unsigned with = __ballot_sync(kFull, first_start < 4) & half;
+  const unsigned after = lane < 31 ? (with >> (lane + 1)) << (lane + 1) : 0u;  // later lanes of the half
+  const int nl = after ? __ffs(after) - 1 : -1;                                 // next lane holding a start
+  const int nfs = __shfl_sync(kFull, first_start, nl < 0 ? lane : nl);
+  const int base = 4 * hl;
+  int nxt = nl >= 0 ? 4 * (nl & 15) + nfs : nvalid;
+  unsigned distinct = 0;
+#pragma unroll
+  for (int j = 3; j >= 0; --j) {
+    if (start[j]) {
+      b.observe((unsigned)(nxt - (base + j)), (unsigned)v[j], a);
+      ++distinct;
+      nxt = base + j;
+    }
+  }
+  return distinct;
+}
+
 // ---------------------------------------------------------------------------
 // mfl_warp: one warp per row of class W (few distinct labels): per-warp shared
 // table of pow2 >= 4*pred slots (<= 512), one 128-bit load per lane per
@@ -1011,17 +1151,27 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
     BinItem mine;
     mine.start = 0; mine.v = 0; mine.d = 0;
     unsigned mpred = 0;
+    int mhint = -1, mhintv = -1;  // L_{t-1} of the row's vertex (and its V: LLP with LV)
     bool ok = il < a.n_items;
     if (ok) {
       mine = a.items[il];
       const unsigned raw = a.pred[il];
       // in this kernel bit 31 of mpred marks a sorted-row candidate
-      const bool cand = mono_cand<VAR>(raw, a.pred_cap, mine.d);
+      const bool cand = mono_cand<VAR>(raw, a.pred_cap, mine.d, a.t);
       mpred = pred_est<VAR>(raw, a.pred_prev[il], a.pred_cap) | (cand ? kMonoTried : 0u);
       ok = row_class(mpred & kPredMask, mine.d, cand, a.mono_kernel) == CLS_W;
       if (ok && !dense_ && !a.flag[a.vb + mine.v]) {
         ok = false;
         a.pred_next[il] = raw;  // inactive: carry the prediction forward
+      }
+      if (GLP_HINT && ok && !cand) {
+        if (VAR == V_LLP && a.LV != nullptr) {
+          const int2 x = __ldg(a.LV + a.vb + mine.v);
+          mhint = x.x;
+          mhintv = x.y;
+        } else {
+          mhint = ld_label(a.R + a.vb + mine.v);
+        }
       }
     }
     unsigned todo = __ballot_sync(kFull, ok);
@@ -1031,6 +1181,56 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
     unsigned long long rkey = 0ull;
     unsigned rlab = kNoLabel, rpred = 0u;
     int rscan = 0;
+    if (GLP_W_PAIR) {
+      // rows of <= 64 arcs (not sorted-row candidates): two per warp, one per
+      // half, sort-and-count (half_sort_count)
+      unsigned shortm = __ballot_sync(kFull, ok && mine.d <= 64 && !(mpred & kMonoTried)) & todo;
+      todo &= ~shortm;
+      while (shortm) {
+        const int ja = __ffs(shortm) - 1;
+        shortm &= shortm - 1;
+        const int jb = shortm ? __ffs(shortm) - 1 : -1;
+        if (jb >= 0) shortm &= shortm - 1;
+        const int jm = lane < 16 ? ja : jb;  // this half's row (-1: none)
+        const int64_t st = __shfl_sync(kFull, mine.start, jm < 0 ? 0 : jm);
+        const int dsrc = __shfl_sync(kFull, mine.d, jm < 0 ? 0 : jm);  // (every lane shuffles)
+        const int dd = jm < 0 ? 0 : dsrc;
+        const int hl = lane & 15;
+        int4 u = make_int4(-1, -1, -1, -1);
+        if (4 * hl < dd) u = ld_stream4(a.col + st + 4 * hl);
+        int v[4] = {gather(a, u.x), gather(a, u.y), gather(a, u.z), gather(a, u.w)};
+        Best<VAR> b;
+        unsigned fr = half_sort_count<VAR>(v, a, b);
+#pragma unroll
+        for (int s2 = 8; s2 > 0; s2 >>= 1) {  // reduce within the half
+          const unsigned long long k2 = __shfl_xor_sync(kFull, b.key, s2);
+          const unsigned l2 = VAR == V_LLP ? __shfl_xor_sync(kFull, b.lab, s2) : 0u;
+          b.merge(k2, l2);
+          fr += __shfl_xor_sync(kFull, fr, s2);
+        }
+        const unsigned long long ka = __shfl_sync(kFull, b.key, 0), kb = __shfl_sync(kFull, b.key, 16);
+        const unsigned la = __shfl_sync(kFull, b.lab, 0), lb = __shfl_sync(kFull, b.lab, 16);
+        const unsigned fa = __shfl_sync(kFull, fr, 0), fb = __shfl_sync(kFull, fr, 16);
+        if (lane == ja || lane == jb) {
+          const bool isa = lane == ja;
+          rdone = true;
+          rkey = isa ? ka : kb;
+          rlab = isa ? la : lb;
+          rscan = mine.d;
+          rpred = max(isa ? fa : fb, 1u);
+        }
+      }
+    }
+    if (!todo) {
+      if (rdone) {
+        Best<VAR> r;
+        r.key = rkey;
+        r.lab = rlab;
+        a.pred_next[il] = rpred;
+        update_vertex<VAR>(a, mine.v, mine.d, r.have(), r.label(), ty, rscan);
+      }
+      continue;
+    }
     int jl = __ffs(todo) - 1;
     todo &= todo - 1;
     int64_t start = __shfl_sync(kFull, mine.start, jl);
@@ -1053,6 +1253,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       const unsigned tsz =
           min(max(64u, 1u << (32 - __clz(GLP_W_LOAD * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
       const Table tab{wtabs + (size_t)wid * kWSlots, tsz};
+      const int hint = __shfl_sync(kFull, mhint, jl), hintv = __shfl_sync(kFull, mhintv, jl);
       // rows of <= 128 arcs predicted mostly distinct: sort-and-count, no table
       const bool wsort = GLP_W_SORT && d <= GLP_W_SORT_MAX && !(pred & kMonoTried) && 4u * (pred & kPredMask) > (unsigned)d;
       if (!wsort) tab.clear(lane, 32);
@@ -1115,7 +1316,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
             m8[2] = gather_lv(a, v0.z, use_v, mv8[2]); m8[3] = gather_lv(a, v0.w, use_v, mv8[3]);
             m8[4] = gather_lv(a, v1.x, use_v, mv8[4]); m8[5] = gather_lv(a, v1.y, use_v, mv8[5]);
             m8[6] = gather_lv(a, v1.z, use_v, mv8[6]); m8[7] = gather_lv(a, v1.w, use_v, mv8[7]);
-            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v, hot, nullptr, pk);
+            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v, hot, nullptr, pk, hint, hintv);
           }
         }
         if (wsort) {  // the whole row is this round (d <= kWRound)
@@ -1133,11 +1334,11 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           break;
         }
         if (kWRound == 256 && d - off > 128) {  // warp-uniform
-          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v, hot, nullptr, pk);
+          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v, hot, nullptr, pk, hint, hintv);
         } else {
           const int l4[4] = {l[0], l[1], l[2], l[3]};
           const int v4[4] = {lv[0], lv[1], lv[2], lv[3]};
-          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v, hot, nullptr, pk);
+          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v, hot, nullptr, pk, hint, hintv);
         }
         __syncwarp();
         over = warp_flag(&s_over[wid]);
@@ -1205,7 +1406,7 @@ __global__ void __launch_bounds__(kMonoBlock, GLP_MONO_MINB) mfl_mono(MflArgs a)
     if (ok) {
       mine = a.items[il];
       const unsigned raw = a.pred[il];
-      ok = mono_cand<VAR>(raw, a.pred_cap, mine.d) &&
+      ok = mono_cand<VAR>(raw, a.pred_cap, mine.d, a.t) &&
            row_class(raw & kPredMask, mine.d, true, true) == CLS_MONO;
       if (ok && !dense_ && !a.flag[a.vb + mine.v]) {
         ok = false;
@@ -1300,7 +1501,8 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
                                             volatile int* overflow, int* distinct, Best<VAR>& b,
                                             volatile int* major, unsigned fparts = 1u, int* scanned = nullptr,
-                                            bool hot = true, const Cms* cms = nullptr, bool peek = false) {
+                                            bool hot = true, const Cms* cms = nullptr, bool peek = false,
+                                            int hint = -1, int hintv = -1) {
   constexpr int STEP = BLOCK * 4 * UNROLL;
   unsigned fresh = 0;
   int base = 0;
@@ -1329,7 +1531,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
     }
-    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot, cms, peek);
+    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot, cms, peek, hint, hintv);
     if (GLP_MAJORITY && VAR != V_LLP && major != nullptr && base + STEP < d) {
       // a strict-majority observation ends the row for every warp (they poll the flag)
       const bool m = strict_majority(b, d);
@@ -1583,6 +1785,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
   __shared__ int s_k0, s_nsel, s_sel[32], s_cand[32];
   __shared__ BinItem s_item[32];
   __shared__ unsigned s_pe[32], s_raw[32];
+  __shared__ int s_hint[32], s_hintv[32];
   const int n_redo = a.mode ? (int)*a.redo_in_n : 0;
   const int lim = a.mode ? n_redo : a.n_items;
   for (;;) {
@@ -1614,7 +1817,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
         itk = a.items[ik];
         raw = a.pred[ik];
         pe = pred_est<VAR>(raw, a.pred_prev[ik], a.pred_cap);
-        cnd = mono_cand<VAR>(raw, a.pred_cap, itk.d);
+        cnd = mono_cand<VAR>(raw, a.pred_cap, itk.d, a.t);
         if (!a.mode) {
           ok = row_class(pe, itk.d, cnd, a.mono_kernel) == CLS;
           if (ok && !dense_ && !a.flag[a.vb + itk.v]) {
@@ -1626,6 +1829,18 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       const unsigned m = __ballot_sync(kFull, ok);
       if (ok) {
         const int pos = __popc(m & ((1u << threadIdx.x) - 1u));
+        int hn = -1, hv = -1;  // L_{t-1} of the row's vertex: the first hot label (GLP_HINT)
+        if (GLP_HINT && !cnd) {
+          if (VAR == V_LLP && a.LV != nullptr) {
+            const int2 x = __ldg(a.LV + a.vb + itk.v);
+            hn = x.x;
+            hv = x.y;
+          } else {
+            hn = ld_label(a.R + a.vb + itk.v);
+          }
+        }
+        s_hint[pos] = hn;
+        s_hintv[pos] = hv;
         s_sel[pos] = ik;
         s_item[pos] = itk;
         s_pe[pos] = pe;
@@ -1698,7 +1913,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : (PART ? tsz : kTabProbe), cur,
                                       (GLP_L_STAGE1 && may_over) ? stageA : nullptr, &s_over, &s_distinct, b,
                                       (may_over && !GLP_L_MAJ) ? nullptr : &s_major, 1u, &s_scan,
-                                      hot_pass(est, d), nullptr, peek_pass<VAR>(est, d));
+                                      hot_pass(est, d), nullptr, peek_pass<VAR>(est, d), s_hint[q], s_hintv[q]);
       __syncthreads();
       over = s_over != 0;
       if (!over && a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
@@ -1739,7 +1954,8 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
             if (gather_pass) {
               block_load_round<BLOCK, UNROLL>(a.col, it.start, d, 0, cur);
               block_count<VAR, BLOCK, UNROLL, GLP_L_IPF>(a, it.start, d, tab, kLProbe, cur, stageA, &s_over,
-                                                         &s_distinct, b, nullptr, nparts, nullptr, GLP_HOT_DIV == 0);
+                                                         &s_distinct, b, nullptr, nparts, nullptr, GLP_HOT_DIV == 0,
+                                                         nullptr, false, s_hint[q], s_hintv[q]);
             } else {
               count_staged<VAR, BLOCK>(a, stageA, d, tab, kLProbe, &s_over, &s_distinct, b, nparts, p);
             }

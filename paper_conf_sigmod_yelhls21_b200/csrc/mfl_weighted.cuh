@@ -113,7 +113,7 @@ __global__ void __launch_bounds__(kWtBlock) mfl_wt_block(MflArgs a) {
     // Sorted-row fast path (t = 1's unique labels on sorted rows, checked on
     // the data): labels strictly increasing along the row occur once each, so
     // a label's weight sum is its arc's weight -- no table, one pass.
-    if (mono_cand<VAR>(raw, a.pred_cap, d)) {
+    if (mono_cand<VAR>(raw, a.pred_cap, d, a.t)) {
       bool inc = true;
       for (int e = threadIdx.x; e < d; e += kWtBlock) {
         const int l = gather(a, a.col[it.start + e]);
