@@ -35,6 +35,7 @@
 #include <stdint.h>
 
 #include <climits>
+#include <type_traits>
 
 #include "glp_internal.cuh"
 
@@ -390,7 +391,7 @@ struct Cms {
 #define GLP_LEAN2 0
 #endif
 #ifndef GLP_HINT
-#define GLP_HINT 1
+#define GLP_HINT 0  // A/B: R24 17.23 -> 17.21, SBM 5.28 -> 5.49, LLP 176.9 -> 174.7 ms/run (not kept)
 #endif
 #ifndef GLP_LEAN_PEEK
 #define GLP_LEAN_PEEK 0  // A/B (R24 ms/run): 0 17.29, 1 17.27, 2 17.72, 3 17.80; LLP 174.5 / 182.6 / 180.4 / 174.5.  0 never, 1 always, 2 rows predicted to repeat labels, 3 = 2 but not LLP
@@ -1043,31 +1044,32 @@ __device__ __forceinline__ unsigned warp_sort_count(int (&v)[K], const MflArgs& 
 // rows ("one-warp-multi-vertices" [P:227-234] for rows past the low bin).
 // Invalid arcs (-1, padding) sort last as INT_MAX.  Observes every run
 // (count, label) into b (the lane's half), returns the lane's runs.
-template <int VAR>
-__device__ __forceinline__ unsigned half_sort_count(int (&v)[4], const MflArgs& a, Best<VAR>& b) {
+template <int VAR, int K>
+__device__ __forceinline__ unsigned half_sort_count(int (&v)[K], const MflArgs& a, Best<VAR>& b) {
+  constexpr int NH = 16 * K;  // keys per half
   const int lane = threadIdx.x & 31, hl = lane & 15;
 #pragma unroll
-  for (int j = 0; j < 4; ++j) v[j] = v[j] < 0 ? INT_MAX : v[j];
+  for (int j = 0; j < K; ++j) v[j] = v[j] < 0 ? INT_MAX : v[j];
 #pragma unroll
-  for (int k = 2; k <= 64; k <<= 1) {
+  for (int k = 2; k <= NH; k <<= 1) {
 #pragma unroll
     for (int st = k >> 1; st > 0; st >>= 1) {
-      if (st >= 4) {
-        const int ls = st / 4;
+      if (st >= K) {
+        const int ls = st / K;
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < K; ++j) {
           const int o = __shfl_xor_sync(kFull, v[j], ls);
-          const int i = 4 * hl + j;
+          const int i = K * hl + j;
           const bool up = (i & k) == 0;
           const bool low = (hl & ls) == 0;
           v[j] = (low == up) ? min(v[j], o) : max(v[j], o);
         }
       } else {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < K; ++j) {
           const int pj = j ^ st;
           if (pj > j) {
-            const int i = 4 * hl + j;
+            const int i = K * hl + j;
             const bool up = (i & k) == 0;
             const int x = v[j], y = v[pj];
             v[j] = up ? min(x, y) : max(x, y);
@@ -1078,26 +1080,26 @@ __device__ __forceinline__ unsigned half_sort_count(int (&v)[4], const MflArgs& 
     }
   }
   const unsigned half = lane < 16 ? 0x0000ffffu : 0xffff0000u;
-  const int prev_last = __shfl_up_sync(kFull, v[3], 1);
-  bool start[4];
+  const int prev_last = __shfl_up_sync(kFull, v[K - 1], 1);
+  bool start[K];
   start[0] = v[0] != INT_MAX && (hl == 0 || prev_last != v[0]);
 #pragma unroll
-  for (int j = 1; j < 4; ++j) start[j] = v[j] != INT_MAX && v[j] != v[j - 1];
+  for (int j = 1; j < K; ++j) start[j] = v[j] != INT_MAX && v[j] != v[j - 1];
   int nvalid = 0;
 #pragma unroll
-  for (int j = 0; j < 4; ++j) nvalid += __popc(__ballot_sync(kFull, v[j] != INT_MAX) & half);
-  int first_start = 4;
+  for (int j = 0; j < K; ++j) nvalid += __popc(__ballot_sync(kFull, v[j] != INT_MAX) & half);
+  int first_start = K;
 #pragma unroll
-  for (int j = 3; j >= 0; --j) first_start = start[j] ? j : first_start;
-  const unsigned with = __ballot_sync(kFull, first_start < 4) & half;
+  for (int j = K - 1; j >= 0; --j) first_start = start[j] ? j : first_start;
+  const unsigned with = __ballot_sync(kFull, first_start < K) & half;
   const unsigned after = lane < 31 ? (with >> (lane + 1)) << (lane + 1) : 0u;  // later lanes of the half
   const int nl = after ? __ffs(after) - 1 : -1;                                 // next lane holding a start
   const int nfs = __shfl_sync(kFull, first_start, nl < 0 ? lane : nl);
-  const int base = 4 * hl;
-  int nxt = nl >= 0 ? 4 * (nl & 15) + nfs : nvalid;
+  const int base = K * hl;
+  int nxt = nl >= 0 ? K * (nl & 15) + nfs : nvalid;
   unsigned distinct = 0;
 #pragma unroll
-  for (int j = 3; j >= 0; --j) {
+  for (int j = K - 1; j >= 0; --j) {
     if (start[j]) {
       b.observe((unsigned)(nxt - (base + j)), (unsigned)v[j], a);
       ++distinct;
@@ -1181,10 +1183,12 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
     unsigned long long rkey = 0ull;
     unsigned rlab = kNoLabel, rpred = 0u;
     int rscan = 0;
-    if (GLP_W_PAIR) {
-      // rows of <= 64 arcs (not sorted-row candidates): two per warp, one per
-      // half, sort-and-count (half_sort_count)
-      unsigned shortm = __ballot_sync(kFull, ok && mine.d <= 64 && !(mpred & kMonoTried)) & todo;
+    // rows of <= 64 (<= 128: GLP_W_PAIR 2) arcs, not sorted-row candidates:
+    // two per warp, one per half, sort-and-count (half_sort_count)
+    auto pair_pass = [&](auto kc) {
+      constexpr int K = decltype(kc)::value;
+      unsigned shortm =
+          __ballot_sync(kFull, ok && mine.d <= 16 * K && mine.d > (K == 4 ? 0 : 64) && !(mpred & kMonoTried)) & todo;
       todo &= ~shortm;
       while (shortm) {
         const int ja = __ffs(shortm) - 1;
@@ -1196,11 +1200,15 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
         const int dsrc = __shfl_sync(kFull, mine.d, jm < 0 ? 0 : jm);  // (every lane shuffles)
         const int dd = jm < 0 ? 0 : dsrc;
         const int hl = lane & 15;
-        int4 u = make_int4(-1, -1, -1, -1);
-        if (4 * hl < dd) u = ld_stream4(a.col + st + 4 * hl);
-        int v[4] = {gather(a, u.x), gather(a, u.y), gather(a, u.z), gather(a, u.w)};
+        int v[K];
+#pragma unroll
+        for (int q = 0; q < K; q += 4) {
+          int4 u = make_int4(-1, -1, -1, -1);
+          if (K * hl + q < dd) u = ld_stream4(a.col + st + K * hl + q);
+          v[q] = gather(a, u.x); v[q + 1] = gather(a, u.y); v[q + 2] = gather(a, u.z); v[q + 3] = gather(a, u.w);
+        }
         Best<VAR> b;
-        unsigned fr = half_sort_count<VAR>(v, a, b);
+        unsigned fr = half_sort_count<VAR, K>(v, a, b);
 #pragma unroll
         for (int s2 = 8; s2 > 0; s2 >>= 1) {  // reduce within the half
           const unsigned long long k2 = __shfl_xor_sync(kFull, b.key, s2);
@@ -1220,7 +1228,9 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           rpred = max(isa ? fa : fb, 1u);
         }
       }
-    }
+    };
+    if (GLP_W_PAIR >= 1) pair_pass(std::integral_constant<int, 4>());
+    if (GLP_W_PAIR >= 2) pair_pass(std::integral_constant<int, 8>());
     if (!todo) {
       if (rdone) {
         Best<VAR> r;
