@@ -47,12 +47,13 @@ __global__ void k_unpermute(const int32_t* __restrict__ L, const int32_t* __rest
 // labelled neighbour and keeps -1, R5).
 __global__ void k_init_seeds(const int32_t* __restrict__ seeds, int64_t ns, const int32_t* __restrict__ pos,
                              int32_t* __restrict__ L0, int32_t* __restrict__ L1, uint8_t* __restrict__ is_seed,
-                             int2* __restrict__ so, int64_t vb, int64_t ve) {
+                             int2* __restrict__ so, int64_t vb, int64_t ve, uint32_t* __restrict__ lbits) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < ns; i += (int64_t)gridDim.x * blockDim.x) {
     const int32_t s = seeds[i];
     const int32_t q = pos[s];
     L0[q] = s;
     L1[q] = s;
+    if (lbits) atomicOr(lbits + (q >> 5), 1u << (q & 31));
     if (q >= vb && q < ve) {
       is_seed[q - vb] = 1;
       so[q - vb] = make_int2(0, s);

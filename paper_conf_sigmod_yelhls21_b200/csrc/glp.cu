@@ -1018,6 +1018,16 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
       CK(cudaMemsetAsync(g->flag[f], 0, std::max<int64_t>(g->npad, 1), s));
       g->flag_clean[f] = true;
     }
+  // SEEDED presence filter (mfl_kernels.cuh lbit_clear): one rank, label
+  // array larger than ~3/4 of L2 (GLP_LBITS=0 off, =1 forced)
+  const char* lbenv = getenv("GLP_LBITS");
+  const bool use_lbits = variant == GLP_VARIANT_SEEDED && !g->comm && !(lbenv && lbenv[0] == '0') &&
+                         ((lbenv && lbenv[0] == '1') || g->npad * (int64_t)sizeof(int32_t) >= (96ll << 20));
+  if (use_lbits) {
+    const int64_t words = (g->npad + 31) / 32;
+    if (!g->lbits) g->lbits = dalloc<uint32_t>(g, std::max<int64_t>(words, 1));
+    CK(cudaMemsetAsync(g->lbits, 0, std::max<int64_t>(words, 1) * sizeof(uint32_t), s));
+  }
   if (variant == GLP_VARIANT_SEEDED && n_seeds > 0) {
     if (n_seeds > g->seeds_cap) {
       g->d_seeds = dalloc<int32_t>(g, n_seeds);
@@ -1025,7 +1035,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     }
     CK(cudaMemcpyAsync(g->d_seeds, seeds, n_seeds * sizeof(int32_t), cudaMemcpyHostToDevice, s));
     k_init_seeds<<<ga, 256, 0, s>>>(g->d_seeds, n_seeds, g->pos, g->L[0], g->L[1], g->is_seed, g->so, g->vb,
-                                     g->ve);
+                                     g->ve, use_lbits ? g->lbits : nullptr);
     g->init_launches += 1;
     CK(cudaGetLastError());
   }
@@ -1125,6 +1135,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
   int32_t iters = 0;
   int reason = GLP_STOP_MAX_ITERS;
   int64_t changed_last = 0, arcs_total = 0;
+  int64_t labelled_bound = variant == GLP_VARIANT_SEEDED ? n_seeds : g->n;  // presence filter: vertices that may hold a label
   int64_t launches = 0;  // kernels of this run (excluding memsets/copies)
 
   // ---- device-driven loop (one rank, not profiled): the stop rule and the
@@ -1310,6 +1321,10 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     a.cms = p.tail_cms ? 1 : 0;
     a.cms_ht = p.cms_ht_slots > 0 ? (unsigned)p.cms_ht_slots : 0u;
     a.cms_depth = p.cms_depth > 0 ? (unsigned)p.cms_depth : 4u;
+    // the filter pays while at most half the vertices can hold a label
+    // (bound: seeds + every change so far; it only grows, so once off the
+    // bitmap is never read again and need not be maintained)
+    if (use_lbits && 2.0 * (double)labelled_bound < (double)g->n) { a.lbits = g->lbits; a.lbits_w = g->lbits; }
     if (g->weighted) {
       launches += variant == GLP_VARIANT_SEEDED ? launch_wt<V_SEEDED>(g, a, prof, pend, used)
                                                 : launch_wt<V_CLASSIC>(g, a, prof, pend, used);
@@ -1386,6 +1401,7 @@ void run_impl(glp_graph* g, glp_variant variant, int32_t max_iters, const int32_
     used = 1;  // ev_run0 stays; everything else is recycled
     iters = t;
     changed_last = st.changed;
+    labelled_bound += st.changed;
     arcs_total += st.active_arcs;
     // stop rule (R8): fixed point, or L_t == L_{t-2} (d2 == 0) with changes
     bool stop = false;

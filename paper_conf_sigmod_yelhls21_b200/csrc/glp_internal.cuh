@@ -212,6 +212,9 @@ struct MflArgs {
   int32_t cms;                          // 1: L rows count with HT + CMS
   unsigned cms_ht;                      // HT slots (0 = the whole L table)
   unsigned cms_depth;                   // sketch rows d (width = 8192 / d)
+  // SEEDED presence filter (mfl_kernels.cuh lbit_clear): read / maintained bitmap, or null
+  const uint32_t* __restrict__ lbits;
+  uint32_t* lbits_w;
 };
 
 // Internal error: thrown inside the library, converted to glp_status at the ABI.
@@ -301,6 +304,7 @@ struct glp_graph {
   int32_t* Vloc = nullptr;  // LLP, sharded histogram: this rank's counts (summed into V)
   int2* LV = nullptr;  // LLP: (label, V of the label) of each vertex
   uint8_t* is_seed = nullptr;
+  uint32_t* lbits = nullptr;  // SEEDED presence filter: bit q = L[q] >= 0 (single rank)
   uint8_t* flag[2] = {nullptr, nullptr};
   bool flag_clean[2] = {true, true};
   int32_t* stage = nullptr;  // huge bin staging buffers (grid_huge x stage_stride)

@@ -395,3 +395,23 @@ def test_l_partition_retries_exact(case):
     assert_same_run(csr, 0, 6)
     assert_same_run(csr, 2, 4, gamma=0.5)
     assert_same_run(csr, 1, 6, seeds=[0, int(lab.min()), csr.n - 1])
+
+
+# --------------------------------------------------------------------------- SEEDED presence filter
+@pytest.mark.parametrize("case", ["taobao", "hubs", "rmat_few_seeds"])
+def test_seeded_presence_filter_forced(case, monkeypatch):
+    """GLP_LBITS=1 forces the SEEDED presence bitmap (normally only for label
+    arrays larger than L2): labels and per-iteration changes stay those of the
+    oracle through every row class (low, W pairs, W, M, L, giant)."""
+    monkeypatch.setenv("GLP_LBITS", "1")
+    if case == "taobao":
+        csr, seeds = graphs.taobao(users=200_000, items=50_000, pairs=2_000_000, rings=200, seed=7)
+    elif case == "hubs":
+        csr = _degree_mix([3, 40, 70, 300, 3000, 9000, 70000], seed=4, extra_pairs=200_000)
+        seeds = torch.tensor([0, 5, 17, 123, 4000], dtype=torch.int32)
+    else:
+        csr = graphs.rmat(15, seed=9)
+        seeds = torch.tensor([1, 2, 3, 100, 2000, 30000], dtype=torch.int32)
+    ref, lab, info, st = assert_same_run(csr, 1, 30, seeds=seeds)
+    # the filter is on while at most half the vertices can be labelled
+    assert info.iterations >= 2
