@@ -98,6 +98,10 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_W_LOAD
 #define GLP_W_LOAD 4
 #endif
+#ifndef GLP_LLP_CTH
+#define GLP_LLP_CTH 0  // LLP observe: skip counts below ceil(best score) (Best::cth); A/B R28 LLP 3744 -> 4044 ms/run, R24 LLP 175.1 -> 176.6: off
+#endif
+
 __device__ __forceinline__ int ld_stream(const int32_t* p) {
   int r;
 #if GLP_STREAM_POLICY
@@ -192,13 +196,23 @@ struct Best {
   unsigned long long key = 0ull;
   unsigned lab = kNoLabel;
   int bv = -1;  // LLP: V of the best label
+  // LLP: integer count threshold ceil(best score).  A label with V >= count
+  // scores at most its count (gamma >= 0), so a count below the threshold
+  // cannot reach the best score -- not even tie it -- and needs no double
+  // arithmetic.  (V < count only with repeated arcs: always scored.)
+  int cth = INT_MIN;
   // vl: V[l] when the caller has it (carried with the label, a.LV), else -1
   __device__ __forceinline__ void observe(unsigned cnt, unsigned l, const MflArgs& a, int vl = -1) {
     if (VAR == V_LLP) {
       // V of a permutation labelling is all ones (t = 1)
       const int v = vl >= 0 ? vl : (a.v_ones ? 1 : ld_label(a.V + l));
-      const unsigned long long k = dkey(llp_score(cnt, v, a.gamma));
-      if (k > key || (k == key && l < lab)) { key = k; lab = l; bv = v; }
+      if (GLP_LLP_CTH && v >= (int)cnt && (int)cnt < cth) return;
+      const double sc = llp_score(cnt, v, a.gamma);
+      const unsigned long long k = dkey(sc);
+      if (k > key || (k == key && l < lab)) {
+        key = k; lab = l; bv = v;
+        if (GLP_LLP_CTH) cth = sc >= 2.0e9 ? INT_MAX : sc <= -2.0e9 ? INT_MIN : (int)ceil(sc);
+      }
     } else {
       const unsigned long long k = ((unsigned long long)cnt << 32) | (unsigned long long)(~l);
       key = k > key ? k : key;
