@@ -987,6 +987,9 @@ __device__ __forceinline__ bool warp_quads_increasing(const int (&x)[4], int bas
 #ifndef GLP_W_SORT
 #define GLP_W_SORT 1
 #endif
+#ifndef GLP_W_PAIR_PIPE
+#define GLP_W_PAIR_PIPE 0  // pair p+1's labels and p+2's arcs in flight while pair p is sorted
+#endif
 #ifndef GLP_W_PAIR
 #define GLP_W_PAIR 1  // rows of <= 64 arcs: two per warp, sort-and-count per half (half_sort_count)
 #endif
@@ -1216,25 +1219,52 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       unsigned shortm =
           __ballot_sync(kFull, ok && mine.d <= 16 * K && mine.d > (K == 4 ? 0 : 64) && !(mpred & kMonoTried)) & todo;
       todo &= ~shortm;
-      while (shortm) {
-        const int ja = __ffs(shortm) - 1;
-        shortm &= shortm - 1;
-        const int jb = shortm ? __ffs(shortm) - 1 : -1;
+      const int hl = lane & 15;
+      // pop the next pair of rows (ja: lower half, jb: upper half; -1: none)
+      auto pop = [&](int& ja, int& jb) {
+        ja = shortm ? __ffs(shortm) - 1 : -1;
+        if (ja >= 0) shortm &= shortm - 1;
+        jb = shortm ? __ffs(shortm) - 1 : -1;
         if (jb >= 0) shortm &= shortm - 1;
-        const int jm = lane < 16 ? ja : jb;  // this half's row (-1: none)
+      };
+      // the arcs of this lane's half of a pair (every lane shuffles)
+      auto load_pair = [&](int ja, int jb, int4 (&u)[K / 4]) {
+        const int jm = lane < 16 ? ja : jb;
         const int64_t st = __shfl_sync(kFull, mine.start, jm < 0 ? 0 : jm);
-        const int dsrc = __shfl_sync(kFull, mine.d, jm < 0 ? 0 : jm);  // (every lane shuffles)
+        const int dsrc = __shfl_sync(kFull, mine.d, jm < 0 ? 0 : jm);
         const int dd = jm < 0 ? 0 : dsrc;
-        const int hl = lane & 15;
-        int v[K];
 #pragma unroll
-        for (int q = 0; q < K; q += 4) {
-          int4 u = make_int4(-1, -1, -1, -1);
-          if (K * hl + q < dd) u = ld_stream4(a.col + st + K * hl + q);
-          v[q] = gather(a, u.x); v[q + 1] = gather(a, u.y); v[q + 2] = gather(a, u.z); v[q + 3] = gather(a, u.w);
+        for (int q = 0; q < K / 4; ++q)
+          u[q] = K * hl + 4 * q < dd ? ld_stream4(a.col + st + K * hl + 4 * q) : make_int4(-1, -1, -1, -1);
+      };
+      auto gather_pair = [&](const int4 (&u)[K / 4], int (&v)[K]) {
+#pragma unroll
+        for (int q = 0; q < K / 4; ++q) {
+          v[4 * q] = gather(a, u[q].x); v[4 * q + 1] = gather(a, u[q].y);
+          v[4 * q + 2] = gather(a, u[q].z); v[4 * q + 3] = gather(a, u[q].w);
+        }
+      };
+      // software pipeline over pairs: the arcs of pair p+2 and the labels of
+      // pair p+1 are in flight while pair p is sorted (GLP_W_PAIR_PIPE)
+      int ja0, jb0, ja1, jb1;
+      int4 u0[K / 4], u1[K / 4];
+      int v0[K];
+      pop(ja0, jb0);
+      load_pair(ja0, jb0, u0);
+      gather_pair(u0, v0);
+      pop(ja1, jb1);
+      load_pair(ja1, jb1, u1);
+      while (ja0 >= 0) {
+        int ja2, jb2;
+        int4 u2[K / 4];
+        int v1[K];
+        if (GLP_W_PAIR_PIPE) {
+          pop(ja2, jb2);
+          load_pair(ja2, jb2, u2);
+          gather_pair(u1, v1);
         }
         Best<VAR> b;
-        unsigned fr = half_sort_count<VAR, K>(v, a, b);
+        unsigned fr = half_sort_count<VAR, K>(v0, a, b);
 #pragma unroll
         for (int s2 = 8; s2 > 0; s2 >>= 1) {  // reduce within the half
           const unsigned long long k2 = __shfl_xor_sync(kFull, b.key, s2);
@@ -1245,14 +1275,24 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
         const unsigned long long ka = __shfl_sync(kFull, b.key, 0), kb = __shfl_sync(kFull, b.key, 16);
         const unsigned la = __shfl_sync(kFull, b.lab, 0), lb = __shfl_sync(kFull, b.lab, 16);
         const unsigned fa = __shfl_sync(kFull, fr, 0), fb = __shfl_sync(kFull, fr, 16);
-        if (lane == ja || lane == jb) {
-          const bool isa = lane == ja;
+        if (lane == ja0 || lane == jb0) {
+          const bool isa = lane == ja0;
           rdone = true;
           rkey = isa ? ka : kb;
           rlab = isa ? la : lb;
           rscan = mine.d;
           rpred = max(isa ? fa : fb, 1u);
         }
+        if (!GLP_W_PAIR_PIPE) {
+          pop(ja2, jb2);
+          load_pair(ja2, jb2, u2);
+          gather_pair(u1, v1);
+        }
+        ja0 = ja1; jb0 = jb1; ja1 = ja2; jb1 = jb2;
+#pragma unroll
+        for (int q = 0; q < K; ++q) v0[q] = v1[q];
+#pragma unroll
+        for (int q = 0; q < K / 4; ++q) u1[q] = u2[q];
       }
     };
     if (GLP_W_PAIR >= 1) pair_pass(std::integral_constant<int, 4>());
@@ -2144,7 +2184,10 @@ __device__ __forceinline__ unsigned giant_add(unsigned long long* tab, unsigned 
 #endif
 constexpr int kGSlots = 8192;  // shared pre-aggregation table (64 KB)
 template <int VAR>
-__global__ void __launch_bounds__(kGBlock) mfl_giant_count(MflArgs a) {
+#ifndef GLP_G_MINB
+#define GLP_G_MINB 1  // 1: 56-64 registers, no spills (3: 32 registers + spills); A/B TaoBao 97.3 -> 94.2 ms/run, R24 17.51 -> 17.41
+#endif
+__global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a) {
   GLP_CTL_PROLOGUE(a)
   extern __shared__ __align__(16) unsigned long long gsm[];  // kGSlots (GLP_GIANT_SMEM)
   __shared__ int s_k;
