@@ -123,6 +123,27 @@ __global__ void k_push_big(const int64_t* __restrict__ ioff, const int32_t* __re
   }
 }
 
+// Weighted LP: the largest weight total of the giant rows (one block per
+// row): giant tables hold counts in kGCountBits bits.
+__global__ void k_giant_wsum_max(const BinItem* __restrict__ rows, int32_t n_giant, const uint32_t* __restrict__ w2,
+                                 unsigned long long* __restrict__ out) {
+  __shared__ unsigned long long red[32];
+  for (int i = blockIdx.x; i < n_giant; i += gridDim.x) {
+    const BinItem it = rows[i];
+    unsigned long long s = 0;
+    for (int e = threadIdx.x; e < it.d; e += blockDim.x) s += w2[it.start + e];
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long t = 0;
+      for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
+      atomicMax(out, t);
+    }
+    __syncthreads();
+  }
+}
+
 // Sparse iterations: a low-degree chunk is active if any of its vertices is.
 __global__ void k_chunk_flags(const LowChunk* __restrict__ chunks, int32_t n_chunks, int64_t low_base,
                               const uint8_t* __restrict__ flag, int64_t vb, uint8_t* __restrict__ cflag,

@@ -670,6 +670,20 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       CK(cudaStreamSynchronize(g->stream));
       if (bad & 16) fail(GLP_ERR_INVALID_GRAPH, "weights must be in [1, 2^31) with every row total < 2^31");
       g->weighted = true;
+      // giant rows whose weight totals fit the giant tables' count field are
+      // counted by the segmented giant kernels (else one block per row)
+      const char* wg = getenv("GLP_WT_GIANT");
+      if (g->n_giant > 0 && !(wg && wg[0] == '0')) {
+        unsigned long long* dmx = nullptr;
+        CK(cudaMallocAsync((void**)&dmx, sizeof(unsigned long long), g->stream));
+        CK(cudaMemsetAsync(dmx, 0, sizeof(unsigned long long), g->stream));
+        k_giant_wsum_max<<<std::min(g->n_giant, g->sms * 4), 256, 0, g->stream>>>(g->rows, g->n_giant, g->w2, dmx);
+        unsigned long long mx = 0;
+        CK(cudaMemcpyAsync(&mx, dmx, sizeof(mx), cudaMemcpyDeviceToHost, g->stream));
+        CK(cudaFreeAsync(dmx, g->stream));
+        CK(cudaStreamSynchronize(g->stream));
+        g->wt_giant = mx < (1ull << kGCountBits);
+      }
     }
     if (g->registered) {  // the caller's arcs are not read after the relayout
       CK(cudaStreamSynchronize(g->stream));
@@ -952,11 +966,26 @@ int launch_wt(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, si
   cudaStream_t s0 = g->stream;
   a.w2 = g->w2; a.ioff = g->ioff; a.ideg = g->ideg;
   int n = 0;
-  if (g->n_gt512) {
+  // giant rows (deg > kGiantMin): segments over all blocks, weights added
+  // into the per-row global tables (mfl_giant_count), when their totals fit
+  const int g0 = g->wt_giant ? g->n_giant : 0;
+  if (g0) {
     MflArgs b = a;
-    b.items = g->rows; b.n_items = g->n_gt512; b.cnt = c + 3; b.work = &sc->work_l;
-    b.pred = g->pred[g->pb]; b.pred_next = g->pred[(g->pb + 1) % 3];
-    const int grid = std::min(g->grid_wtb, g->n_gt512);
+    b.items = g->rows; b.pred = g->pred[g->pb]; b.pred_next = g->pred[(g->pb + 1) % 3];
+    b.cnt = c + 4; b.work = &sc->work_g;
+    b.gsegs = g->gsegs; b.n_gsegs = g->n_gsegs; b.gtab = g->gtab; b.gtab_off = g->gtab_off;
+    b.gcand_key = g->gcand_key; b.gcand_lab = g->gcand_lab; b.gdistinct = g->gdistinct; b.epoch = g->gepoch;
+    timed(g, prof, 7, pend, used, s0, [&] {
+      mfl_giant_count<VAR><<<std::min(g->grid_g, g->n_gsegs), kGBlock, GLP_GIANT_SMEM ? kGSlots * 8 : 0, s0>>>(b);
+      mfl_giant_finish<VAR><<<g->n_giant, 256, 0, s0>>>(b, g->gseg_first);
+    });
+    n += 2;
+  }
+  if (g->n_gt512 > g0) {
+    MflArgs b = a;
+    b.items = g->rows + g0; b.n_items = g->n_gt512 - g0; b.cnt = c + 3; b.work = &sc->work_l;
+    b.pred = g->pred[g->pb] + g0; b.pred_next = g->pred[(g->pb + 1) % 3] + g0;
+    const int grid = std::min(g->grid_wtb, g->n_gt512 - g0);
     timed(g, prof, 10, pend, used, s0,
           [&] { mfl_wt_block<VAR><<<grid, kWtBlock, kWtSlots * 8, s0>>>(b); });
     ++n;

@@ -61,6 +61,9 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_LOW_REDUX
 #define GLP_LOW_REDUX 0
 #endif
+#ifndef GLP_LOW_PIPE
+#define GLP_LOW_PIPE 0  // mfl_low: gathers of the next chunk in flight while this one is counted
+#endif
 #ifndef GLP_LOW_MATCH
 #define GLP_LOW_MATCH 6  // low segments of at least this degree count with match.any (33 = never);
                          // A/B: 6 / 12 / 17 all -2.8 % per R24 run vs never (shuffle loop)
@@ -841,7 +844,38 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
     int u, v, total, d;
     unsigned segs;
     issue(j, u, v, total, d, segs);
+#if GLP_LOW_PIPE
+    // two-stage pipeline: chunk c+1's labels and chunk c+2's arcs are in
+    // flight while chunk c is counted
+    int lvp;
+    int labp = gather_lv(a, u, VAR == V_LLP && a.LV != nullptr, lvp);
+    int pu = -1, pvid = -1, ptotal = 0, pd = 1;
+    unsigned psegs = 0u;
+    bool pmore = todo != 0;
+    if (pmore) {
+      const int nj = __ffs(todo) - 1;
+      todo &= todo - 1;
+      issue(nj, pu, pvid, ptotal, pd, psegs);
+    }
+#endif
     for (;;) {
+#if GLP_LOW_PIPE
+      const bool more = pmore;
+      int nu = pu, nvid = pvid, ntotal = ptotal, nd = pd;
+      unsigned nsegs = psegs;
+      int nlv = -1, nlab = -1;
+      if (more) nlab = gather_lv(a, nu, VAR == V_LLP && a.LV != nullptr, nlv);
+      pmore = todo != 0;
+      pu = -1; pvid = -1; ptotal = 0; pd = 1; psegs = 0u;
+      if (pmore) {
+        const int nj = __ffs(todo) - 1;
+        todo &= todo - 1;
+        issue(nj, pu, pvid, ptotal, pd, psegs);
+      }
+      const int nv = __popc(segs);
+      int lv = lvp;
+      int lab = labp;
+#else
       // prefetch the next chunk while this one is counted
       int nu = -1, nvid = -1, ntotal = 0, nd = 1;
       unsigned nsegs = 0u;
@@ -855,6 +889,7 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       const int nv = __popc(segs);
       int lv;
       int lab = gather_lv(a, u, VAR == V_LLP && a.LV != nullptr, lv);
+#endif
       int r = 0;
       int2 so = make_int2(0, 0);
       if (lane < nv) {
@@ -923,6 +958,10 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       }  // counted
       if (lane < nv) update_vertex_pre<VAR>(a, v, d, h.have(), h.label(), r, so, ty);
       if (!more) break;
+#if GLP_LOW_PIPE
+      labp = nlab;
+      lvp = nlv;
+#endif
       u = nu;
       v = nvid;
       total = ntotal;
@@ -2221,13 +2260,19 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
         const int idx = base + (int)threadIdx.x * 4;
         const int4 u = idx < end ? ld_stream4(a.col + it.start + idx) : make_int4(-1, -1, -1, -1);
         int lab[4] = {gather(a, u.x), gather(a, u.y), gather(a, u.z), gather(a, u.w)};
+        // weighted LP (§8(f)3): a label adds its arc's weight (w2 beside col2)
+        unsigned w[4] = {1u, 1u, 1u, 1u};
+        if (a.w2 != nullptr && idx < end) {
+          const int4 wv = ld_stream4((const int32_t*)a.w2 + it.start + idx);
+          w[0] = (unsigned)wv.x; w[1] = (unsigned)wv.y; w[2] = (unsigned)wv.z; w[3] = (unsigned)wv.w;
+        }
         // hot label of the warp: one shared atomic for all its copies
         const int hot = __shfl_sync(kFull, hotb.have() ? (int)hotb.label() : lab[0] >= 0 ? lab[0] : lab[1], 0);
         if (hot >= 0) {
           unsigned hc = 0;
 #pragma unroll
           for (int j = 0; j < 4; ++j) {
-            hc += lab[j] == hot ? 1u : 0u;
+            hc += lab[j] == hot ? w[j] : 0u;
             lab[j] = lab[j] == hot ? -1 : lab[j];
           }
           const unsigned tot = __reduce_add_sync(kFull, hc);
@@ -2246,10 +2291,10 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
           if (lab[j] < 0) continue;
-          const unsigned c = ht_add(st, (unsigned)lab[j], 1u, kTabProbe, &lf);
+          const unsigned c = ht_add(st, (unsigned)lab[j], w[j], kTabProbe, &lf);
           if (c == 0u) {
             bool fr = false;
-            const unsigned gc = giant_add(tab, tsz, (unsigned)lab[j], 1u, a.epoch, &fr);
+            const unsigned gc = giant_add(tab, tsz, (unsigned)lab[j], w[j], a.epoch, &fr);
             fresh += fr ? 1u : 0u;
             b.observe(gc, (unsigned)lab[j], a);
           }
@@ -2269,10 +2314,15 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
     } else {
       for (int base = sg.begin; base < end; base += kGBlock * 4 * kGUnroll) {
         int lab[4 * kGUnroll], gv[4 * kGUnroll];
+        unsigned wt[4 * kGUnroll];
 #pragma unroll
         for (int j = 0; j < kGUnroll; ++j) {
           const int idx = base + (j * kGBlock + (int)threadIdx.x) * 4;
           const int4 u = idx < end ? ld_stream4(a.col + it.start + idx) : make_int4(-1, -1, -1, -1);
+          int4 wv = make_int4(1, 1, 1, 1);
+          if (a.w2 != nullptr && idx < end) wv = ld_stream4((const int32_t*)a.w2 + it.start + idx);
+          wt[4 * j + 0] = (unsigned)wv.x; wt[4 * j + 1] = (unsigned)wv.y;
+          wt[4 * j + 2] = (unsigned)wv.z; wt[4 * j + 3] = (unsigned)wv.w;
           lab[4 * j + 0] = gather_lv(a, u.x, use_v, gv[4 * j + 0]);
           lab[4 * j + 1] = gather_lv(a, u.y, use_v, gv[4 * j + 1]);
           lab[4 * j + 2] = gather_lv(a, u.z, use_v, gv[4 * j + 2]);
@@ -2284,7 +2334,8 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
           const bool vote = lab[j] >= 0;
           const int hot = __shfl_sync(kFull, cand0 == -2 ? lab[j] : cand0, 0);
           const unsigned m = __ballot_sync(kFull, vote && lab[j] == hot);
-          const unsigned c = vote ? (lab[j] != hot ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u)) : 0u;
+          unsigned c = vote ? (lab[j] != hot ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u)) : 0u;
+          if (a.w2 != nullptr) c = vote ? wt[j] : 0u;  // weighted: every arc adds its own weight
           if (c) {
             bool fr = false;
             const unsigned cnt = giant_add(tab, tsz, (unsigned)lab[j], c, a.epoch, &fr);

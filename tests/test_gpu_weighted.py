@@ -111,3 +111,27 @@ def test_weighted_local_group(P):
         labs = [grp.labels(r).numpy() for r in range(P)]
     for r in range(P):
         assert infos[r].iterations == ref.iterations and (labs[r] == ref.labels).all()
+
+
+@pytest.mark.parametrize("variant", ["classic", "seeded"])
+@pytest.mark.parametrize("giant_kernel", ["1", "0"])
+def test_weighted_giant_rows(variant, giant_kernel, monkeypatch):
+    """Rows past kGiantMin (65536 arcs) with weights: the segmented giant
+    kernels add each arc's weight into the per-row global tables (default),
+    or one block per row (GLP_WT_GIANT=0); both equal the weighted oracle."""
+    monkeypatch.setenv("GLP_WT_GIANT", giant_kernel)
+    rng = np.random.default_rng(11)
+    n_leaf = 90_000
+    hubs = [70_000, 80_000, 66_000]
+    src, dst = [], []
+    for h, d in enumerate(hubs):  # hub h -> d leaves (distinct), leaves cross-linked
+        leaves = rng.choice(n_leaf, d, replace=False) + len(hubs)
+        src.append(np.full(d, h)); dst.append(leaves)
+    a = rng.integers(len(hubs), len(hubs) + n_leaf, 150_000)
+    b = rng.integers(len(hubs), len(hubs) + n_leaf, 150_000)
+    src.append(a); dst.append(b)
+    csr = from_edges(len(hubs) + n_leaf, torch.from_numpy(np.concatenate(src).astype(np.int64)),
+                     torch.from_numpy(np.concatenate(dst).astype(np.int64)), "wgiant")
+    w = weights_for(csr, 4)
+    seeds = np.array([0, 5, 17, 400, 9000], dtype=np.int32) if variant == "seeded" else None
+    check(csr, w, variant, 15, seeds=seeds)
