@@ -684,6 +684,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
         CK(cudaStreamSynchronize(g->stream));
         g->wt_giant = mx < (1ull << kGCountBits);
       }
+      const char* wl = getenv("GLP_WT_LOW");
+      g->wt_low_off = wl && wl[0] == '0';
     }
     if (g->registered) {  // the caller's arcs are not read after the relayout
       CK(cudaStreamSynchronize(g->stream));
@@ -757,7 +759,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaFuncSetAttribute(mfl_wt_block<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, wtb_));
     CK(cudaFuncSetAttribute(mfl_wt_block<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, wtb_));
     g->grid_wtw = grid_for(sms, (const void*)mfl_wt_warp<V_CLASSIC>, kWtBlock, wtw_);
-    g->grid_wtb = grid_for(sms, (const void*)mfl_wt_block<V_CLASSIC>, kWtBlock, wtb_);
+    g->grid_wtb = grid_for(sms, (const void*)mfl_wt_block<V_CLASSIC>, kWtBBlock, wtb_);
     g->grid_l = grid_for(sms, (const void*)GLP_L_KERNEL(V_LLP), kLBlock, ls_);
     const int gs_ = GLP_GIANT_SMEM ? kGSlots * 8 : 0;
     CK(cudaFuncSetAttribute(mfl_giant_count<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
@@ -987,10 +989,18 @@ int launch_wt(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, si
     b.pred = g->pred[g->pb] + g0; b.pred_next = g->pred[(g->pb + 1) % 3] + g0;
     const int grid = std::min(g->grid_wtb, g->n_gt512 - g0);
     timed(g, prof, 10, pend, used, s0,
-          [&] { mfl_wt_block<VAR><<<grid, kWtBlock, kWtSlots * 8, s0>>>(b); });
+          [&] { mfl_wt_block<VAR><<<grid, kWtBBlock, kWtSlots * 8, s0>>>(b); });
     ++n;
   }
-  const int64_t lo = g->n_gt512, hi = (int64_t)g->n_rows + g->n_low;
+  // low-degree vertices (deg <= 32): the packed-warp kernel with weight sums
+  if (g->n_chunks && !g->wt_low_off) {
+    MflArgs b = a;
+    b.low_base = g->low_base; b.chunks = g->chunks; b.cflag = g->cflag; b.n_chunks = g->n_chunks; b.cnt = c + 0;
+    const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock - 1) / kLowBlock);
+    timed(g, prof, 0, pend, used, s0, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, s0>>>(b); });
+    ++n;
+  }
+  const int64_t lo = g->n_gt512, hi = (int64_t)g->n_rows + (g->wt_low_off ? g->n_low : 0);
   if (hi > lo) {
     MflArgs b = a;
     b.wt_lo = lo; b.wt_hi = hi; b.cnt = c + 1;

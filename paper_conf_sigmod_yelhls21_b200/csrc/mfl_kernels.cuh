@@ -61,9 +61,6 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_LOW_REDUX
 #define GLP_LOW_REDUX 0
 #endif
-#ifndef GLP_LOW_PIPE
-#define GLP_LOW_PIPE 0  // mfl_low: gathers of the next chunk in flight while this one is counted
-#endif
 #ifndef GLP_LOW_MATCH
 #define GLP_LOW_MATCH 6  // low segments of at least this degree count with match.any (33 = never);
                          // A/B: 6 / 12 / 17 all -2.8 % per R24 run vs never (shuffle loop)
@@ -829,7 +826,8 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
     unsigned todo = __ballot_sync(kFull, act);
     if (!todo) continue;
     // issue the arc and vertex-id loads of chunk j
-    auto issue = [&](int j, int& u, int& v, int& total, int& d, unsigned& segs) {
+    // weighted LP (§8(f)3, a.w2): each lane also loads its arc's weight
+    auto issue = [&](int j, int& u, int& v, int& total, int& d, unsigned& segs, unsigned& wt) {
       const unsigned long long st = __shfl_sync(kFull, mine.st, j);
       const int vbase = __shfl_sync(kFull, mine.vbase, j);
       segs = __shfl_sync(kFull, mine.segmask, j);
@@ -838,58 +836,27 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       const int64_t start = (int64_t)(st & ((1ull << 48) - 1));
       u = lane < total ? ld_stream(a.col + start + lane) : -1;
       v = lane < __popc(segs) ? (int)(a.low_base + vbase + lane) : -1;
+      wt = (a.w2 != nullptr && lane < total) ? (unsigned)ld_stream((const int32_t*)a.w2 + start + lane) : 1u;
     };
     int j = __ffs(todo) - 1;
     todo &= todo - 1;
     int u, v, total, d;
-    unsigned segs;
-    issue(j, u, v, total, d, segs);
-#if GLP_LOW_PIPE
-    // two-stage pipeline: chunk c+1's labels and chunk c+2's arcs are in
-    // flight while chunk c is counted
-    int lvp;
-    int labp = gather_lv(a, u, VAR == V_LLP && a.LV != nullptr, lvp);
-    int pu = -1, pvid = -1, ptotal = 0, pd = 1;
-    unsigned psegs = 0u;
-    bool pmore = todo != 0;
-    if (pmore) {
-      const int nj = __ffs(todo) - 1;
-      todo &= todo - 1;
-      issue(nj, pu, pvid, ptotal, pd, psegs);
-    }
-#endif
+    unsigned segs, wt;
+    issue(j, u, v, total, d, segs, wt);
     for (;;) {
-#if GLP_LOW_PIPE
-      const bool more = pmore;
-      int nu = pu, nvid = pvid, ntotal = ptotal, nd = pd;
-      unsigned nsegs = psegs;
-      int nlv = -1, nlab = -1;
-      if (more) nlab = gather_lv(a, nu, VAR == V_LLP && a.LV != nullptr, nlv);
-      pmore = todo != 0;
-      pu = -1; pvid = -1; ptotal = 0; pd = 1; psegs = 0u;
-      if (pmore) {
-        const int nj = __ffs(todo) - 1;
-        todo &= todo - 1;
-        issue(nj, pu, pvid, ptotal, pd, psegs);
-      }
-      const int nv = __popc(segs);
-      int lv = lvp;
-      int lab = labp;
-#else
       // prefetch the next chunk while this one is counted
       int nu = -1, nvid = -1, ntotal = 0, nd = 1;
-      unsigned nsegs = 0u;
+      unsigned nsegs = 0u, nwt = 1u;
       const bool more = todo != 0;
       if (more) {
         const int nj = __ffs(todo) - 1;
         todo &= todo - 1;
-        issue(nj, nu, nvid, ntotal, nd, nsegs);
+        issue(nj, nu, nvid, ntotal, nd, nsegs, nwt);
       }
       // every vertex of the chunk has degree d; nv vertices, lanes [0, total)
       const int nv = __popc(segs);
       int lv;
       int lab = gather_lv(a, u, VAR == V_LLP && a.LV != nullptr, lv);
-#endif
       int r = 0;
       int2 so = make_int2(0, 0);
       if (lane < nv) {
@@ -908,14 +875,15 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       // t; LLP only while V == 1 (equal scores).
       const int up = __shfl_up_sync(kFull, lab, 1);
       const bool inc = lane >= total || (vote && (lane == sstart || up < lab));
-      if ((VAR != V_LLP || a.v_ones) && __all_sync(kFull, inc)) {
+      const bool wtd = a.w2 != nullptr;  // weighted: counts are weight sums (no shortcut, no match.any)
+      if ((VAR != V_LLP || a.v_ones) && !wtd && __all_sync(kFull, inc)) {
         const int hl = __shfl_sync(kFull, lab, head);
         h.observe(1u, (unsigned)hl, a, 1);
       } else {
       // label frequency inside the vertex's lanes [P:231-232]
       unsigned k = 0;
       bool first = true;  // LLP: only a label's first lane scores it (one V[l] gather per distinct label)
-      if (d >= GLP_LOW_MATCH) {
+      if (d >= GLP_LOW_MATCH && !wtd) {
         // long segments: one match.any over the warp, restricted to the
         // segment's lanes (d warp-uniform), instead of d shuffles
         const unsigned segm = d >= 32 ? kFull : (((1u << d) - 1u) << sstart);
@@ -926,7 +894,8 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
 #pragma unroll 4
         for (int i = 0; i < d; ++i) {
           const bool eq = __shfl_sync(kFull, lab, sstart + i) == lab;
-          k += eq ? 1u : 0u;
+          const unsigned wi = wtd ? __shfl_sync(kFull, wt, sstart + i) : 1u;
+          k += eq ? wi : 0u;
           if (VAR == V_LLP) first = first && !(eq && sstart + i < lane);
         }
       }
@@ -958,15 +927,12 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       }  // counted
       if (lane < nv) update_vertex_pre<VAR>(a, v, d, h.have(), h.label(), r, so, ty);
       if (!more) break;
-#if GLP_LOW_PIPE
-      labp = nlab;
-      lvp = nlv;
-#endif
       u = nu;
       v = nvid;
       total = ntotal;
       d = nd;
       segs = nsegs;
+      wt = nwt;
     }
   }
   tally_flush(ty, a.cnt);

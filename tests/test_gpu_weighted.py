@@ -135,3 +135,21 @@ def test_weighted_giant_rows(variant, giant_kernel, monkeypatch):
     w = weights_for(csr, 4)
     seeds = np.array([0, 5, 17, 400, 9000], dtype=np.int32) if variant == "seeded" else None
     check(csr, w, variant, 15, seeds=seeds)
+
+
+@pytest.mark.parametrize("variant", ["classic", "seeded"])
+@pytest.mark.parametrize("low_kernel", ["1", "0"])
+def test_weighted_low_rows(variant, low_kernel, monkeypatch):
+    """Vertices of degree <= 32 with weights: the packed-warp kernel sums the
+    weights of equal labels per segment (default) or the warp-per-vertex
+    kernel (GLP_WT_LOW=0); every low degree 1..32 occurs."""
+    monkeypatch.setenv("GLP_WT_LOW", low_kernel)
+    rng = np.random.default_rng(21)
+    n = 60_000
+    deg = rng.integers(1, 33, n)
+    src = np.repeat(np.arange(n), deg)
+    dst = rng.integers(0, n // 8, src.size)  # few targets: labels repeat inside segments
+    csr = from_edges(n, torch.from_numpy(src.astype(np.int64)), torch.from_numpy(dst.astype(np.int64)), "wlow")
+    w = weights_for(csr, 9, hi=50)
+    seeds = np.array([1, 2, 3, 50, 700, 5000], dtype=np.int32) if variant == "seeded" else None
+    check(csr, w, variant, 20, seeds=seeds)
