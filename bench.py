@@ -402,6 +402,8 @@ def bench_gpu(args):
             except (OSError, ValueError):
                 gceil = None
         gath = s["arcs"] / (s["ms"] / 1e3) / 1e9  # one label gather per arc
+        gb = 8 if variant == "llp" else 4
+        label_mb = n * gb / 1e6
         roof = {"bound": bound, "kernel": dom, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
                 "bytes_per_launch": s["bytes"] / s["launches"], "ms_per_launch": s["ms"] / s["launches"],
@@ -411,6 +413,14 @@ def bench_gpu(args):
                 "gather_ceiling": {"achieved": round(gath, 1), "peak": gceil, "unit": "G label gathers/s",
                                    "frac": round(gath / gceil, 4) if gceil else None,
                                    "source": "profiles/gather_ceilings.json"},
+                # SURVEY §8(d) "labels beyond L2" (TaoBao, R28): the label
+                # gathers are HBM traffic too -- 4 B per gathered label (8 B:
+                # LLP's (label, V) pairs), credited here as a second figure
+                "with_gathers": ({"achieved": round((s["bytes"] + gb * s["arcs"]) / (s["ms"] / 1e3) / 1e9, 1),
+                                  "frac": round((s["bytes"] + gb * s["arcs"]) / (s["ms"] / 1e3) / 1e9 / peak, 4),
+                                  "bytes_per_gather": gb,
+                                  "why": f"label array {label_mb:.0f} MB exceeds the 126 MB L2"}
+                                 if label_mb > 126 else None),
                 "kernel_timing": f"{kprof_steps} profiled steps with the class kernels serialised (CUDA events per "
                                  f"launch; {sum(prof_ms) / kprof_steps:.3f} ms/step serialised vs the timed region's "
                                  f"concurrent steps)",
