@@ -765,6 +765,8 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaFuncSetAttribute(mfl_giant_count<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
     CK(cudaFuncSetAttribute(mfl_giant_count<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
     CK(cudaFuncSetAttribute(mfl_giant_count<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
+    CK(cudaFuncSetAttribute(mfl_giant_count<V_CLASSIC, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
+    CK(cudaFuncSetAttribute(mfl_giant_count<V_SEEDED, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, gs_));
     g->grid_g = grid_for(sms, (const void*)mfl_giant_count<V_LLP>, kGBlock, gs_);
     g->grid_aux = sms * 8;
     if (g->n_rows > 0) {
@@ -978,7 +980,7 @@ int launch_wt(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, si
     b.gsegs = g->gsegs; b.n_gsegs = g->n_gsegs; b.gtab = g->gtab; b.gtab_off = g->gtab_off;
     b.gcand_key = g->gcand_key; b.gcand_lab = g->gcand_lab; b.gdistinct = g->gdistinct; b.epoch = g->gepoch;
     timed(g, prof, 7, pend, used, s0, [&] {
-      mfl_giant_count<VAR><<<std::min(g->grid_g, g->n_gsegs), kGBlock, GLP_GIANT_SMEM ? kGSlots * 8 : 0, s0>>>(b);
+      mfl_giant_count<VAR, true><<<std::min(g->grid_g, g->n_gsegs), kGBlock, GLP_GIANT_SMEM ? kGSlots * 8 : 0, s0>>>(b);
       mfl_giant_finish<VAR><<<g->n_giant, 256, 0, s0>>>(b, g->gseg_first);
     });
     n += 2;
@@ -997,7 +999,7 @@ int launch_wt(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, si
     MflArgs b = a;
     b.low_base = g->low_base; b.chunks = g->chunks; b.cflag = g->cflag; b.n_chunks = g->n_chunks; b.cnt = c + 0;
     const int grid = std::min<int>(g->grid_low, (g->n_chunks + kLowBlock - 1) / kLowBlock);
-    timed(g, prof, 0, pend, used, s0, [&] { mfl_low<VAR><<<grid, kLowBlock, 0, s0>>>(b); });
+    timed(g, prof, 0, pend, used, s0, [&] { mfl_low<VAR, true><<<grid, kLowBlock, 0, s0>>>(b); });
     ++n;
   }
   const int64_t lo = g->n_gt512, hi = (int64_t)g->n_rows + (g->wt_low_off ? g->n_low : 0);

@@ -805,7 +805,9 @@ __device__ __forceinline__ void update_vertex_pre(const MflArgs& a, int v, int d
   }
 }
 
-template <int VAR>
+// WT: weighted LP (a.w2), a separate instantiation so the unweighted kernel
+// carries no weight code
+template <int VAR, bool WT = false>
 __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
   GLP_CTL_PROLOGUE(a)
   const int lane = threadIdx.x & 31;
@@ -836,7 +838,7 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       const int64_t start = (int64_t)(st & ((1ull << 48) - 1));
       u = lane < total ? ld_stream(a.col + start + lane) : -1;
       v = lane < __popc(segs) ? (int)(a.low_base + vbase + lane) : -1;
-      wt = (a.w2 != nullptr && lane < total) ? (unsigned)ld_stream((const int32_t*)a.w2 + start + lane) : 1u;
+      wt = (WT && lane < total) ? (unsigned)ld_stream((const int32_t*)a.w2 + start + lane) : 1u;
     };
     int j = __ffs(todo) - 1;
     todo &= todo - 1;
@@ -875,7 +877,7 @@ __global__ void __launch_bounds__(kLowBlock) mfl_low(MflArgs a) {
       // t; LLP only while V == 1 (equal scores).
       const int up = __shfl_up_sync(kFull, lab, 1);
       const bool inc = lane >= total || (vote && (lane == sstart || up < lab));
-      const bool wtd = a.w2 != nullptr;  // weighted: counts are weight sums (no shortcut, no match.any)
+      constexpr bool wtd = WT;  // weighted: counts are weight sums (no shortcut, no match.any)
       if ((VAR != V_LLP || a.v_ones) && !wtd && __all_sync(kFull, inc)) {
         const int hl = __shfl_sync(kFull, lab, head);
         h.observe(1u, (unsigned)hl, a, 1);
@@ -2188,10 +2190,10 @@ __device__ __forceinline__ unsigned giant_add(unsigned long long* tab, unsigned 
 #define GLP_GIANT_SMEM 1
 #endif
 constexpr int kGSlots = 8192;  // shared pre-aggregation table (64 KB)
-template <int VAR>
 #ifndef GLP_G_MINB
 #define GLP_G_MINB 1  // 1: 56-64 registers, no spills (3: 32 registers + spills); A/B TaoBao 97.3 -> 94.2 ms/run, R24 17.51 -> 17.41
 #endif
+template <int VAR, bool WT = false>
 __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a) {
   GLP_CTL_PROLOGUE(a)
   extern __shared__ __align__(16) unsigned long long gsm[];  // kGSlots (GLP_GIANT_SMEM)
@@ -2228,7 +2230,7 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
         int lab[4] = {gather(a, u.x), gather(a, u.y), gather(a, u.z), gather(a, u.w)};
         // weighted LP (§8(f)3): a label adds its arc's weight (w2 beside col2)
         unsigned w[4] = {1u, 1u, 1u, 1u};
-        if (a.w2 != nullptr && idx < end) {
+        if (WT && idx < end) {
           const int4 wv = ld_stream4((const int32_t*)a.w2 + it.start + idx);
           w[0] = (unsigned)wv.x; w[1] = (unsigned)wv.y; w[2] = (unsigned)wv.z; w[3] = (unsigned)wv.w;
         }
@@ -2286,7 +2288,7 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
           const int idx = base + (j * kGBlock + (int)threadIdx.x) * 4;
           const int4 u = idx < end ? ld_stream4(a.col + it.start + idx) : make_int4(-1, -1, -1, -1);
           int4 wv = make_int4(1, 1, 1, 1);
-          if (a.w2 != nullptr && idx < end) wv = ld_stream4((const int32_t*)a.w2 + it.start + idx);
+          if (WT && idx < end) wv = ld_stream4((const int32_t*)a.w2 + it.start + idx);
           wt[4 * j + 0] = (unsigned)wv.x; wt[4 * j + 1] = (unsigned)wv.y;
           wt[4 * j + 2] = (unsigned)wv.z; wt[4 * j + 3] = (unsigned)wv.w;
           lab[4 * j + 0] = gather_lv(a, u.x, use_v, gv[4 * j + 0]);
@@ -2301,7 +2303,7 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
           const int hot = __shfl_sync(kFull, cand0 == -2 ? lab[j] : cand0, 0);
           const unsigned m = __ballot_sync(kFull, vote && lab[j] == hot);
           unsigned c = vote ? (lab[j] != hot ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u)) : 0u;
-          if (a.w2 != nullptr) c = vote ? wt[j] : 0u;  // weighted: every arc adds its own weight
+          if (WT) c = vote ? wt[j] : 0u;  // weighted: every arc adds its own weight
           if (c) {
             bool fr = false;
             const unsigned cnt = giant_add(tab, tsz, (unsigned)lab[j], c, a.epoch, &fr);

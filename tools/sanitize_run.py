@@ -2,7 +2,9 @@
 racecheck / synccheck / initcheck): classic, seeded (sparse frontier, long
 push rows), LLP, forced W -> M -> L re-queues (debug_pred_cap), the L
 partition passes, giant rows, weighted, hybrid (host arcs) and a 2-rank local
-group.  Graphs are small so the sanitizers finish in minutes."""
+group; the W pair path (33-64-arc rows), the SEEDED presence filter and
+the weighted low / warp / block / giant kernels.  Graphs are small so the
+sanitizers finish in minutes."""
 import os, sys
 import numpy as np
 import torch
@@ -40,6 +42,12 @@ if which in ("all", "modes"):
         print(G.run("slp", 8, slp_max_labels=5, slp_threshold=0.1))
     with glp.Graph(hubs) as G:  # HT + CMS, small HT: sketch, rescans, fallbacks
         print(G.run("classic", 4, tail_cms=True, cms_ht_slots=256))
+    os.environ["GLP_LBITS"] = "1"  # SEEDED presence filter (normally only for label arrays beyond L2)
+    with glp.Graph(csr) as G:
+        print(G.run("seeded", 20, [1, 50, 900]))
+    with glp.Graph(hubs) as G:
+        print(G.run("seeded", 6, [0, 7, 2 * n_priv]))
+    del os.environ["GLP_LBITS"]
     os.environ["GLP_DEVICE_LOOP"] = "1"
     with glp.Graph(csr) as G:
         print(G.run("classic", 20)); print(G.run("seeded", 20, [1, 50, 900]))
