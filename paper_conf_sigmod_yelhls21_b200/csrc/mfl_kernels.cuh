@@ -2189,6 +2189,9 @@ __device__ __forceinline__ unsigned giant_add(unsigned long long* tab, unsigned 
 #ifndef GLP_GIANT_SMEM
 #define GLP_GIANT_SMEM 1
 #endif
+#ifndef GLP_GIANT_PRE_DIV
+#define GLP_GIANT_PRE_DIV 4ull  // pre-aggregate rows whose last distinct count is <= d / this (1: always)
+#endif
 constexpr int kGSlots = 8192;  // shared pre-aggregation table (64 KB)
 #ifndef GLP_G_MINB
 #define GLP_G_MINB 1  // 1: 56-64 registers, no spills (3: 32 registers + spills); A/B TaoBao 97.3 -> 94.2 ms/run, R24 17.51 -> 17.41
@@ -2217,7 +2220,8 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
     // rows predicted to repeat labels (last count <= d / 4: collapsed or
     // seeded hubs) pre-aggregate; distinct-heavy rows (t = 2, LLP's
     // oscillation) would only pay the shared insert and flush on top
-    const bool pre = GLP_GIANT_SMEM && (unsigned long long)(a.pred[sg.row] & kPredMask) * 4ull <= (unsigned long long)it.d;
+    const bool pre = GLP_GIANT_SMEM && (unsigned long long)(a.pred[sg.row] & kPredMask) * GLP_GIANT_PRE_DIV <=
+                                           (unsigned long long)it.d;
     if (pre) {
       const Table st{gsm, (unsigned)kGSlots};
       st.clear(threadIdx.x, kGBlock);

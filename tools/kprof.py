@@ -9,7 +9,7 @@ T = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 spec, variant, max_iters, gamma = bench.WORKLOADS[wl]
 csr, seeds = bench.make_graph(spec, 'cuda')
 torch.cuda.synchronize(); torch.cuda.empty_cache()
-g = glp.Graph(csr)
+g = glp.Graph(csr, weights=bench.workload_weights(wl, csr))
 info = g.run(variant, max_iters, seeds, gamma=gamma, profile=True)
 print(info)
 print({k['name']: round(k['ms'], 3) for k in g.kernel_stats() if k['launches']})

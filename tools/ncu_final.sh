@@ -2,7 +2,7 @@
 # ncu evidence for profiles/: (1) the launch list of the bench command,
 # (2) one --set full capture of every MFL launch of a whole R24 run,
 # summarised on the box (the report itself exceeds gpurun's copy-back limit).
-ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv --log-file gpurun_out/r2_ncu_launches_rmat24.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu > gpurun_out/r2_ncu_launches_bench.log 2>&1
+ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"mfl_|k_|glp" -c 3000 --csv --log-file gpurun_out/r2_ncu_launches_rmat24.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu > gpurun_out/r2_ncu_launches_bench.log 2>&1
 echo "launches rc=$?"
 ncu --set full --import-source on --clock-control none --profile-from-start off -k regex:mfl_ -o /tmp/r2_rmat24_full python tools/prof_it.py rmat24 20 > gpurun_out/r2_ncu_full.log 2>&1
 echo "full rc=$?"
