@@ -98,9 +98,6 @@ enum Variant { V_CLASSIC = 0, V_SEEDED = 1, V_LLP = 2 };
 #ifndef GLP_W_LOAD
 #define GLP_W_LOAD 4
 #endif
-#ifndef GLP_LLP_CTH
-#define GLP_LLP_CTH 0  // LLP observe: skip counts below ceil(best score) (Best::cth); A/B R28 LLP 3744 -> 4044 ms/run, R24 LLP 175.1 -> 176.6: off
-#endif
 
 __device__ __forceinline__ int ld_stream(const int32_t* p) {
   int r;
@@ -196,23 +193,13 @@ struct Best {
   unsigned long long key = 0ull;
   unsigned lab = kNoLabel;
   int bv = -1;  // LLP: V of the best label
-  // LLP: integer count threshold ceil(best score).  A label with V >= count
-  // scores at most its count (gamma >= 0), so a count below the threshold
-  // cannot reach the best score -- not even tie it -- and needs no double
-  // arithmetic.  (V < count only with repeated arcs: always scored.)
-  int cth = INT_MIN;
   // vl: V[l] when the caller has it (carried with the label, a.LV), else -1
   __device__ __forceinline__ void observe(unsigned cnt, unsigned l, const MflArgs& a, int vl = -1) {
     if (VAR == V_LLP) {
       // V of a permutation labelling is all ones (t = 1)
       const int v = vl >= 0 ? vl : (a.v_ones ? 1 : ld_label(a.V + l));
-      if (GLP_LLP_CTH && v >= (int)cnt && (int)cnt < cth) return;
-      const double sc = llp_score(cnt, v, a.gamma);
-      const unsigned long long k = dkey(sc);
-      if (k > key || (k == key && l < lab)) {
-        key = k; lab = l; bv = v;
-        if (GLP_LLP_CTH) cth = sc >= 2.0e9 ? INT_MAX : sc <= -2.0e9 ? INT_MIN : (int)ceil(sc);
-      }
+      const unsigned long long k = dkey(llp_score(cnt, v, a.gamma));
+      if (k > key || (k == key && l < lab)) { key = k; lab = l; bv = v; }
     } else {
       const unsigned long long k = ((unsigned long long)cnt << 32) | (unsigned long long)(~l);
       key = k > key ? k : key;
@@ -408,15 +395,6 @@ struct Cms {
 #ifndef GLP_LEAN
 #define GLP_LEAN 1
 #endif
-#ifndef GLP_HOTK
-#define GLP_HOTK 1
-#endif
-#ifndef GLP_LEAN2
-#define GLP_LEAN2 0
-#endif
-#ifndef GLP_HINT
-#define GLP_HINT 0  // A/B: R24 17.23 -> 17.21, SBM 5.28 -> 5.49, LLP 176.9 -> 174.7 ms/run (not kept)
-#endif
 #ifndef GLP_LEAN_PEEK
 #define GLP_LEAN_PEEK 0  // A/B (R24 ms/run): 0 17.29, 1 17.27, 2 17.72, 3 17.80; LLP 174.5 / 182.6 / 180.4 / 174.5.  0 never, 1 always, 2 rows predicted to repeat labels, 3 = 2 but not LLP
 #endif
@@ -457,58 +435,6 @@ __device__ __forceinline__ unsigned lean_insert4(const MflArgs& a, const Table& 
   cswap(q0, q2, v0, v2);
   cswap(q1, q3, v1, v3);
   cswap(q1, q2, v1, v2);
-#if GLP_LEAN2
-  // two heads (q0, q1) probe per trip with independent CAS / add chains (twice
-  // the shared-memory operations in flight per lane); q2, q3 queue behind them
-  unsigned fresh = 0u, npa = 0u, npb = 0u;
-  unsigned ha = slot_hash((unsigned)q0, t.tsz), hb = slot_hash((unsigned)q1, t.tsz);
-  const unsigned mask = t.tsz - 1u;
-  while (__any_sync(kFull, (q0 & q1) >= 0 || q0 >= 0 || q1 >= 0)) {
-    const bool ia = q0 >= 0, ib = q1 >= 0;
-    unsigned ka = 0u, kb = 0u;
-    if (ia) ka = atomicCAS(t.key + ha, kFree, (unsigned)q0);
-    if (ib) kb = atomicCAS(t.key + hb, kFree, (unsigned)q1);
-    const bool hita = ia && (ka == kFree || ka == (unsigned)q0);
-    const bool hitb = ib && (kb == kFree || kb == (unsigned)q1);
-    unsigned ca = 0u, cb = 0u;
-    if (hita) ca = atomicAdd(t.cnt + ha, 1u) + 1u;
-    if (hitb) cb = atomicAdd(t.cnt + hb, 1u) + 1u;
-    fresh += (hita && ka == kFree ? 1u : 0u) + (hitb && kb == kFree ? 1u : 0u);
-    if (obs) {
-      if (hita) b.observe(ca, (unsigned)q0, a, (kV && use_v) ? v0 : -1);
-      if (hitb) b.observe(cb, (unsigned)q1, a, (kV && use_v) ? v1 : -1);
-    }
-    bool fa = hita, fb = hitb;
-    if (ia && !hita) {
-      if (++npa >= max_probe) {
-        if (cms) { cms->add((unsigned)q0, 1u); fa = true; }
-        else { flag_set(overflow); q0 = q1 = q2 = q3 = -1; continue; }
-      } else {
-        ha = (ha + 1u) & mask;
-      }
-    }
-    if (ib && !hitb) {
-      if (++npb >= max_probe) {
-        if (cms) { cms->add((unsigned)q1, 1u); fb = true; }
-        else { flag_set(overflow); q0 = q1 = q2 = q3 = -1; continue; }
-      } else {
-        hb = (hb + 1u) & mask;
-      }
-    }
-    if (fa) {
-      q0 = q2; q2 = q3; q3 = -1;
-      if (kV) { v0 = v2; v2 = v3; }
-      ha = slot_hash((unsigned)q0, t.tsz);
-      npa = 0u;
-    }
-    if (fb) {
-      q1 = q2; q2 = q3; q3 = -1;
-      if (kV) { v1 = v2; v2 = v3; }
-      hb = slot_hash((unsigned)q1, t.tsz);
-      npb = 0u;
-    }
-  }
-#else
   unsigned fresh = 0u, np = 0u;
   unsigned h = slot_hash((unsigned)q0, t.tsz);
   const unsigned mask = t.tsz - 1u;
@@ -549,7 +475,6 @@ __device__ __forceinline__ unsigned lean_insert4(const MflArgs& a, const Table& 
       }
     }
   }
-#endif
   return fresh;
 }
 
@@ -557,8 +482,7 @@ template <int VAR, int N>
 __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table& t, unsigned max_probe,
                                                   const int (&labin)[N], Best<VAR>& b, volatile int* overflow,
                                                   const int (&vin)[N], bool use_v, bool hot_ok = true,
-                                                  const Cms* cms = nullptr, bool peek = false, int hint = -1,
-                                                  int hintv = -1) {
+                                                  const Cms* cms = nullptr, bool peek = false) {
   // use_v (LLP with a.LV): labels carry their V, so LLP observes at insert
   // like CLASSIC; otherwise LLP scores from the final table (table_scan)
   const bool obs = VAR != V_LLP || use_v;
@@ -567,52 +491,14 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
 #pragma unroll
   for (int j = 0; j < N; ++j) lab[j] = labin[j];
   unsigned nfresh = 0;
-  // hot candidate: the lane's best so far, else the hint (the vertex's own
-  // label L_{t-1}[v], the row's MFL of the last iteration: GLP_HINT), else
-  // the lane's first label of this batch
-  int cand = b.have() ? (int)b.label() : (GLP_HINT ? hint : -1);
-  int candv = b.have() ? b.bv : (GLP_HINT ? hintv : -1);
+  // hot candidate: the lane's best so far, else its first label of this batch
+  int cand = b.have() ? (int)b.label() : -1;
+  int candv = b.have() ? b.bv : -1;
 #pragma unroll
   for (int j = N - 1; j >= 0; --j) {
     candv = (cand < 0 && lab[j] >= 0) ? (use_v ? vin[j] : -1) : candv;
     cand = (cand < 0 && lab[j] >= 0) ? lab[j] : cand;
   }
-#if GLP_HOTK > 1
-  // GLP_HOTK hot labels: the candidates of lanes 0..K-1 (duplicates dropped);
-  // every lane counts its copies of each, K warp sums, then lane c inserts
-  // candidate c with its sum -- the K single-lane inserts in one instruction
-  if (hot_ok && GLP_MATCH_INSERT != 2) {
-    int hk[GLP_HOTK];
-    unsigned mytot = 0u;
-    int mine = -1, minev = -1;
-#pragma unroll
-    for (int c = 0; c < GLP_HOTK; ++c) {
-      hk[c] = __shfl_sync(kFull, cand, c);
-      const int hv = __shfl_sync(kFull, candv, c);
-#pragma unroll
-      for (int e = 0; e < c; ++e) hk[c] = hk[c] == hk[e] ? -1 : hk[c];
-      if (hk[c] >= 0) {  // warp-uniform
-        unsigned hc = 0;
-#pragma unroll
-        for (int j = 0; j < N; ++j) {
-          hc += lab[j] == hk[c] ? 1u : 0u;
-          lab[j] = lab[j] == hk[c] ? -1 : lab[j];
-        }
-        const unsigned tot = __reduce_add_sync(kFull, hc);
-        if (lane == c) { mytot = tot; mine = hk[c]; minev = hv; }
-      }
-    }
-    if (mytot) {
-      const unsigned cnt = ht_add(t, (unsigned)mine, mytot, max_probe, &nfresh);
-      if (cnt == 0u) {
-        if (cms) cms->add((unsigned)mine, mytot);
-        else flag_set(overflow);
-      } else if (obs) {
-        b.observe(cnt, (unsigned)mine, a, minev);
-      }
-    }
-  }
-#else
   const int hot = (hot_ok && GLP_MATCH_INSERT != 2) ? __shfl_sync(kFull, cand, 0) : -1;
   const int hotv = __shfl_sync(kFull, candv, 0);
   if (hot >= 0) {  // warp-uniform
@@ -633,7 +519,6 @@ __device__ __forceinline__ unsigned warp_insert_n(const MflArgs& a, const Table&
       }
     }
   }
-#endif
 #if GLP_LEAN && !GLP_MATCH_INSERT
 #pragma unroll
   for (int j0 = 0; j0 < N; j0 += 4)
@@ -994,9 +879,6 @@ __device__ __forceinline__ bool warp_quads_increasing(const int (&x)[4], int bas
 #ifndef GLP_W_SORT
 #define GLP_W_SORT 1
 #endif
-#ifndef GLP_W_PAIR_PIPE
-#define GLP_W_PAIR_PIPE 0  // pair p+1's labels and p+2's arcs in flight while pair p is sorted
-#endif
 #ifndef GLP_W_PAIR
 #define GLP_W_PAIR 1  // rows of <= 64 arcs: two per warp, sort-and-count per half (half_sort_count)
 #endif
@@ -1189,7 +1071,6 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
     BinItem mine;
     mine.start = 0; mine.v = 0; mine.d = 0;
     unsigned mpred = 0;
-    int mhint = -1, mhintv = -1;  // L_{t-1} of the row's vertex (and its V: LLP with LV)
     bool ok = il < a.n_items;
     if (ok) {
       mine = a.items[il];
@@ -1201,15 +1082,6 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       if (ok && !dense_ && !a.flag[a.vb + mine.v]) {
         ok = false;
         a.pred_next[il] = raw;  // inactive: carry the prediction forward
-      }
-      if (GLP_HINT && ok && !cand) {
-        if (VAR == V_LLP && a.LV != nullptr) {
-          const int2 x = __ldg(a.LV + a.vb + mine.v);
-          mhint = x.x;
-          mhintv = x.y;
-        } else {
-          mhint = ld_label(a.R + a.vb + mine.v);
-        }
       }
     }
     unsigned todo = __ballot_sync(kFull, ok);
@@ -1251,8 +1123,8 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           v[4 * q + 2] = gather(a, u[q].z); v[4 * q + 3] = gather(a, u[q].w);
         }
       };
-      // software pipeline over pairs: the arcs of pair p+2 and the labels of
-      // pair p+1 are in flight while pair p is sorted (GLP_W_PAIR_PIPE)
+      // the arcs of pair p+1 are loaded ahead (a software pipeline that also
+      // gathered pair p+1's labels during pair p's sort measured no gain)
       int ja0, jb0, ja1, jb1;
       int4 u0[K / 4], u1[K / 4];
       int v0[K];
@@ -1265,11 +1137,6 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
         int ja2, jb2;
         int4 u2[K / 4];
         int v1[K];
-        if (GLP_W_PAIR_PIPE) {
-          pop(ja2, jb2);
-          load_pair(ja2, jb2, u2);
-          gather_pair(u1, v1);
-        }
         Best<VAR> b;
         unsigned fr = half_sort_count<VAR, K>(v0, a, b);
 #pragma unroll
@@ -1290,11 +1157,9 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           rscan = mine.d;
           rpred = max(isa ? fa : fb, 1u);
         }
-        if (!GLP_W_PAIR_PIPE) {
-          pop(ja2, jb2);
-          load_pair(ja2, jb2, u2);
-          gather_pair(u1, v1);
-        }
+        pop(ja2, jb2);
+        load_pair(ja2, jb2, u2);
+        gather_pair(u1, v1);
         ja0 = ja1; jb0 = jb1; ja1 = ja2; jb1 = jb2;
 #pragma unroll
         for (int q = 0; q < K; ++q) v0[q] = v1[q];
@@ -1336,7 +1201,6 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
       const unsigned tsz =
           min(max(64u, 1u << (32 - __clz(GLP_W_LOAD * max(pred & kPredMask, 1u) - 1u))), (unsigned)kWSlots);
       const Table tab{wtabs + (size_t)wid * kWSlots, tsz};
-      const int hint = __shfl_sync(kFull, mhint, jl), hintv = __shfl_sync(kFull, mhintv, jl);
       // rows of <= 128 arcs predicted mostly distinct: sort-and-count, no table
       const bool wsort = GLP_W_SORT && d <= GLP_W_SORT_MAX && !(pred & kMonoTried) && 4u * (pred & kPredMask) > (unsigned)d;
       if (!wsort) tab.clear(lane, 32);
@@ -1399,7 +1263,7 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
             m8[2] = gather_lv(a, v0.z, use_v, mv8[2]); m8[3] = gather_lv(a, v0.w, use_v, mv8[3]);
             m8[4] = gather_lv(a, v1.x, use_v, mv8[4]); m8[5] = gather_lv(a, v1.y, use_v, mv8[5]);
             m8[6] = gather_lv(a, v1.z, use_v, mv8[6]); m8[7] = gather_lv(a, v1.w, use_v, mv8[7]);
-            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v, hot, nullptr, pk, hint, hintv);
+            fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, m8, b, &s_over[wid], mv8, use_v, hot, nullptr, pk);
           }
         }
         if (wsort) {  // the whole row is this round (d <= kWRound)
@@ -1417,11 +1281,11 @@ __global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
           break;
         }
         if (kWRound == 256 && d - off > 128) {  // warp-uniform
-          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v, hot, nullptr, pk, hint, hintv);
+          fresh += warp_insert_n<VAR, 8>(a, tab, kTabProbe, l, b, &s_over[wid], lv, use_v, hot, nullptr, pk);
         } else {
           const int l4[4] = {l[0], l[1], l[2], l[3]};
           const int v4[4] = {lv[0], lv[1], lv[2], lv[3]};
-          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v, hot, nullptr, pk, hint, hintv);
+          fresh += warp_insert_n<VAR, 4>(a, tab, kTabProbe, l4, b, &s_over[wid], v4, use_v, hot, nullptr, pk);
         }
         __syncwarp();
         over = warp_flag(&s_over[wid]);
@@ -1584,8 +1448,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
                                             unsigned max_probe, int4 (&u)[UNROLL], int32_t* stage_out,
                                             volatile int* overflow, int* distinct, Best<VAR>& b,
                                             volatile int* major, unsigned fparts = 1u, int* scanned = nullptr,
-                                            bool hot = true, const Cms* cms = nullptr, bool peek = false,
-                                            int hint = -1, int hintv = -1) {
+                                            bool hot = true, const Cms* cms = nullptr, bool peek = false) {
   constexpr int STEP = BLOCK * 4 * UNROLL;
   unsigned fresh = 0;
   int base = 0;
@@ -1614,7 +1477,7 @@ __device__ __forceinline__ void block_count(const MflArgs& a, int64_t start, int
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) u[j] = un[j];
     }
-    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot, cms, peek, hint, hintv);
+    fresh += warp_insert_n<VAR, 4 * UNROLL>(a, tab, max_probe, lab, b, overflow, lv, use_v, hot, cms, peek);
     if (GLP_MAJORITY && VAR != V_LLP && major != nullptr && base + STEP < d) {
       // a strict-majority observation ends the row for every warp (they poll the flag)
       const bool m = strict_majority(b, d);
@@ -1868,7 +1731,6 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
   __shared__ int s_k0, s_nsel, s_sel[32], s_cand[32];
   __shared__ BinItem s_item[32];
   __shared__ unsigned s_pe[32], s_raw[32];
-  __shared__ int s_hint[32], s_hintv[32];
   const int n_redo = a.mode ? (int)*a.redo_in_n : 0;
   const int lim = a.mode ? n_redo : a.n_items;
   for (;;) {
@@ -1912,18 +1774,6 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       const unsigned m = __ballot_sync(kFull, ok);
       if (ok) {
         const int pos = __popc(m & ((1u << threadIdx.x) - 1u));
-        int hn = -1, hv = -1;  // L_{t-1} of the row's vertex: the first hot label (GLP_HINT)
-        if (GLP_HINT && !cnd) {
-          if (VAR == V_LLP && a.LV != nullptr) {
-            const int2 x = __ldg(a.LV + a.vb + itk.v);
-            hn = x.x;
-            hv = x.y;
-          } else {
-            hn = ld_label(a.R + a.vb + itk.v);
-          }
-        }
-        s_hint[pos] = hn;
-        s_hintv[pos] = hv;
         s_sel[pos] = ik;
         s_item[pos] = itk;
         s_pe[pos] = pe;
@@ -1996,7 +1846,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
       block_count<VAR, BLOCK, UNROLL, !PART || GLP_L_IPF>(a, it.start, d, tab, may_over ? kLProbe : (PART ? tsz : kTabProbe), cur,
                                       (GLP_L_STAGE1 && may_over) ? stageA : nullptr, &s_over, &s_distinct, b,
                                       (may_over && !GLP_L_MAJ) ? nullptr : &s_major, 1u, &s_scan,
-                                      hot_pass(est, d), nullptr, peek_pass<VAR>(est, d), s_hint[q], s_hintv[q]);
+                                      hot_pass(est, d), nullptr, peek_pass<VAR>(est, d));
       __syncthreads();
       over = s_over != 0;
       if (!over && a.LV == nullptr) table_scan<VAR>(tab, threadIdx.x, BLOCK, a, b);
@@ -2037,8 +1887,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
             if (gather_pass) {
               block_load_round<BLOCK, UNROLL>(a.col, it.start, d, 0, cur);
               block_count<VAR, BLOCK, UNROLL, GLP_L_IPF>(a, it.start, d, tab, kLProbe, cur, stageA, &s_over,
-                                                         &s_distinct, b, nullptr, nparts, nullptr, GLP_HOT_DIV == 0,
-                                                         nullptr, false, s_hint[q], s_hintv[q]);
+                                                         &s_distinct, b, nullptr, nparts, nullptr, GLP_HOT_DIV == 0);
             } else {
               count_staged<VAR, BLOCK>(a, stageA, d, tab, kLProbe, &s_over, &s_distinct, b, nparts, p);
             }
