@@ -2038,6 +2038,9 @@ __device__ __forceinline__ unsigned giant_add(unsigned long long* tab, unsigned 
 #ifndef GLP_GIANT_SMEM
 #define GLP_GIANT_SMEM 1
 #endif
+#ifndef GLP_GIANT_BATCH
+#define GLP_GIANT_BATCH 1  // giant count: first probes of a lane's labels in flight together
+#endif
 #ifndef GLP_GIANT_PRE_DIV
 #define GLP_GIANT_PRE_DIV 4ull  // pre-aggregate rows whose last distinct count is <= d / this (1: always)
 #endif
@@ -2150,16 +2153,59 @@ __global__ void __launch_bounds__(kGBlock, GLP_G_MINB) mfl_giant_count(MflArgs a
           lab[4 * j + 3] = gather_lv(a, u.w, use_v, gv[4 * j + 3]);
         }
         const int cand0 = b.have() ? (int)b.label() : -2;
+        constexpr int NG = 4 * kGUnroll;
+        unsigned cc[NG];
 #pragma unroll
-        for (int j = 0; j < 4 * kGUnroll; ++j) {
+        for (int j = 0; j < NG; ++j) {
           const bool vote = lab[j] >= 0;
           const int hot = __shfl_sync(kFull, cand0 == -2 ? lab[j] : cand0, 0);
           const unsigned m = __ballot_sync(kFull, vote && lab[j] == hot);
           unsigned c = vote ? (lab[j] != hot ? 1u : (lane == __ffs(m) - 1 ? (unsigned)__popc(m) : 0u)) : 0u;
           if (WT) c = vote ? wt[j] : 0u;  // weighted: every arc adds its own weight
-          if (c) {
+          cc[j] = c;
+        }
+#if GLP_GIANT_BATCH
+        // The lane's NG inserts go to the row's table in L2 with their first
+        // probes in flight together (home-slot loads, then the adds on slots
+        // already holding the label and the claims of slots of older epochs,
+        // each batch independent); only labels whose home slot holds another
+        // label of this epoch, or whose claim lost a race, walk giant_add.
+        // LLP only (A/B: R28 LLP -4 %; classic / seeded +0.5-1 %).
+        if (VAR == V_LLP) {
+          constexpr int kShift = 31 + kGCountBits;
+          const unsigned long long keymask = ~((1ull << kGCountBits) - 1ull);
+          const unsigned long long cmask = (1ull << kGCountBits) - 1ull;
+          unsigned long long hh[NG], ee[NG];
+#pragma unroll
+          for (int j = 0; j < NG; ++j) {
+            hh[j] = (unsigned long long)(((unsigned)lab[j] * 0x9E3779B97F4A7C15ull) >> 20) & (tsz - 1ull);
+            ee[j] = cc[j] ? *((volatile unsigned long long*)(tab + hh[j])) : 0ull;
+          }
+#pragma unroll
+          for (int j = 0; j < NG; ++j) {
+            if (!cc[j]) continue;
+            const unsigned long long tag = (a.epoch << kShift) | ((unsigned long long)(unsigned)lab[j] << kGCountBits);
+            unsigned cnt = 0u;
+            if ((ee[j] & keymask) == tag) {
+              cnt = (unsigned)((atomicAdd(tab + hh[j], (unsigned long long)cc[j]) & cmask) + cc[j]);
+            } else if ((ee[j] >> kShift) != a.epoch) {
+              if (atomicCAS(tab + hh[j], ee[j], tag | cc[j]) == ee[j]) {
+                cnt = cc[j];
+                ++fresh;
+              }
+            }
+            if (cnt) {
+              b.observe(cnt, (unsigned)lab[j], a, use_v ? gv[j] : -1);
+              cc[j] = 0u;
+            }
+          }
+        }
+#endif
+#pragma unroll
+        for (int j = 0; j < NG; ++j) {
+          if (cc[j]) {
             bool fr = false;
-            const unsigned cnt = giant_add(tab, tsz, (unsigned)lab[j], c, a.epoch, &fr);
+            const unsigned cnt = giant_add(tab, tsz, (unsigned)lab[j], cc[j], a.epoch, &fr);
             fresh += fr ? 1u : 0u;
             b.observe(cnt, (unsigned)lab[j], a, use_v ? gv[j] : -1);
           }
