@@ -356,12 +356,17 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
   g->nnz2 = rows_base + padded_total;
   if (g->nnz2 >= ((int64_t)1 << 48)) fail(GLP_ERR_INVALID_ARGUMENT, "graph too large");
   g->n_gt256 = g->n_gt2048 = g->n_ge8k = g->n_gt512 = 0;
+  int64_t arcs_le64 = 0, arcs_rows = 0;
   for (const BinItem& it : row_i) {
+    arcs_le64 += it.d <= 64 ? it.d : 0;
+    arcs_rows += it.d;
     g->n_gt256 += it.d > 256;
     g->n_gt2048 += it.d > 2048;
     g->n_ge8k += it.d >= 8192;
     g->n_gt512 += it.d > kWtWarpMax;
   }
+  const char* wse = getenv("GLP_W_SHORT");  // A/B: 0 / 1 forces the W variant
+  g->w_short = wse ? wse[0] == '1' : 2 * arcs_le64 > arcs_rows;
   for (int k = 0; k < 3; ++k) g->pred[k] = dalloc<unsigned>(g, std::max<int64_t>(n_rows, 1));
   g->redo_m = dalloc<int32_t>(g, std::max<int64_t>(n_rows, 1));
   g->redo_l = dalloc<int32_t>(g, std::max<int64_t>(n_rows, 1));
@@ -750,7 +755,11 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     CK(cudaFuncSetAttribute(mfl_warp<V_CLASSIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
     CK(cudaFuncSetAttribute(mfl_warp<V_SEEDED>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
     CK(cudaFuncSetAttribute(mfl_warp<V_LLP>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
-    g->grid_w = grid_for(sms, (const void*)mfl_warp<V_LLP>, kWBlock, ws_);
+    CK(cudaFuncSetAttribute(mfl_warp<V_CLASSIC, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
+    CK(cudaFuncSetAttribute(mfl_warp<V_SEEDED, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
+    CK(cudaFuncSetAttribute(mfl_warp<V_LLP, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, ws_));
+    g->grid_w = g->w_short ? grid_for(sms, (const void*)mfl_warp<V_LLP, 3>, kWBlock, ws_)
+                           : grid_for(sms, (const void*)mfl_warp<V_LLP>, kWBlock, ws_);
     g->grid_m = grid_for(sms, (const void*)GLP_M_KERNEL(V_LLP), kMBlock, ms_);
     g->grid_mono = grid_for(sms, (const void*)mfl_mono<V_LLP>, kMonoBlock, 0);
     const int wtw_ = (kWtBlock / 32) * kWtWarpSlots * 8, wtb_ = kWtSlots * 8;
@@ -924,7 +933,10 @@ int launch_mfl(glp_graph* g, MflArgs a, bool prof, std::vector<Pending>& pend, s
     b.n_items = g->n_rows; b.cnt = c + 1; b.redo_out = g->redo_m; b.redo_out_n = &sc->n_redo_m;
     const int grid = std::min<int>(g->grid_w, (g->n_rows + kWBlock - 1) / kWBlock);
     timed(g, prof, 1, pend, used, s0,
-          [&] { mfl_warp<VAR><<<grid, kWBlock, (kWBlock / 32) * kWSlots * 8, s0>>>(b); });
+          [&] {
+            if (g->w_short) mfl_warp<VAR, 3><<<grid, kWBlock, (kWBlock / 32) * kWSlots * 8, s0>>>(b);
+            else mfl_warp<VAR><<<grid, kWBlock, (kWBlock / 32) * kWSlots * 8, s0>>>(b);
+          });
     ++n;
   }
   if (g->n_chunks) {

@@ -272,6 +272,7 @@ struct glp_graph {
   glp::BinItem* rows = nullptr; int32_t n_rows = 0;  // deg > 32, degree-descending
   int32_t n_gt256 = 0, n_gt2048 = 0;                 // prefixes with deg > 256 / > 2048
   int32_t n_ge8k = 0;                                // prefix with deg >= 8192
+  bool w_short = false;                              // W kernel at 3 blocks/SM (mostly <= 64-arc rows)
   int32_t n_giant = 0;                               // prefix with deg > kGiantMin
   glp::GiantSeg* gsegs = nullptr; int32_t n_gsegs = 0;
   unsigned long long* gtab = nullptr; int64_t gtab_slots = 0;

@@ -1054,11 +1054,14 @@ __device__ __forceinline__ void load_round(const int32_t* col, int64_t start, in
   if (kWRound == 256 && off + 128 + 4 * lane < d) u1 = ld_stream4(col + start + off + 128 + 4 * lane);
 }
 
-template <int VAR>
 #ifndef GLP_W_MINB
 #define GLP_W_MINB 4
 #endif
-__global__ void __launch_bounds__(kWBlock, GLP_W_MINB) mfl_warp(MflArgs a) {
+// MINB: resident blocks per SM.  4 (64 registers, the pair path spills) by
+// default; 3 (no spills) when most arcs of the deg > 32 rows are in rows of
+// <= 64 arcs (glp_graph::w_short: SBM -6 %, while R24 / LLP lose 1.3 % at 3)
+template <int VAR, int MINB = GLP_W_MINB>
+__global__ void __launch_bounds__(kWBlock, MINB) mfl_warp(MflArgs a) {
   GLP_CTL_PROLOGUE(a)
   extern __shared__ __align__(16) unsigned long long wtabs[];  // [kWBlock / 32][kWSlots] (dynamic)
   __shared__ int s_over[kWBlock / 32];
