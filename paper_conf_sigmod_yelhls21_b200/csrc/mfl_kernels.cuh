@@ -1735,6 +1735,7 @@ __global__ void __launch_bounds__(BLOCK, PART ? GLP_L_MINB : GLP_M_MINB) mfl_blo
   __shared__ BinItem s_item[32];
   __shared__ unsigned s_pe[32], s_raw[32];
   const int n_redo = a.mode ? (int)*a.redo_in_n : 0;
+  if (a.mode && n_redo == 0) return;  // empty redo queue (block-uniform): no tally to flush
   const int lim = a.mode ? n_redo : a.n_items;
   for (;;) {
     // dynamic fetch of 32 rows (row costs vary by orders of magnitude); warp 0
