@@ -442,13 +442,20 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
     CK(cudaMemsetAsync(g->col2, 0xff, std::max<int64_t>(g->nnz2, 1) * sizeof(int32_t), s));  // padding = -1
   }
   if (nl > 0 && g->nnz > 0) {
+    // rows past kRelayBig arcs: listed by k_relayout, copied by the grid
+    const int64_t big_cap = g->nnz / kRelayBig + 1;
+    int32_t* rbig = dalloc<int32_t>(g, big_cap + 1);
+    unsigned* rnbig = (unsigned*)(rbig + big_cap);
+    CK(cudaMemsetAsync(rnbig, 0, sizeof(unsigned), s));
     for (size_t c = 0; c + 1 < g->arc_chunks.size(); ++c) {
       if (c < g->arc_chunk_ev.size()) CK(cudaStreamWaitEvent(s, g->arc_chunk_ev[c], 0));
       else CK(cudaStreamWaitEvent(s, g->xev[1], 0));
       k_relayout<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, g->pos, g->arc_chunks[c], g->arc_chunks[c + 1], g->vb,
-                                    g->n, g->col2);
+                                    g->n, g->col2, rbig, rnbig);
       CK(cudaGetLastError());
     }
+    k_relayout_big<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, g->pos, g->vb, g->n, g->col2, rbig, rnbig);
+    CK(cudaGetLastError());
   }
   CK(cudaStreamWaitEvent(s, g->xev[1], 0));
   {
@@ -598,6 +605,13 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       }
       g->arc_chunks.push_back(g->nl);
     }
+    // GLP_TRACE_CREATE: time the arc copy on the side stream
+    cudaEvent_t tc0 = nullptr, tc1 = nullptr;
+    if (g_trace) {
+      CK(cudaEventCreate(&tc0));
+      CK(cudaEventCreate(&tc1));
+      CK(cudaEventRecord(tc0, g->xs[0]));
+    }
     for (size_t c = 0; c + 1 < g->arc_chunks.size(); ++c) {
       const int64_t a0 = csr->on_device || g->host_arcs ? 0 : csr->row_offsets[g->arc_chunks[c]];
       const int64_t a1 = csr->on_device || g->host_arcs ? g->nnz : csr->row_offsets[g->arc_chunks[c + 1]];
@@ -614,6 +628,16 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       }
     }
     CK(cudaEventRecord(g->xev[1], g->xs[0]));
+    if (g_trace) {
+      CK(cudaEventRecord(tc1, g->xs[0]));
+      CK(cudaEventSynchronize(tc1));
+      float cms = 0.f;
+      CK(cudaEventElapsedTime(&cms, tc0, tc1));
+      fprintf(stderr, "[glp create] arc copy + check on the side stream: %.2f ms (%.1f GB/s)\n", cms,
+              g->nnz * 4.0 / 1e6 / std::max(cms, 1e-3f));
+      cudaEventDestroy(tc0);
+      cudaEventDestroy(tc1);
+    }
     struct TempGuard {
       std::vector<void*>& v;
       cudaStream_t s;
