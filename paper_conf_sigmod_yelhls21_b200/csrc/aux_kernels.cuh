@@ -214,8 +214,23 @@ __global__ void k_relayout_w(const int64_t* __restrict__ off, const uint32_t* __
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t v = gw; v < nl; v += nw) {
-    const int64_t s = off[v], d = off[v + 1] - s, o = ioff[pos[vb + v] - vb];
+    const int64_t s = off[v], d = off[v + 1] - s;
+    if (d > kRelayBig) continue;  // listed by k_relayout: k_relayout_w_big
+    const int64_t o = ioff[pos[vb + v] - vb];
     for (int64_t j = lane; j < d; j += 32) w2[o + j] = w[s + j];
+  }
+}
+__global__ void k_relayout_w_big(const int64_t* __restrict__ off, const uint32_t* __restrict__ w,
+                                 const int64_t* __restrict__ ioff, const int32_t* __restrict__ pos, int64_t vb,
+                                 uint32_t* __restrict__ w2, const int32_t* __restrict__ big,
+                                 const unsigned* __restrict__ n_big) {
+  const unsigned nb = *n_big;
+  const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+  for (unsigned i = 0; i < nb; ++i) {
+    const int64_t v = big[i];
+    const int64_t s = off[v], d = off[v + 1] - s, o = ioff[pos[vb + v] - vb];
+    for (int64_t j = tid; j < d; j += nth) w2[o + j] = w[s + j];
   }
 }
 // weights in [1, 2^31) and every row's total < 2^31 (exact 32-bit sums)

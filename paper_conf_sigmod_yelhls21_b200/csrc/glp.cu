@@ -443,10 +443,16 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
   }
   if (nl > 0 && g->nnz > 0) {
     // rows past kRelayBig arcs: listed by k_relayout, copied by the grid
-    const int64_t big_cap = g->nnz / kRelayBig + 1;
-    int32_t* rbig = dalloc<int32_t>(g, big_cap + 1);
-    unsigned* rnbig = (unsigned*)(rbig + big_cap);
-    CK(cudaMemsetAsync(rnbig, 0, sizeof(unsigned), s));
+    int32_t* rbig = nullptr;
+    unsigned* rnbig = nullptr;
+    if (g->max_deg > kRelayBig) {
+      const int64_t big_cap = g->nnz / kRelayBig + 1;
+      rbig = dalloc<int32_t>(g, big_cap + 1);
+      rnbig = (unsigned*)(rbig + big_cap);
+      g->relay_big = rbig;
+      g->relay_nbig = rnbig;
+      CK(cudaMemsetAsync(rnbig, 0, sizeof(unsigned), s));
+    }
     for (size_t c = 0; c + 1 < g->arc_chunks.size(); ++c) {
       if (c < g->arc_chunk_ev.size()) CK(cudaStreamWaitEvent(s, g->arc_chunk_ev[c], 0));
       else CK(cudaStreamWaitEvent(s, g->xev[1], 0));
@@ -454,8 +460,10 @@ void build_layout(glp_graph* g, const int64_t* off_d, const int32_t* col_d) {
                                     g->n, g->col2, rbig, rnbig);
       CK(cudaGetLastError());
     }
-    k_relayout_big<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, g->pos, g->vb, g->n, g->col2, rbig, rnbig);
-    CK(cudaGetLastError());
+    if (rbig) {
+      k_relayout_big<<<gb, 256, 0, s>>>(off_d, col_d, g->ioff, g->pos, g->vb, g->n, g->col2, rbig, rnbig);
+      CK(cudaGetLastError());
+    }
   }
   CK(cudaStreamWaitEvent(s, g->xev[1], 0));
   {
@@ -607,7 +615,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
     }
     // GLP_TRACE_CREATE: time the arc copy on the side stream
     cudaEvent_t tc0 = nullptr, tc1 = nullptr;
-    if (g_trace) {
+    if (g_trace && g_trace->on) {
       CK(cudaEventCreate(&tc0));
       CK(cudaEventCreate(&tc1));
       CK(cudaEventRecord(tc0, g->xs[0]));
@@ -628,7 +636,7 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       }
     }
     CK(cudaEventRecord(g->xev[1], g->xs[0]));
-    if (g_trace) {
+    if (g_trace && g_trace->on) {
       CK(cudaEventRecord(tc1, g->xs[0]));
       CK(cudaEventSynchronize(tc1));
       float cms = 0.f;
@@ -692,6 +700,9 @@ void create_impl(const glp_csr* csr, const glp_dist* dist, const glp_params* prm
       if (g->nl && g->nnz) {
         k_validate_w<<<g->sms * 4, 256, 0, g->stream>>>(off_d, w_d, g->nl, dbad);
         k_relayout_w<<<g->sms * 8, 256, 0, g->stream>>>(off_d, w_d, g->ioff, g->pos, g->nl, g->vb, g->w2);
+        if (g->relay_big)
+          k_relayout_w_big<<<g->sms * 8, 256, 0, g->stream>>>(off_d, w_d, g->ioff, g->pos, g->vb, g->w2, g->relay_big,
+                                                             g->relay_nbig);
         CK(cudaGetLastError());
       }
       int bad = 0;

@@ -252,6 +252,8 @@ struct glp_graph {
   bool weighted = false;        // weighted LP: w2 holds the arc weights
   uint32_t* w2 = nullptr;       // [nnz2] weights beside col2 (padding 0)
   int32_t n_gt512 = 0;          // prefix of rows with deg > kWtWarpMax
+  int32_t* relay_big = nullptr;   // create: rows past kRelayBig arcs (listed by k_relayout)
+  unsigned* relay_nbig = nullptr;
   bool wt_low_off = false;      // weighted low rows in mfl_wt_warp (GLP_WT_LOW=0) instead of mfl_low
   bool wt_giant = false;        // weighted giant rows go to the segmented giant kernels (totals fit kGCountBits)
   void* col2_host = nullptr;    // its host allocation
