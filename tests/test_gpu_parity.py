@@ -415,3 +415,13 @@ def test_seeded_presence_filter_forced(case, monkeypatch):
     ref, lab, info, st = assert_same_run(csr, 1, 30, seeds=seeds)
     # the filter is on while at most half the vertices can be labelled
     assert info.iterations >= 2
+
+
+@pytest.mark.parametrize("short", ["0", "1"])
+def test_w_kernel_block_variants(short, monkeypatch):
+    """The W kernel at 4 or 3 blocks/SM (GLP_W_SHORT forces the choice made
+    from the graph's row lengths) gives the oracle's labels, on a graph with
+    both 33-64-arc rows (pair path) and longer W rows."""
+    monkeypatch.setenv("GLP_W_SHORT", short)
+    assert_same_run(graphs.sbm(n=60_000, k=60, m=1_500_000, seed=9), 0, 30)
+    assert_same_run(graphs.rmat(14, seed=6), 0, 20)
